@@ -1,0 +1,209 @@
+/*
+ * epi4_oracle.c — plain CPU oracle for the exhaustive fourth-order K2 epistasis search.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  It shares no code,
+ * header, table or constant generator with the CUDA path (paper_conf_icpp_nobreiss22_b200/),
+ * and it reads BYTE genotypes, never bit planes.
+ *
+ * What it computes is the plain definition; the passages followed:
+ *   PAPER.md:L47  (§2)   a fourth-order search finds the SNP quad most associated with the
+ *                        phenotype; each quad has 81 (3^4) genotypes, counted separately for
+ *                        cases and controls -> a 2 x 81 contingency table (162 values).
+ *   PAPER.md:L53-59, L143 (§2, §3.5)  Bayesian K2 score, sums of logarithms written as
+ *                        log-factorials via Gamma(x) = (x-1)!  (reading #1 in DESIGN.md):
+ *                        K2 = sum_{c=0}^{80} [ lgamma(r_c + 2) - lgamma(r_c0 + 1) - lgamma(r_c1 + 1) ],
+ *                        r_c = r_c0 + r_c1, natural log.
+ *   PAPER.md:L66   (§3.1) genotype codes: 0 = AA, 1 = Aa, 2 = aa.
+ *   PAPER.md:L74   (§3.2) a genotype count = number of samples having genotype (a,b,c,d) on the
+ *                        four SNPs (AND of 4 indicator vectors + POPC) — here: a per-sample loop.
+ *   PAPER.md:L109, L145 (§3.2, §3.5) output = best quad + score; a quad index is packed into 64 bits
+ *                        as 4 x 16-bit SNP indices.
+ *   PAPER.md:L268  (§4.5) combinations (i<j<k<l), not permutations.
+ * Readings fixed by DESIGN.md: #2 best = argmin K2; #3 ties -> the
+ * lexicographically smallest quad (= smallest packed index); #4 K2 accumulated in double in
+ * canonical cell order c = 27a + 9b + 3c + d, t = (L(r+1) - L(r0)) - L(r1), K2 += t, with
+ * L(n) = lgamma(n + 1.0) from glibc; #14 top-k = the k smallest (K2, index) keys, ascending.
+ *
+ * Pins (tests/test_oracle.py): hand-enumerated dataset (K2 = log 576), closed forms, cell sums
+ * equal n0/n1, 4-way -> 3-way/2-way marginalisation vs a separately written numpy brute force,
+ * planted-interaction recovery, brute-force top-k on tiny inputs, duplicated-SNP exact ties.
+ */
+#define _GNU_SOURCE
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define NCELL 81
+
+/* L(n) = log(n!) = lgamma(n + 1)  (Gamma(x) = (x-1)!) */
+static double log_factorial(uint32_t n) {
+    int sign;
+    return lgamma_r((double)n + 1.0, &sign);
+}
+
+/* K2 of one 2 x 81 table, r[0..80] = controls, r[81..161] = cases (reading #1/#4). */
+double oracle_k2(const uint32_t *r) {
+    double k2 = 0.0;
+    for (int c = 0; c < NCELL; ++c) {
+        uint32_t r0 = r[c], r1 = r[NCELL + c];
+        double t = (log_factorial(r0 + r1 + 1) - log_factorial(r0)) - log_factorial(r1);
+        k2 = k2 + t;
+    }
+    return k2;
+}
+
+/* packed quad index: i<<48 | j<<32 | k<<16 | l */
+uint64_t oracle_pack(int32_t i, int32_t j, int32_t k, int32_t l) {
+    return ((uint64_t)(uint16_t)i << 48) | ((uint64_t)(uint16_t)j << 32) |
+           ((uint64_t)(uint16_t)k << 16) | (uint64_t)(uint16_t)l;
+}
+
+/* 2 x 81 table of one quad by a per-sample loop.
+ * geno: N x M SNP-major bytes, phen: M bytes (0 control / 1 case). */
+static void count_quad(const uint8_t *geno, const uint8_t *phen, int64_t m,
+                       int32_t i, int32_t j, int32_t k, int32_t l, uint32_t *r) {
+    const uint8_t *gi = geno + (int64_t)i * m, *gj = geno + (int64_t)j * m;
+    const uint8_t *gk = geno + (int64_t)k * m, *gl = geno + (int64_t)l * m;
+    memset(r, 0, sizeof(uint32_t) * 2 * NCELL);
+    for (int64_t s = 0; s < m; ++s) {
+        int cell = 27 * gi[s] + 9 * gj[s] + 3 * gk[s] + gl[s];
+        r[phen[s] * NCELL + cell] += 1;
+    }
+}
+
+static int validate(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m) {
+    if (n < 4 || n > 65536 || m < 1) return -1;
+    for (int64_t s = 0; s < m; ++s) if (phen[s] > 1) return -2;
+    for (int64_t x = 0; x < (int64_t)n * m; ++x) if (geno[x] > 2) return -3;
+    return 0;
+}
+
+/* Tables for an explicit list of quads (any order of the 4 indices is accepted and used as given:
+ * cell = 27 g[q0] + 9 g[q1] + 3 g[q2] + g[q3]).  counts: nq x 2 x 81. */
+int oracle_tables(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m,
+                  const int32_t *quads, int64_t nq, uint32_t *counts, int32_t n_threads) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    for (int64_t q = 0; q < nq; ++q)
+        for (int t = 0; t < 4; ++t)
+            if (quads[4 * q + t] < 0 || quads[4 * q + t] >= n) return -4;
+#ifdef _OPENMP
+    if (n_threads > 0) omp_set_num_threads(n_threads);
+#pragma omp parallel for schedule(dynamic, 16)
+#endif
+    for (int64_t q = 0; q < nq; ++q)
+        count_quad(geno, phen, m, quads[4 * q], quads[4 * q + 1], quads[4 * q + 2], quads[4 * q + 3],
+                   counts + q * 2 * NCELL);
+    return 0;
+}
+
+/* K2 for an explicit list of quads. */
+int oracle_score(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m,
+                 const int32_t *quads, int64_t nq, double *k2_out, int32_t n_threads) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+#ifdef _OPENMP
+    if (n_threads > 0) omp_set_num_threads(n_threads);
+#pragma omp parallel for schedule(dynamic, 16)
+#endif
+    for (int64_t q = 0; q < nq; ++q) {
+        uint32_t r[2 * NCELL];
+        count_quad(geno, phen, m, quads[4 * q], quads[4 * q + 1], quads[4 * q + 2], quads[4 * q + 3], r);
+        k2_out[q] = oracle_k2(r);
+    }
+    return 0;
+}
+
+/* key order: (K2, packed index) lexicographic (readings #2, #3) */
+static int key_less(double ka, uint64_t ia, double kb, uint64_t ib) {
+    return ka < kb || (ka == kb && ia < ib);
+}
+
+/* insert into a sorted list of capacity cap holding *len entries */
+static void topk_insert(double *k2, uint64_t *idx, int32_t *len, int32_t cap, double kv, uint64_t iv) {
+    int32_t n = *len;
+    if (n == cap && !key_less(kv, iv, k2[n - 1], idx[n - 1])) return;
+    int32_t p = (n < cap) ? n : cap - 1;
+    while (p > 0 && key_less(kv, iv, k2[p - 1], idx[p - 1])) {
+        k2[p] = k2[p - 1];
+        idx[p] = idx[p - 1];
+        --p;
+    }
+    k2[p] = kv;
+    idx[p] = iv;
+    if (n < cap) *len = n + 1;
+}
+
+/* Exhaustive search over every quad i<j<k<l of SNPs [0, n).
+ * Returns the top_k smallest (K2, packed index) keys, ascending; *n_out = min(top_k, C(n,4)). */
+int oracle_search(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m, int32_t top_k,
+                  uint64_t *idx_out, double *k2_out, int32_t *n_out, int32_t n_threads) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    if (top_k < 1) return -5;
+    int64_t npairs = (int64_t)n * (n - 1) / 2;
+    int32_t nthr = 1;
+#ifdef _OPENMP
+    if (n_threads > 0) omp_set_num_threads(n_threads);
+    nthr = omp_get_max_threads();
+#endif
+    double *tk = (double *)malloc(sizeof(double) * (size_t)top_k * nthr);
+    uint64_t *ti = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)top_k * nthr);
+    int32_t *tl = (int32_t *)calloc(nthr, sizeof(int32_t));
+    if (!tk || !ti || !tl) { free(tk); free(ti); free(tl); return -6; }
+#ifdef _OPENMP
+#pragma omp parallel
+#endif
+    {
+        int32_t tid = 0;
+#ifdef _OPENMP
+        tid = omp_get_thread_num();
+#endif
+        double *mk = tk + (size_t)tid * top_k;
+        uint64_t *mi = ti + (size_t)tid * top_k;
+        uint32_t r[2 * NCELL];
+#ifdef _OPENMP
+#pragma omp for schedule(dynamic, 1)
+#endif
+        for (int64_t p = 0; p < npairs; ++p) {
+            /* p -> (i, j), i < j, lexicographic */
+            int32_t i = 0;
+            int64_t rem = p;
+            while (rem >= n - 1 - i) { rem -= n - 1 - i; ++i; }
+            int32_t j = i + 1 + (int32_t)rem;
+            for (int32_t k = j + 1; k < n; ++k)
+                for (int32_t l = k + 1; l < n; ++l) {
+                    count_quad(geno, phen, m, i, j, k, l, r);
+                    topk_insert(mk, mi, &tl[tid], top_k, oracle_k2(r), oracle_pack(i, j, k, l));
+                }
+        }
+    }
+    /* deterministic merge of the per-thread lists */
+    int32_t len = 0;
+    double *fk = (double *)malloc(sizeof(double) * top_k);
+    uint64_t *fi = (uint64_t *)malloc(sizeof(uint64_t) * top_k);
+    for (int32_t t = 0; t < nthr; ++t)
+        for (int32_t e = 0; e < tl[t]; ++e)
+            topk_insert(fk, fi, &len, top_k, tk[(size_t)t * top_k + e], ti[(size_t)t * top_k + e]);
+    memcpy(k2_out, fk, sizeof(double) * len);
+    memcpy(idx_out, fi, sizeof(uint64_t) * len);
+    *n_out = len;
+    free(fk); free(fi); free(tk); free(ti); free(tl);
+    return 0;
+}
+
+/* threads the OpenMP runtime will use (for the cpu_baseline "cores" field) */
+int32_t oracle_max_threads(int32_t n_threads) {
+#ifdef _OPENMP
+    if (n_threads > 0) omp_set_num_threads(n_threads);
+    return omp_get_max_threads();
+#else
+    (void)n_threads;
+    return 1;
+#endif
+}
