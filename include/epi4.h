@@ -1,0 +1,143 @@
+/*
+ * epi4.h — C ABI of libepi4, the B200 (sm_100a) exhaustive fourth-order K2 epistasis search.
+ *
+ * The boundary of the hot path.  Plain C types only: no torch types, host or
+ * device pointers plus sizes.  Every step of the search runs in libepi4's CUDA kernels; the thin
+ * Python binding (paper_conf_icpp_nobreiss22_b200/binding.py) only marshals arguments.
+ *
+ * Notation (repo naming; PAPER.md swaps the symbols):
+ *   N  = number of SNPs (PAPER.md's M), 4 <= N <= 65536 (16-bit SNP indices)
+ *   n0 = controls, n1 = cases, M = n0 + n1 samples (PAPER.md's N0, N1, N).
+ *
+ * Errors: every int-returning call returns 0 on success or a negative EPI4_E* code; the message
+ * of the last failure on the calling thread is available from epi4_last_error().  No call
+ * throws, aborts or exits across the ABI.
+ *
+ * Threading: a context is used by one host thread at a time.  One context per GPU / rank.
+ */
+#ifndef EPI4_H
+#define EPI4_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- error codes ---------------------------------------------------------------------- */
+#define EPI4_OK       0
+#define EPI4_EINVAL  (-1)  /* bad argument: N<4 or N>65536, n_controls<1 or n_cases<1, top_k out of
+                              range, pad bits set, AA&Aa != 0, genotype code > 2, phenotype > 1 */
+#define EPI4_ENOMEM  (-2)  /* device or host allocation failed (incl. tables too large for HBM) */
+#define EPI4_ECUDA   (-3)  /* a CUDA runtime call or kernel failed */
+#define EPI4_ESTATE  (-4)  /* call out of order, e.g. search before any load */
+#define EPI4_ENODEV  (-5)  /* no sm_100 device / the requested device is unusable */
+
+/* ---- options ---------------------------------------------------------------------------- */
+#define EPI4_PIPE_I8TC  0  /* tcgen05.mma kind::i8 on {0,1}-expanded tiles, TMEM accumulators */
+#define EPI4_PIPE_LOP3  1  /* CUDA-core LOP3 (AND) + POPC contraction (cross-check path) */
+
+#define EPI4_PTR_HOST   0
+#define EPI4_PTR_DEVICE 1
+
+#define EPI4_MAX_TOPK   1024
+
+typedef struct epi4_ctx epi4_ctx;   /* opaque; owns its device memory and CUDA stream */
+
+typedef struct {
+    int32_t block;    /* SNP block size B.  Only 32 is supported.            */
+    int32_t pipe;     /* EPI4_PIPE_*                                                               */
+    int32_t rank;     /* this process' rank and the world size: epi4_search evaluates only the     */
+    int32_t world;    /*   work units the static LPT plan assigns to `rank`       */
+    int32_t grid;     /* persistent-kernel CTAs (0 = 2 x number of SMs)                             */
+    int32_t reserved[3];
+} epi4_opts;
+
+/* Fill *opts with defaults (block 32, pipe I8TC, rank 0, world 1, grid 0). */
+void epi4_default_opts(epi4_opts* opts);
+
+/* Create a context on CUDA device `cuda_device` (selects it on the calling thread).
+ * opts may be NULL (defaults).  *out receives the context; destroy it with epi4_destroy. */
+int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts);
+void epi4_destroy(epi4_ctx* ctx);
+
+/* Use `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream().cuda_stream) for all later
+ * work of this context; NULL restores the context's own stream. */
+int epi4_set_stream(epi4_ctx* ctx, void* cuda_stream);
+
+/* ---- data loading (step a1 of SURVEY.md §8(a); §3.1) --------------------------
+ * Bit-packed genotype planes, one matrix per phenotype: row r = 2*snp + g with
+ * g = 0 -> AA (homozygous major), g = 1 -> Aa (heterozygous); aa is not stored (inferred).
+ * Each row holds ceil(n/32) uint32 words, sample s of that phenotype at bit s%32 of word s/32
+ * (LSB first).  Pad bits beyond n must be 0 and AA & Aa must be 0 (checked -> EPI4_EINVAL).
+ * The data is copied (the caller keeps ownership).  ptr_kind selects host or device pointers. */
+int epi4_load_bits(epi4_ctx* ctx, const uint32_t* planes_ctrl, const uint32_t* planes_case,
+                   int32_t n_snps, int64_t n_controls, int64_t n_cases, int32_t ptr_kind);
+
+/* Same, from byte genotypes: geno is N x M, SNP-major, codes {0 = AA, 1 = Aa, 2 = aa};
+ * phen[M] is 0 (control) or 1 (case).  The split by phenotype and the bit packing run on the GPU
+ * (the pack kernel).  Codes > 2 or phenotypes > 1 -> EPI4_EINVAL. */
+int epi4_pack_genotypes(epi4_ctx* ctx, const uint8_t* geno, const uint8_t* phen,
+                        int32_t n_snps, int64_t n_samples, int32_t ptr_kind);
+
+/* Copy the packed planes back (host pointers, sized 2*N*ceil(n_p/32) words each). */
+int epi4_get_bits(epi4_ctx* ctx, uint32_t* planes_ctrl, uint32_t* planes_case);
+
+/* ---- search (steps a2-a7; Algorithm 1, L109 output s) ------------------------
+ * Exhaustive search over every quad i<j<k<l assigned to this rank.  Writes the `top_k` smallest
+ * (K2, quad) keys in ascending order (ties -> smaller packed index), K2 in double
+ * (readings #1-#4).  Packed quad index:
+ * i<<48 | j<<32 | k<<16 | l.  quads_out / k2_out are HOST arrays of top_k entries; *n_out gets
+ * min(top_k, number of quads evaluated).  1 <= top_k <= EPI4_MAX_TOPK. */
+int epi4_search(epi4_ctx* ctx, int32_t top_k, uint64_t* quads_out, double* k2_out, int32_t* n_out);
+
+/* Search restricted to the work units [unit_begin, unit_end) of this rank's plan (tests, bounded
+ * samples of a full-size workload).  unit_end = -1 means "to the end". */
+int epi4_search_units(epi4_ctx* ctx, int64_t unit_begin, int64_t unit_end, int32_t top_k,
+                      uint64_t* quads_out, double* k2_out, int32_t* n_out);
+
+/* Verification hook: the 2 x 81 contingency table (controls row first, cell 27a+9b+3c+d,
+ * 0=AA 1=Aa 2=aa) of each listed quad (packed, any SNP order), computed from the device planes:
+ * 16 cells by AND+POPC of the planes and the other 65 by the same lower-order recovery the search
+ * epilogue uses.  quads and counts_out are host arrays; counts_out has
+ * n * 162 entries. */
+int epi4_tables(epi4_ctx* ctx, const uint64_t* quads, int64_t n, uint32_t* counts_out);
+
+/* Debug/verification: make the next search also write the 162 counts of EVERY evaluated quad into
+ * a device buffer indexed by the quad's colex rank C(l,4)+C(k,3)+C(j,2)+i (162 uint32 each);
+ * counts_dev = NULL disables.  Only for small N (the buffer has C(N,4)*162 entries). */
+int epi4_set_dump(epi4_ctx* ctx, uint32_t* counts_dev);
+
+/* ---- plan --------------------------------------------------------------------
+ * Work unit u = (w-block, x): all quads whose first SNP lies in w-block [32*wb, 32*wb+32) and
+ * whose second SNP is x.  The plan lists this rank's units (static LPT by modelled cost, identical
+ * on every rank).  Host-only; usable without a GPU. */
+int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world);
+int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* wb_x_out /* 2 x count */,
+                    double* cost_out /* count, may be NULL */);
+
+/* ---- measurement ---------------------------------------------------------------------------- */
+typedef struct {
+    double ms_pack;        /* last load: H2D + pack kernel                         */
+    double ms_pop;         /* last load: T1 + T2 + T3 kernels                      */
+    double ms_quad;        /* last search: 4-way contraction + fused epilogue      */
+    double ms_merge;       /* last search: top-k merge + D2H                       */
+    int64_t quads;         /* quads evaluated by the last search (useful)          */
+    int64_t tiles;         /* tiles executed by the last search                    */
+    int64_t launches;      /* kernels launched by the last search                  */
+    int64_t launches_load; /* kernels launched by the last load                    */
+    double executed_macs;  /* MACs issued by the last search's contraction (incl. padding/masking) */
+} epi4_stats;
+
+int epi4_get_stats(epi4_ctx* ctx, epi4_stats* out);
+
+/* Message of the last failure on this thread ("" if none). */
+const char* epi4_last_error(void);
+
+/* Library build string (arch, pipe list). */
+const char* epi4_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EPI4_H */

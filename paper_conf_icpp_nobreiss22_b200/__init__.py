@@ -1,0 +1,112 @@
+"""B200-native exhaustive fourth-order K2 epistasis search (Epi4Tensor's hot path, PAPER.md).
+
+The search runs in libepi4 (CUDA kernels for sm_100a behind the C ABI of include/epi4.h); this
+package is the thin Python layer: the ctypes binding (``binding``), a small object wrapper and the
+multi-GPU glue (one process per GPU; the per-rank top-k lists are all-gathered over NCCL/NVLink and
+merged deterministically — SURVEY.md §8(e)).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import binding
+from .binding import Epi4Error, epi4_last_error, epi4_version  # noqa: F401
+
+__all__ = ["Epi4", "merge_topk", "search_distributed", "pack_index", "unpack_index", "binding", "Epi4Error"]
+
+
+def pack_index(i, j, k, l) -> int:
+    """four 16-bit SNP indices in one 64-bit word."""
+    return (int(i) << 48) | (int(j) << 32) | (int(k) << 16) | int(l)
+
+
+def unpack_index(idx) -> tuple:
+    idx = int(idx)
+    return ((idx >> 48) & 0xFFFF, (idx >> 32) & 0xFFFF, (idx >> 16) & 0xFFFF, idx & 0xFFFF)
+
+
+class Epi4:
+    """One search context on one GPU (one per rank)."""
+
+    def __init__(self, device: int = 0, pipe: str = "i8tc", rank: int = 0, world: int = 1, grid: int = 0):
+        o = binding.epi4_default_opts()
+        o.pipe = binding.PIPES[pipe]
+        o.rank, o.world, o.grid = int(rank), int(world), int(grid)
+        self.pipe, self.rank, self.world = pipe, int(rank), int(world)
+        self.ctx = binding.epi4_create(device, o)
+
+    def close(self):
+        if getattr(self, "ctx", None):
+            binding.epi4_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def set_stream(self, stream):
+        binding.epi4_set_stream(self.ctx, stream)
+
+    def load_genotypes(self, geno, phen):
+        """Byte genotypes N x M (SNP-major, {0,1,2}) + phenotypes M; host (numpy) or device (torch)."""
+        n, m = geno.shape
+        binding.epi4_pack_genotypes(self.ctx, geno, phen, n, m)
+
+    def load_bits(self, planes_ctrl, planes_case, n_snps, n_controls, n_cases):
+        binding.epi4_load_bits(self.ctx, planes_ctrl, planes_case, n_snps, n_controls, n_cases)
+
+    def search(self, top_k: int = 1):
+        return binding.epi4_search(self.ctx, top_k)
+
+    def search_units(self, unit_begin: int, unit_end: int, top_k: int = 1):
+        return binding.epi4_search_units(self.ctx, unit_begin, unit_end, top_k)
+
+    def tables(self, quads):
+        return binding.epi4_tables(self.ctx, quads)
+
+    def stats(self) -> dict:
+        return binding.epi4_get_stats(self.ctx)
+
+
+def merge_topk(parts, top_k: int):
+    """Deterministic merge of (idx uint64[], k2 float64[]) lists by the (K2, index) key."""
+    idx = np.concatenate([np.asarray(p[0], dtype=np.uint64) for p in parts]) if parts else np.zeros(0, np.uint64)
+    k2 = np.concatenate([np.asarray(p[1], dtype=np.float64) for p in parts]) if parts else np.zeros(0)
+    order = np.lexsort((idx, k2))[:top_k]
+    return idx[order], k2[order]
+
+
+def search_distributed(local_search, top_k: int, group=None, device=None):
+    """Run ``local_search(top_k)`` on every rank, all-gather the per-rank lists and merge them
+    (the single collective of the search).  Works with NCCL (device tensors) and
+    gloo (CPU tensors)."""
+    import torch
+    import torch.distributed as dist
+
+    idx, k2 = local_search(top_k)
+    world = dist.get_world_size(group)
+    dev = device if device is not None else ("cuda" if dist.get_backend(group) == "nccl" else "cpu")
+    buf = torch.full((top_k, 2), float("inf"), dtype=torch.float64)
+    n = len(idx)
+    buf[:n, 0] = torch.from_numpy(np.asarray(k2, dtype=np.float64))
+    buf[:n, 1] = torch.from_numpy(np.asarray(idx, dtype=np.uint64).view(np.float64))   # bit-cast
+    cnt = torch.tensor([n], dtype=torch.int64)
+    buf, cnt = buf.to(dev), cnt.to(dev)
+    bufs = [torch.empty_like(buf) for _ in range(world)]
+    cnts = [torch.empty_like(cnt) for _ in range(world)]
+    dist.all_gather(bufs, buf, group=group)
+    dist.all_gather(cnts, cnt, group=group)
+    parts = []
+    for b, c in zip(bufs, cnts):
+        b = b.cpu().numpy()
+        c = int(c.item())
+        parts.append((b[:c, 1].copy().view(np.uint64), b[:c, 0].copy()))
+    return merge_topk(parts, top_k)

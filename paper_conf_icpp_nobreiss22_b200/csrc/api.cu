@@ -1,0 +1,566 @@
+// api.cu — host side of libepi4: the C ABI (include/epi4.h), context and device memory, the
+// static LPT work plan, search orchestration and measurement.
+//
+// Flow of one search (Algorithm 1, L80-L104, re-designed B200-first):
+//   load:   H2D of the planes or byte genotypes -> pack / retile kernels -> T1, T2, T3 kernels
+//           -> host-built lgamma table (double, "each GPU stores a full copy").
+//   search: this rank's units (static LPT) -> tile prefix -> ONE persistent contraction kernel with
+//           the fused epilogue over all tiles -> merge of the per-CTA top-k lists -> D2H of top_k.
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "epi4_internal.cuh"
+
+using namespace epi4;
+
+namespace {
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CU(call)                                                                                   \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess)                                                                     \
+            return fail(e_ == cudaErrorMemoryAllocation ? EPI4_ENOMEM : EPI4_ECUDA, "%s: %s (%s:%d)", \
+                        #call, cudaGetErrorString(e_), __FILE__, __LINE__);                        \
+    } while (0)
+
+template <class T>
+void dfree(T*& p) {
+    if (p) cudaFree((void*)p);
+    p = nullptr;
+}
+}  // namespace
+
+struct epi4_ctx {
+    int device = 0;
+    epi4_opts opts{};
+    int sm_count = 0;
+    cudaStream_t own_stream = nullptr, stream = nullptr;
+    // dataset
+    bool loaded = false;
+    int32_t n = 0, npad = 0;
+    int64_t np[2] = {0, 0};
+    int32_t nchunks[2] = {0, 0};
+    uint32_t* planes[2] = {nullptr, nullptr};
+    uint32_t *T1 = nullptr, *T2 = nullptr, *T3 = nullptr;
+    double* lgam = nullptr;
+    // search workspace
+    Unit* d_units = nullptr;
+    int64_t* d_prefix = nullptr;
+    size_t units_cap = 0;
+    unsigned long long* d_counters = nullptr;   // [0] tile counter, [1] quads done
+    double* d_list_k2 = nullptr;
+    uint64_t* d_list_idx = nullptr;
+    int32_t* d_list_cnt = nullptr;
+    size_t list_entries = 0;
+    int32_t list_slots = 0;
+    double* d_out_k2 = nullptr;
+    uint64_t* d_out_idx = nullptr;
+    int32_t* d_out_n = nullptr;
+    unsigned int* d_status = nullptr;
+    uint32_t* dump = nullptr;
+    cudaEvent_t ev[6] = {};
+    epi4_stats stats{};
+};
+
+namespace {
+
+DevData devdata(const epi4_ctx* c) {
+    DevData d;
+    d.planes[0] = c->planes[0];
+    d.planes[1] = c->planes[1];
+    d.nchunks[0] = c->nchunks[0];
+    d.nchunks[1] = c->nchunks[1];
+    d.n = c->n;
+    d.npad = c->npad;
+    d.np[0] = (uint32_t)c->np[0];
+    d.np[1] = (uint32_t)c->np[1];
+    d.T1 = c->T1;
+    d.T2 = c->T2;
+    d.T3 = c->T3;
+    d.lgam = c->lgam;
+    return d;
+}
+
+void free_data(epi4_ctx* c) {
+    dfree(c->planes[0]);
+    dfree(c->planes[1]);
+    dfree(c->T1);
+    dfree(c->T2);
+    dfree(c->T3);
+    dfree(c->lgam);
+    c->loaded = false;
+}
+
+// ---- plan: units, modelled cost, static LPT --------------------------------------------------------
+struct PlanEntry {
+    Unit u;
+    double cost;
+};
+
+std::vector<PlanEntry> all_units(int32_t n) {
+    std::vector<PlanEntry> v;
+    const int32_t nb = (n + EPI4_B - 1) / EPI4_B;
+    for (int32_t wb = 0; wb < nb; ++wb)
+        for (int32_t x = wb * EPI4_B + 1; x <= n - 3; ++x) {
+            const double cost = (double)unit_tiles(n, x, 1);
+            if (cost > 0) v.push_back({{wb, x}, cost});
+        }
+    return v;
+}
+
+std::vector<PlanEntry> plan_rank(int32_t n, int32_t rank, int32_t world) {
+    std::vector<PlanEntry> v = all_units(n);
+    // longest processing time first; ties broken by (wb, x) so every rank computes the same plan
+    std::stable_sort(v.begin(), v.end(), [](const PlanEntry& a, const PlanEntry& b) {
+        if (a.cost != b.cost) return a.cost > b.cost;
+        if (a.u.wb != b.u.wb) return a.u.wb < b.u.wb;
+        return a.u.x < b.u.x;
+    });
+    if (world <= 1) return v;
+    std::vector<double> load(world, 0.0);
+    std::vector<PlanEntry> mine;
+    for (const PlanEntry& e : v) {
+        int best = 0;
+        for (int r = 1; r < world; ++r)
+            if (load[r] < load[best]) best = r;
+        load[best] += e.cost;
+        if (best == rank) mine.push_back(e);
+    }
+    return mine;
+}
+
+int ensure_lists(epi4_ctx* c, int32_t slots, int32_t cap) {
+    const size_t need = (size_t)slots * cap;
+    if (need > c->list_entries) {
+        dfree(c->d_list_k2);
+        dfree(c->d_list_idx);
+        CU(cudaMalloc(&c->d_list_k2, need * sizeof(double)));
+        CU(cudaMalloc(&c->d_list_idx, need * sizeof(uint64_t)));
+        c->list_entries = need;
+    }
+    if (slots > c->list_slots) {
+        dfree(c->d_list_cnt);
+        CU(cudaMalloc(&c->d_list_cnt, (size_t)slots * sizeof(int32_t)));
+        c->list_slots = slots;
+    }
+    return 0;
+}
+
+int finish_load(epi4_ctx* c) {
+    // status of the pack / retile kernels
+    unsigned int st = 0;
+    CU(cudaMemcpyAsync(&st, c->d_status, sizeof st, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaStreamSynchronize(c->stream));
+    if (st & EPI4_ST_BAD_GENO) return fail(EPI4_EINVAL, "genotype code > 2");
+    if (st & EPI4_ST_BAD_PHEN) return fail(EPI4_EINVAL, "phenotype value > 1");
+    if (st & EPI4_ST_PAD_BITS) return fail(EPI4_EINVAL, "pad bits beyond the sample count are set");
+    if (st & EPI4_ST_AA_AND_Aa) return fail(EPI4_EINVAL, "a sample has both AA and Aa bits set");
+    // lower-order tables
+    const int64_t n = c->n;
+    CU(cudaMalloc(&c->T1, (size_t)n * 4 * sizeof(uint32_t)));
+    CU(cudaMalloc(&c->T2, (size_t)c2(n) * 8 * sizeof(uint32_t)));
+    const size_t t3b = (size_t)c3(n) * 16 * sizeof(uint32_t);
+    size_t freeb = 0, totb = 0;
+    CU(cudaMemGetInfo(&freeb, &totb));
+    if (t3b + ((size_t)1 << 30) > freeb)
+        return fail(EPI4_ENOMEM, "3-way tables need %.1f GB but only %.1f GB of HBM are free (N=%d); "
+                    "the windowed T3 path for larger N is not built yet", t3b / 1e9, freeb / 1e9, c->n);
+    CU(cudaMalloc(&c->T3, t3b));
+    // lgamma table L[k] = lgamma(k + 1) for k in [0, M + 1]
+    const int64_t m = c->np[0] + c->np[1];
+    std::vector<double> L((size_t)m + 2);
+    for (int64_t k = 0; k < m + 2; ++k) L[(size_t)k] = std::lgamma((double)k + 1.0);
+    CU(cudaMalloc(&c->lgam, L.size() * sizeof(double)));
+    CU(cudaMemcpyAsync(c->lgam, L.data(), L.size() * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+    CU(cudaEventRecord(c->ev[2], c->stream));
+    CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, c->stream, &c->stats.launches_load));
+    CU(cudaEventRecord(c->ev[3], c->stream));
+    CU(cudaStreamSynchronize(c->stream));
+    float ms = 0;
+    CU(cudaEventElapsedTime(&ms, c->ev[2], c->ev[3]));
+    c->stats.ms_pop = ms;
+    c->loaded = true;
+    return 0;
+}
+
+int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
+    free_data(c);
+    c->n = n;
+    c->npad = (n + EPI4_B - 1) / EPI4_B * EPI4_B;
+    c->np[0] = n0;
+    c->np[1] = n1;
+    for (int p = 0; p < 2; ++p) {
+        c->nchunks[p] = (int32_t)((c->np[p] + EPI4_CHUNK_SAMPLES - 1) / EPI4_CHUNK_SAMPLES);
+        const size_t words = (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_WORDS;
+        CU(cudaMalloc(&c->planes[p], words * sizeof(uint32_t)));
+        CU(cudaMemsetAsync(c->planes[p], 0, words * sizeof(uint32_t), c->stream));
+    }
+    CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
+    return 0;
+}
+
+int check_dims(int32_t n_snps, int64_t n0, int64_t n1) {
+    if (n_snps < 4 || n_snps > 65536) return fail(EPI4_EINVAL, "n_snps=%d outside [4, 65536]", n_snps);
+    if (n0 < 1 || n1 < 1) return fail(EPI4_EINVAL, "need at least one control and one case (n0=%lld n1=%lld)",
+                                       (long long)n0, (long long)n1);
+    if (n0 + n1 > ((int64_t)1 << 31) - 4) return fail(EPI4_EINVAL, "too many samples");
+    return 0;
+}
+
+}  // namespace
+
+// =====================================================================================================
+extern "C" {
+
+void epi4_default_opts(epi4_opts* o) {
+    if (!o) return;
+    std::memset(o, 0, sizeof *o);
+    o->block = EPI4_B;
+    o->pipe = EPI4_PIPE_I8TC;
+    o->rank = 0;
+    o->world = 1;
+    o->grid = 0;
+}
+
+const char* epi4_last_error(void) { return g_err.c_str(); }
+
+const char* epi4_version(void) {
+    return "libepi4 sm_100a (pipes: i8tc=tcgen05.mma.kind::i8, lop3=CUDA-core AND+POPC)";
+}
+
+int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
+    if (!out) return fail(EPI4_EINVAL, "out is NULL");
+    *out = nullptr;
+    epi4_opts o;
+    epi4_default_opts(&o);
+    if (opts) o = *opts;
+    if (o.block != EPI4_B) return fail(EPI4_EINVAL, "block=%d: only B=32 is supported", o.block);
+    if (o.pipe != EPI4_PIPE_I8TC && o.pipe != EPI4_PIPE_LOP3) return fail(EPI4_EINVAL, "unknown pipe %d", o.pipe);
+    if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return fail(EPI4_EINVAL, "bad rank/world %d/%d", o.rank, o.world);
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(EPI4_ENODEV, "no CUDA device");
+    if (cuda_device < 0 || cuda_device >= ndev) return fail(EPI4_ENODEV, "device %d out of range", cuda_device);
+    CU(cudaSetDevice(cuda_device));
+    cudaDeviceProp prop;
+    CU(cudaGetDeviceProperties(&prop, cuda_device));
+    if (prop.major != 10 || prop.minor != 0)
+        return fail(EPI4_ENODEV, "device %d is sm_%d%d; libepi4 is built for sm_100a only", cuda_device, prop.major,
+                    prop.minor);
+    epi4_ctx* c = new epi4_ctx();
+    c->device = cuda_device;
+    c->opts = o;
+    c->sm_count = prop.multiProcessorCount;
+    cudaError_t e = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaMalloc(&c->d_status, sizeof(unsigned int));
+    if (e == cudaSuccess) e = cudaMalloc(&c->d_counters, 4 * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc(&c->d_out_k2, EPI4_MAX_TOPK * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&c->d_out_idx, EPI4_MAX_TOPK * sizeof(uint64_t));
+    if (e == cudaSuccess) e = cudaMalloc(&c->d_out_n, sizeof(int32_t));
+    for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&c->ev[i]);
+    if (e != cudaSuccess) {
+        epi4_destroy(c);
+        return fail(EPI4_ECUDA, "create: %s", cudaGetErrorString(e));
+    }
+    c->stream = c->own_stream;
+    *out = c;
+    return 0;
+}
+
+void epi4_destroy(epi4_ctx* c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    free_data(c);
+    dfree(c->d_units);
+    dfree(c->d_prefix);
+    dfree(c->d_counters);
+    dfree(c->d_list_k2);
+    dfree(c->d_list_idx);
+    dfree(c->d_list_cnt);
+    dfree(c->d_out_k2);
+    dfree(c->d_out_idx);
+    dfree(c->d_out_n);
+    dfree(c->d_status);
+    for (int i = 0; i < 6; ++i)
+        if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+    if (c->own_stream) cudaStreamDestroy(c->own_stream);
+    delete c;
+}
+
+int epi4_set_stream(epi4_ctx* c, void* s) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    c->stream = s ? (cudaStream_t)s : c->own_stream;
+    return 0;
+}
+
+int epi4_load_bits(epi4_ctx* c, const uint32_t* pc, const uint32_t* pk, int32_t n_snps, int64_t n0, int64_t n1,
+                   int32_t ptr_kind) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (!pc || !pk) return fail(EPI4_EINVAL, "planes pointer is NULL");
+    if (int r = check_dims(n_snps, n0, n1)) return r;
+    CU(cudaSetDevice(c->device));
+    c->stats.launches_load = 0;
+    if (int r = alloc_planes(c, n_snps, n0, n1)) return r;
+    CU(cudaEventRecord(c->ev[0], c->stream));
+    const uint32_t* src[2] = {pc, pk};
+    for (int p = 0; p < 2; ++p) {
+        const size_t words = (size_t)2 * n_snps * (size_t)((c->np[p] + 31) / 32);
+        const uint32_t* rows = src[p];
+        uint32_t* tmp = nullptr;
+        if (ptr_kind == EPI4_PTR_HOST) {
+            CU(cudaMalloc(&tmp, words * sizeof(uint32_t)));
+            CU(cudaMemcpyAsync(tmp, src[p], words * sizeof(uint32_t), cudaMemcpyHostToDevice, c->stream));
+            rows = tmp;
+        } else if (ptr_kind != EPI4_PTR_DEVICE) {
+            return fail(EPI4_EINVAL, "ptr_kind %d", ptr_kind);
+        }
+        cudaError_t e = launch_retile(rows, n_snps, c->np[p], c->npad, c->nchunks[p], c->planes[p], c->d_status,
+                                      c->stream, &c->stats.launches_load);
+        if (tmp) {
+            cudaStreamSynchronize(c->stream);
+            cudaFree(tmp);
+        }
+        CU(e);
+    }
+    CU(cudaEventRecord(c->ev[1], c->stream));
+    int r = finish_load(c);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, c->ev[0], c->ev[1]);
+    c->stats.ms_pack = ms;
+    return r;
+}
+
+int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, int32_t n_snps, int64_t m,
+                        int32_t ptr_kind) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (!geno || !phen) return fail(EPI4_EINVAL, "genotype pointer is NULL");
+    if (n_snps < 4 || n_snps > 65536) return fail(EPI4_EINVAL, "n_snps=%d outside [4, 65536]", n_snps);
+    if (m < 2 || m > ((int64_t)1 << 31) - 4) return fail(EPI4_EINVAL, "n_samples=%lld", (long long)m);
+    if (ptr_kind != EPI4_PTR_HOST && ptr_kind != EPI4_PTR_DEVICE) return fail(EPI4_EINVAL, "ptr_kind %d", ptr_kind);
+    CU(cudaSetDevice(c->device));
+    c->stats.launches_load = 0;
+    const uint8_t *dg = geno, *dp = phen;
+    uint8_t *tg = nullptr, *tp = nullptr;
+    int32_t* idx = nullptr;   // [m] (idx0 then idx1) + 2 counts
+    CU(cudaEventRecord(c->ev[0], c->stream));
+    if (ptr_kind == EPI4_PTR_HOST) {
+        CU(cudaMalloc(&tg, (size_t)n_snps * m));
+        CU(cudaMalloc(&tp, (size_t)m));
+        CU(cudaMemcpyAsync(tg, geno, (size_t)n_snps * m, cudaMemcpyHostToDevice, c->stream));
+        CU(cudaMemcpyAsync(tp, phen, (size_t)m, cudaMemcpyHostToDevice, c->stream));
+        dg = tg;
+        dp = tp;
+    }
+    CU(cudaMalloc(&idx, (size_t)(2 * m + 2) * sizeof(int32_t)));
+    CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
+    // pass 1: split by phenotype (idx0 at [0, m), idx1 at [m, 2m), counts at [2m, 2m+2))
+    CU(launch_split_phen(dp, m, idx, idx + m, idx + 2 * m, c->d_status, c->stream, &c->stats.launches_load));
+    int32_t cnt[2] = {0, 0};
+    unsigned int st = 0;
+    CU(cudaMemcpyAsync(cnt, idx + 2 * m, sizeof cnt, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(&st, c->d_status, sizeof st, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaStreamSynchronize(c->stream));
+    int r = 0;
+    if (st & EPI4_ST_BAD_PHEN) r = fail(EPI4_EINVAL, "phenotype value > 1");
+    else r = check_dims(n_snps, cnt[0], cnt[1]);
+    if (!r) r = alloc_planes(c, n_snps, cnt[0], cnt[1]);
+    if (!r) {
+        for (int p = 0; p < 2 && !r; ++p) {
+            cudaError_t e = launch_pack(dg, n_snps, m, idx + (p ? m : 0), c->np[p], c->npad, c->nchunks[p],
+                                        c->planes[p], c->d_status, c->stream, &c->stats.launches_load);
+            if (e != cudaSuccess) r = fail(EPI4_ECUDA, "pack: %s", cudaGetErrorString(e));
+        }
+    }
+    cudaEventRecord(c->ev[1], c->stream);
+    cudaStreamSynchronize(c->stream);
+    cudaFree(idx);
+    if (tg) cudaFree(tg);
+    if (tp) cudaFree(tp);
+    if (r) return r;
+    r = finish_load(c);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, c->ev[0], c->ev[1]);
+    c->stats.ms_pack = ms;
+    return r;
+}
+
+int epi4_get_bits(epi4_ctx* c, uint32_t* pc, uint32_t* pk) {
+    if (!c || !pc || !pk) return fail(EPI4_EINVAL, "NULL argument");
+    if (!c->loaded) return fail(EPI4_ESTATE, "no data loaded");
+    CU(cudaSetDevice(c->device));
+    uint32_t* dst[2] = {pc, pk};
+    for (int p = 0; p < 2; ++p) {
+        const size_t words = (size_t)2 * c->n * (size_t)((c->np[p] + 31) / 32);
+        uint32_t* tmp = nullptr;
+        CU(cudaMalloc(&tmp, words * sizeof(uint32_t)));
+        cudaError_t e = launch_untile(c->planes[p], c->n, c->np[p], c->npad, c->nchunks[p], tmp, c->stream, nullptr);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(dst[p], tmp, words * sizeof(uint32_t), cudaMemcpyDeviceToHost, c->stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+        cudaFree(tmp);
+        CU(e);
+    }
+    return 0;
+}
+
+int epi4_set_dump(epi4_ctx* c, uint32_t* counts_dev) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    c->dump = counts_dev;
+    return 0;
+}
+
+int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world) {
+    if (n_snps < 4 || n_snps > 65536 || world < 1 || rank < 0 || rank >= world) {
+        fail(EPI4_EINVAL, "bad plan arguments");
+        return EPI4_EINVAL;
+    }
+    return (int64_t)plan_rank(n_snps, rank, world).size();
+}
+
+int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* out, double* cost_out) {
+    if (n_snps < 4 || n_snps > 65536 || world < 1 || rank < 0 || rank >= world || !out)
+        return fail(EPI4_EINVAL, "bad plan arguments");
+    std::vector<PlanEntry> v = plan_rank(n_snps, rank, world);
+    for (size_t i = 0; i < v.size(); ++i) {
+        out[2 * i] = v[i].u.wb;
+        out[2 * i + 1] = v[i].u.x;
+        if (cost_out) cost_out[i] = v[i].cost;
+    }
+    return 0;
+}
+
+int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64_t* quads_out, double* k2_out,
+                      int32_t* n_out) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
+    if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
+    if (!quads_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
+    CU(cudaSetDevice(c->device));
+    std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
+    const int64_t nall = (int64_t)plan.size();
+    if (ue < 0 || ue > nall) ue = nall;
+    if (ub < 0) ub = 0;
+    if (ub > ue) ub = ue;
+    const int64_t nu = ue - ub;
+    const int32_t zt = quad_zt(c->opts.pipe);
+    std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
+    std::vector<int64_t> prefix((size_t)std::max<int64_t>(nu, 1));
+    int64_t acc = 0;
+    for (int64_t i = 0; i < nu; ++i) {
+        units[(size_t)i] = plan[(size_t)(ub + i)].u;
+        acc += unit_tiles(c->n, units[(size_t)i].x, zt);
+        prefix[(size_t)i] = acc;
+    }
+    if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
+        dfree(c->d_units);
+        dfree(c->d_prefix);
+        c->units_cap = (size_t)std::max<int64_t>(nu, 1);
+        CU(cudaMalloc(&c->d_units, c->units_cap * sizeof(Unit)));
+        CU(cudaMalloc(&c->d_prefix, c->units_cap * sizeof(int64_t)));
+    }
+    if (nu > 0) {
+        CU(cudaMemcpyAsync(c->d_units, units.data(), nu * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
+        CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), nu * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
+    }
+    const int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
+    if (int r = ensure_lists(c, grid, top_k)) return r;
+    CU(cudaMemsetAsync(c->d_list_cnt, 0, (size_t)grid * sizeof(int32_t), c->stream));
+    CU(cudaMemsetAsync(c->d_counters, 0, 4 * sizeof(unsigned long long), c->stream));
+    CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
+
+    SearchParams sp;
+    sp.d = devdata(c);
+    sp.units = c->d_units;
+    sp.prefix = c->d_prefix;
+    sp.nunits = nu;
+    sp.ntiles = acc;
+    sp.zt = zt;
+    sp.tile_counter = c->d_counters;
+    sp.topk = top_k;
+    sp.list_k2 = c->d_list_k2;
+    sp.list_idx = c->d_list_idx;
+    sp.list_cnt = c->d_list_cnt;
+    sp.dump = c->dump;
+    sp.status = c->d_status;
+    sp.quads_done = c->d_counters + 1;
+
+    c->stats.launches = 0;
+    CU(cudaEventRecord(c->ev[2], c->stream));
+    if (acc > 0) {
+        cudaError_t e = c->opts.pipe == EPI4_PIPE_LOP3 ? launch_quad_lop3(sp, grid, c->stream, &c->stats.launches)
+                                                       : launch_quad_i8tc(sp, grid, c->stream, &c->stats.launches);
+        CU(e);
+    }
+    CU(cudaEventRecord(c->ev[3], c->stream));
+    CU(launch_merge(sp, grid, c->d_out_k2, c->d_out_idx, c->d_out_n, c->stream, &c->stats.launches));
+    int32_t nout = 0;
+    unsigned long long ctr[2] = {0, 0};
+    CU(cudaMemcpyAsync(&nout, c->d_out_n, sizeof nout, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(quads_out, c->d_out_idx, (size_t)top_k * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(k2_out, c->d_out_k2, (size_t)top_k * sizeof(double), cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(ctr, c->d_counters, sizeof ctr, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaEventRecord(c->ev[4], c->stream));
+    CU(cudaStreamSynchronize(c->stream));
+    float ms = 0;
+    CU(cudaEventElapsedTime(&ms, c->ev[2], c->ev[3]));
+    c->stats.ms_quad = ms;
+    CU(cudaEventElapsedTime(&ms, c->ev[3], c->ev[4]));
+    c->stats.ms_merge = ms;
+    c->stats.quads = (int64_t)ctr[1];
+    c->stats.tiles = acc;
+    c->stats.executed_macs = (double)acc * 1024.0 * 16.0 * zt * (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
+    *n_out = nout;
+    return 0;
+}
+
+int epi4_search(epi4_ctx* c, int32_t top_k, uint64_t* quads_out, double* k2_out, int32_t* n_out) {
+    return epi4_search_units(c, 0, -1, top_k, quads_out, k2_out, n_out);
+}
+
+int epi4_tables(epi4_ctx* c, const uint64_t* quads, int64_t n, uint32_t* counts_out) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (!c->loaded) return fail(EPI4_ESTATE, "tables before any load");
+    if (n < 0 || (n > 0 && (!quads || !counts_out))) return fail(EPI4_EINVAL, "bad quads/counts arguments");
+    if (n == 0) return 0;
+    CU(cudaSetDevice(c->device));
+    uint64_t* dq = nullptr;
+    uint32_t* dc = nullptr;
+    CU(cudaMalloc(&dq, (size_t)n * sizeof(uint64_t)));
+    cudaError_t e = cudaMalloc(&dc, (size_t)n * 162 * sizeof(uint32_t));
+    if (e == cudaSuccess) e = cudaMemcpyAsync(dq, quads, (size_t)n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream);
+    if (e == cudaSuccess) e = launch_tables(devdata(c), dq, n, dc, c->d_status, c->stream, nullptr);
+    unsigned int st = 0;
+    if (e == cudaSuccess)
+        e = cudaMemcpyAsync(counts_out, dc, (size_t)n * 162 * sizeof(uint32_t), cudaMemcpyDeviceToHost, c->stream);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&st, c->d_status, sizeof st, cudaMemcpyDeviceToHost, c->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+    cudaFree(dq);
+    if (dc) cudaFree(dc);
+    CU(e);
+    if (st) return fail(EPI4_EINVAL, "a quad has repeated SNPs or an SNP index >= N");
+    return 0;
+}
+
+int epi4_get_stats(epi4_ctx* c, epi4_stats* out) {
+    if (!c || !out) return fail(EPI4_EINVAL, "NULL argument");
+    *out = c->stats;
+    return 0;
+}
+
+}  // extern "C"

@@ -1,0 +1,278 @@
+// k_prep.cu — data preparation kernels (steps a1 and a2 of SURVEY.md §8(a)):
+//   split_phen : list the sample indices of each phenotype ("genotypic data is split
+//                into cases and controls ... stored in a contiguous memory region")
+//   pack       : byte genotypes -> 2 bit planes per SNP per phenotype, AA and Aa; aa not stored
+//                (§3.1), written in the chunked device layout (epi4_internal.cuh)
+//   retile     : row-major host planes (the ABI format) -> chunked layout, validating pad bits and
+//                AA & Aa == 0;  untile: the reverse (epi4_get_bits)
+//   pop        : T1 (indivPop), T2 (pairwPop, L86, L112-114) and the 3-way tables T3
+//                (8 non-aa cells per triple, the tensorOp_3way proto-tables of) by AND+POPC.
+#include "epi4_internal.cuh"
+
+namespace epi4 {
+
+// ---- split by phenotype ------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024) k_split_phen(const uint8_t* __restrict__ phen, int64_t m,
+                                                     int32_t* __restrict__ idx0, int32_t* __restrict__ idx1,
+                                                     int32_t* counts, unsigned int* status) {
+    __shared__ int s_w1[32];
+    __shared__ int s_base1, s_base0;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    if (tid == 0) { s_base0 = 0; s_base1 = 0; }
+    __syncthreads();
+    for (int64_t off = 0; off < m; off += 1024) {
+        const int64_t s = off + tid;
+        int v = 0, valid = s < m;
+        if (valid) {
+            v = phen[s];
+            if (v > 1) { atomicOr(status, EPI4_ST_BAD_PHEN); v = 1; }
+        }
+        const unsigned b1 = __ballot_sync(0xffffffffu, valid && v == 1);
+        if (lane == 0) s_w1[wid] = __popc(b1);
+        __syncthreads();
+        int pre1 = 0, tot1 = 0;
+        for (int k = 0; k < 32; ++k) {
+            if (k < wid) pre1 += s_w1[k];
+            tot1 += s_w1[k];
+        }
+        // the valid threads of this round are a prefix of the block, so tid = rank among valid
+        const int r1 = pre1 + __popc(b1 & ((1u << lane) - 1));
+        const int r0 = tid - r1;
+        const int base0 = s_base0, base1 = s_base1;
+        if (valid) {
+            if (v == 1) idx1[base1 + r1] = (int32_t)s; else idx0[base0 + r0] = (int32_t)s;
+        }
+        __syncthreads();
+        if (tid == 0) {
+            const int nvalid = (m - off) < 1024 ? (int)(m - off) : 1024;
+            s_base1 = base1 + tot1;
+            s_base0 = base0 + (nvalid - tot1);
+        }
+        __syncthreads();
+    }
+    if (tid == 0) { counts[0] = s_base0; counts[1] = s_base1; }
+}
+
+cudaError_t launch_split_phen(const uint8_t* phen, int64_t m, int32_t* idx0, int32_t* idx1, int32_t* counts,
+                              unsigned int* status, cudaStream_t s, int64_t* launches) {
+    k_split_phen<<<1, 1024, 0, s>>>(phen, m, idx0, idx1, counts, status);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+// ---- pack: one thread = one 32-sample word of (snp, chunk, word) -> AA and Aa words ---------------
+__global__ void __launch_bounds__(256) k_pack(const uint8_t* __restrict__ geno, int32_t n, int64_t m,
+                                              const int32_t* __restrict__ idx, int64_t np, int32_t npad,
+                                              int32_t nchunks, uint32_t* __restrict__ planes,
+                                              unsigned int* status) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t total = (int64_t)n * nchunks * EPI4_CHUNK_WORDS;
+    if (t >= total) return;
+    const int w = (int)(t % EPI4_CHUNK_WORDS);
+    const int32_t snp = (int32_t)((t / EPI4_CHUNK_WORDS) % n);
+    const int64_t kc = t / ((int64_t)EPI4_CHUNK_WORDS * n);
+    const uint8_t* row = geno + (int64_t)snp * m;
+    const int64_t s0 = kc * EPI4_CHUNK_SAMPLES + (int64_t)w * 32;
+    uint32_t aa = 0, het = 0;
+    bool bad = false;
+#pragma unroll 8
+    for (int b = 0; b < 32; ++b) {
+        const int64_t k = s0 + b;
+        if (k < np) {
+            const uint8_t g = row[idx[k]];
+            bad |= g > 2;
+            aa |= (uint32_t)(g == 0) << b;
+            het |= (uint32_t)(g == 1) << b;
+        }
+    }
+    if (bad) atomicOr(status, EPI4_ST_BAD_GENO);
+    planes[plane_off(kc, npad, snp, 0, w)] = aa;
+    planes[plane_off(kc, npad, snp, 1, w)] = het;
+}
+
+cudaError_t launch_pack(const uint8_t* geno, int32_t n, int64_t m, const int32_t* idx, int64_t np, int32_t npad,
+                        int32_t nchunks, uint32_t* planes, unsigned int* status, cudaStream_t s, int64_t* launches) {
+    const int64_t total = (int64_t)n * nchunks * EPI4_CHUNK_WORDS;
+    const int64_t blocks = (total + 255) / 256;
+    if (blocks > 0) {
+        k_pack<<<(unsigned)blocks, 256, 0, s>>>(geno, n, m, idx, np, npad, nchunks, planes, status);
+        if (launches) ++*launches;
+    }
+    return cudaGetLastError();
+}
+
+// ---- retile / untile: row-major [2n][wp] <-> chunked ----------------------------------------------
+__global__ void __launch_bounds__(256) k_retile(const uint32_t* __restrict__ rows, int32_t n, int64_t np,
+                                                int32_t npad, int32_t nchunks, uint32_t* __restrict__ planes,
+                                                unsigned int* status) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t total = (int64_t)n * nchunks * EPI4_CHUNK_WORDS;
+    if (t >= total) return;
+    const int w = (int)(t % EPI4_CHUNK_WORDS);
+    const int32_t snp = (int32_t)((t / EPI4_CHUNK_WORDS) % n);
+    const int64_t kc = t / ((int64_t)EPI4_CHUNK_WORDS * n);
+    const int64_t wp = (np + 31) / 32;
+    const int64_t word = kc * EPI4_CHUNK_WORDS + w;
+    uint32_t aa = 0, het = 0;
+    if (word < wp) {
+        aa = rows[(2 * (int64_t)snp + 0) * wp + word];
+        het = rows[(2 * (int64_t)snp + 1) * wp + word];
+        if (word == wp - 1 && (np & 31)) {
+            const uint32_t pad = ~((1u << (np & 31)) - 1u);
+            if ((aa | het) & pad) atomicOr(status, EPI4_ST_PAD_BITS);
+        }
+        if (aa & het) atomicOr(status, EPI4_ST_AA_AND_Aa);
+    }
+    planes[plane_off(kc, npad, snp, 0, w)] = aa;
+    planes[plane_off(kc, npad, snp, 1, w)] = het;
+}
+
+cudaError_t launch_retile(const uint32_t* rows, int32_t n, int64_t np, int32_t npad, int32_t nchunks,
+                          uint32_t* planes, unsigned int* status, cudaStream_t s, int64_t* launches) {
+    const int64_t total = (int64_t)n * nchunks * EPI4_CHUNK_WORDS;
+    const int64_t blocks = (total + 255) / 256;
+    if (blocks > 0) {
+        k_retile<<<(unsigned)blocks, 256, 0, s>>>(rows, n, np, npad, nchunks, planes, status);
+        if (launches) ++*launches;
+    }
+    return cudaGetLastError();
+}
+
+__global__ void __launch_bounds__(256) k_untile(const uint32_t* __restrict__ planes, int32_t n, int64_t np,
+                                                int32_t npad, int32_t nchunks, uint32_t* __restrict__ rows) {
+    const int64_t wp = (np + 31) / 32;
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= 2 * (int64_t)n * wp) return;
+    const int64_t word = t % wp;
+    const int64_t r = t / wp;
+    const int32_t snp = (int32_t)(r >> 1);
+    const int g = (int)(r & 1);
+    rows[t] = planes[plane_off(word / EPI4_CHUNK_WORDS, npad, snp, g, (int)(word % EPI4_CHUNK_WORDS))];
+}
+
+cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t npad, int32_t nchunks,
+                          uint32_t* rows, cudaStream_t s, int64_t* launches) {
+    (void)nchunks;
+    const int64_t total = 2 * (int64_t)n * ((np + 31) / 32);
+    const int64_t blocks = (total + 255) / 256;
+    if (blocks > 0) {
+        k_untile<<<(unsigned)blocks, 256, 0, s>>>(planes, n, np, npad, nchunks, rows);
+        if (launches) ++*launches;
+    }
+    return cudaGetLastError();
+}
+
+// ---- lower-order tables ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_pop1(DevData d, uint32_t* __restrict__ T1) {
+    const int snp = blockIdx.x * blockDim.x + threadIdx.x;
+    if (snp >= d.n) return;
+    uint32_t c[2][2] = {{0, 0}, {0, 0}};
+    for (int p = 0; p < 2; ++p)
+        for (int kc = 0; kc < d.nchunks[p]; ++kc)
+#pragma unroll
+            for (int g = 0; g < 2; ++g) {
+                const uint4 v = __ldg(reinterpret_cast<const uint4*>(d.planes[p] + plane_off(kc, d.npad, snp, g, 0)));
+                c[p][g] += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+            }
+    uint4 o = make_uint4(c[0][0], c[0][1], c[1][0], c[1][1]);
+    reinterpret_cast<uint4*>(T1)[snp] = o;
+}
+
+__device__ __forceinline__ void decode2(int64_t r, int& i, int& j) {
+    int jj = (int)floor((1.0 + sqrt(1.0 + 8.0 * (double)r)) * 0.5);
+    while (c2(jj) > r) --jj;
+    while (c2(jj + 1) <= r) ++jj;
+    j = jj;
+    i = (int)(r - c2(jj));
+}
+__device__ __forceinline__ void decode3(int64_t r, int& i, int& j, int& k) {
+    int kk = (int)floor(cbrt(6.0 * (double)r)) + 1;
+    while (c3(kk) > r) --kk;
+    while (c3(kk + 1) <= r) ++kk;
+    k = kk;
+    decode2(r - c3(kk), i, j);
+}
+
+__device__ __forceinline__ void ld_planes(const DevData& d, int p, int kc, int snp, uint32_t (&v)[2][4]) {
+    const uint4 a = __ldg(reinterpret_cast<const uint4*>(d.planes[p] + plane_off(kc, d.npad, snp, 0, 0)));
+    const uint4 b = __ldg(reinterpret_cast<const uint4*>(d.planes[p] + plane_off(kc, d.npad, snp, 1, 0)));
+    v[0][0] = a.x; v[0][1] = a.y; v[0][2] = a.z; v[0][3] = a.w;
+    v[1][0] = b.x; v[1][1] = b.y; v[1][2] = b.z; v[1][3] = b.w;
+}
+
+__global__ void __launch_bounds__(256) k_pop2(DevData d, uint32_t* __restrict__ T2, int64_t npairs) {
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= npairs) return;
+    int i, j;
+    decode2(r, i, j);
+    uint32_t out[2][4];
+    for (int p = 0; p < 2; ++p) {
+        uint32_t c[4] = {0, 0, 0, 0};
+        for (int kc = 0; kc < d.nchunks[p]; ++kc) {
+            uint32_t a[2][4], b[2][4];
+            ld_planes(d, p, kc, i, a);
+            ld_planes(d, p, kc, j, b);
+#pragma unroll
+            for (int w = 0; w < 4; ++w)
+#pragma unroll
+                for (int x = 0; x < 2; ++x)
+#pragma unroll
+                    for (int y = 0; y < 2; ++y) c[x * 2 + y] += __popc(a[x][w] & b[y][w]);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) out[p][q] = c[q];
+    }
+    uint4* o = reinterpret_cast<uint4*>(T2 + r * 8);
+    o[0] = make_uint4(out[0][0], out[0][1], out[0][2], out[0][3]);
+    o[1] = make_uint4(out[1][0], out[1][1], out[1][2], out[1][3]);
+}
+
+__global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ T3, int64_t ntri) {
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= ntri) return;
+    int i, j, k;
+    decode3(r, i, j, k);
+    uint32_t out[2][8];
+    for (int p = 0; p < 2; ++p) {
+        uint32_t c[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        for (int kc = 0; kc < d.nchunks[p]; ++kc) {
+            uint32_t a[2][4], b[2][4], e[2][4];
+            ld_planes(d, p, kc, i, a);
+            ld_planes(d, p, kc, j, b);
+            ld_planes(d, p, kc, k, e);
+#pragma unroll
+            for (int w = 0; w < 4; ++w)
+#pragma unroll
+                for (int y = 0; y < 2; ++y)
+#pragma unroll
+                    for (int z = 0; z < 2; ++z) {
+                        const uint32_t yz = b[y][w] & e[z][w];
+                        c[0 * 4 + y * 2 + z] += __popc(a[0][w] & yz);
+                        c[1 * 4 + y * 2 + z] += __popc(a[1][w] & yz);
+                    }
+        }
+#pragma unroll
+        for (int q = 0; q < 8; ++q) out[p][q] = c[q];
+    }
+    uint4* o = reinterpret_cast<uint4*>(T3 + r * 16);
+    o[0] = make_uint4(out[0][0], out[0][1], out[0][2], out[0][3]);
+    o[1] = make_uint4(out[0][4], out[0][5], out[0][6], out[0][7]);
+    o[2] = make_uint4(out[1][0], out[1][1], out[1][2], out[1][3]);
+    o[3] = make_uint4(out[1][4], out[1][5], out[1][6], out[1][7]);
+}
+
+cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, cudaStream_t s,
+                       int64_t* launches) {
+    k_pop1<<<(d.n + 255) / 256, 256, 0, s>>>(d, T1);
+    if (launches) ++*launches;
+    const int64_t np2 = c2(d.n), np3 = c3(d.n);
+    k_pop2<<<(unsigned)((np2 + 255) / 256), 256, 0, s>>>(d, T2, np2);
+    if (launches) ++*launches;
+    if (np3 > 0) {
+        k_pop3<<<(unsigned)((np3 + 255) / 256), 256, 0, s>>>(d, T3, np3);
+        if (launches) ++*launches;
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace epi4

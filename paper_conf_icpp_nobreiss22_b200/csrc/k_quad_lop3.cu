@@ -1,0 +1,137 @@
+// k_quad_lop3.cu — CUDA-core contraction (EPI4_PIPE_LOP3): AND + POPC on bit planes.
+//
+// The cross-check pipe of SURVEY.md §8(a) a5: for each tile (w-block wb, x, y-block yb, z) the 32 x 32
+// (w, y) combinations are counted directly: for each 32-sample word, the pair rows
+// (w,x,a,b) = P_a(w) & P_b(x) ("combine") are ANDed with the pair columns
+// (y,z,c,d) and popcounted (3 ANDs + POPC per sample and genotype).  This is the
+// computation the paper maps to binary tensor-core GEMMs; on sm_100a there is
+// no native b1 tensor op, so this pipe runs on the integer ALUs.  The fused
+// epilogue (epilogue.cuh) recovers the aa cells, scores K2 and updates the CTA's top-k list.
+//
+// CTA = 256 threads; thread (i = tid%32, jg = tid/32) owns quads (32wb+i, x, 32yb+jg+8m, z), m<4.
+#include "epilogue.cuh"
+
+namespace epi4 {
+
+constexpr int LOP3_THREADS = 256;
+constexpr int LOP3_Q = 4;   // quads per thread per tile
+
+__global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    // [0, 128 KiB): per-thread contraction counts staged for the epilogue: cnt[c][tid]
+    uint32_t* s_cnt = reinterpret_cast<uint32_t*>(smem);
+    TopKSmem tk = topk_carve(smem + sizeof(uint32_t) * 2 * LOP3_Q * 16 * LOP3_THREADS, sp.topk);
+    __shared__ long long s_tile;
+    const int tid = threadIdx.x;
+    topk_load(tk, sp, blockIdx.x, tid, LOP3_THREADS);
+    __syncthreads();
+    const DevData& d = sp.d;
+    unsigned long long my_quads = 0;
+
+    for (;;) {
+        if (tid == 0) s_tile = (long long)atomicAdd(sp.tile_counter, 1ull);
+        __syncthreads();
+        const long long tile = s_tile;
+        __syncthreads();
+        if (tile >= sp.ntiles) break;
+        const int64_t u = find_unit(sp.prefix, sp.nunits, tile);
+        const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);
+        const int32_t wb = sp.units[u].wb, x = sp.units[u].x;
+        int32_t yb, z;
+        unit_tile_decode(d.n, x, 1, t, yb, z);
+        const int i = tid & 31, jg = tid >> 5;
+        const int w = wb * EPI4_B + i;
+
+        uint32_t cnt[2][LOP3_Q][16];
+#pragma unroll
+        for (int p = 0; p < 2; ++p)
+#pragma unroll
+            for (int m = 0; m < LOP3_Q; ++m)
+#pragma unroll
+                for (int c = 0; c < 16; ++c) cnt[p][m][c] = 0;
+
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            const uint32_t* P = d.planes[p];
+            const int nch = d.nchunks[p];
+            for (int kc = 0; kc < nch; ++kc) {
+                const uint4 w0 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, w, 0, 0)));
+                const uint4 w1 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, w, 1, 0)));
+                const uint4 x0 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, x, 0, 0)));
+                const uint4 x1 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, x, 1, 0)));
+                const uint4 z0 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, z, 0, 0)));
+                const uint4 z1 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, z, 1, 0)));
+                const uint32_t wv[2][4] = {{w0.x, w0.y, w0.z, w0.w}, {w1.x, w1.y, w1.z, w1.w}};
+                const uint32_t xv[2][4] = {{x0.x, x0.y, x0.z, x0.w}, {x1.x, x1.y, x1.z, x1.w}};
+                const uint32_t zv[2][4] = {{z0.x, z0.y, z0.z, z0.w}, {z1.x, z1.y, z1.z, z1.w}};
+#pragma unroll
+                for (int m = 0; m < LOP3_Q; ++m) {
+                    const int y = yb * EPI4_B + jg + 8 * m;
+                    const uint4 y0 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, y, 0, 0)));
+                    const uint4 y1 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, y, 1, 0)));
+                    const uint32_t yv[2][4] = {{y0.x, y0.y, y0.z, y0.w}, {y1.x, y1.y, y1.z, y1.w}};
+#pragma unroll
+                    for (int wd = 0; wd < 4; ++wd) {
+                        uint32_t wx[4], yz[4];
+#pragma unroll
+                        for (int a = 0; a < 2; ++a)
+#pragma unroll
+                            for (int b = 0; b < 2; ++b) {
+                                wx[a * 2 + b] = wv[a][wd] & xv[b][wd];
+                                yz[a * 2 + b] = yv[a][wd] & zv[b][wd];
+                            }
+#pragma unroll
+                        for (int ab = 0; ab < 4; ++ab)
+#pragma unroll
+                            for (int cd = 0; cd < 4; ++cd) cnt[p][m][ab * 4 + cd] += __popc(wx[ab] & yz[cd]);
+                    }
+                }
+            }
+        }
+        // stage the counts so the epilogue's register budget is free
+#pragma unroll
+        for (int p = 0; p < 2; ++p)
+#pragma unroll
+            for (int m = 0; m < LOP3_Q; ++m)
+#pragma unroll
+                for (int c = 0; c < 16; ++c) s_cnt[((p * LOP3_Q + m) * 16 + c) * LOP3_THREADS + tid] = cnt[p][m][c];
+
+        for (int m = 0; m < LOP3_Q; ++m) {
+            const int y = yb * EPI4_B + jg + 8 * m;
+            const bool valid = (w < x) && (y > x) && (y < z);
+            double key = 0.0;
+            uint64_t idx = 0;
+            if (valid) {
+                uint32_t c0[16], c1[16];
+#pragma unroll
+                for (int c = 0; c < 16; ++c) {
+                    c0[c] = s_cnt[((0 * LOP3_Q + m) * 16 + c) * LOP3_THREADS + tid];
+                    c1[c] = s_cnt[((1 * LOP3_Q + m) * 16 + c) * LOP3_THREADS + tid];
+                }
+                uint32_t* dump = sp.dump ? sp.dump + rank4(w, x, y, z) * 162 : nullptr;
+                key = score_quad(d, w, x, y, z, c0, c1, dump);
+                idx = pack_quad(w, x, y, z);
+                ++my_quads;
+            }
+            warp_offer(tk, valid, key, idx);
+        }
+    }
+    __syncthreads();
+    topk_store(tk, sp, blockIdx.x, tid, LOP3_THREADS);
+    // useful-quad counter
+    unsigned long long v = my_quads;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((tid & 31) == 0) atomicAdd(sp.quads_done, v);
+}
+
+cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches) {
+    const size_t smem = sizeof(uint32_t) * 2 * LOP3_Q * 16 * LOP3_THREADS + topk_smem_bytes(sp.topk);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_lop3, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k_quad_lop3<<<grid, LOP3_THREADS, smem, s>>>(sp);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+}  // namespace epi4
