@@ -59,6 +59,7 @@ struct epi4_ctx {
     uint32_t* planes[2] = {nullptr, nullptr};
     uint32_t *T1 = nullptr, *T2 = nullptr, *T3 = nullptr;
     double* lgam = nullptr;
+    uint8_t* expl[2] = {nullptr, nullptr};
     // search workspace
     Unit* d_units = nullptr;
     int64_t* d_prefix = nullptr;
@@ -94,6 +95,8 @@ DevData devdata(const epi4_ctx* c) {
     d.T2 = c->T2;
     d.T3 = c->T3;
     d.lgam = c->lgam;
+    d.expl[0] = c->expl[0];
+    d.expl[1] = c->expl[1];
     return d;
 }
 
@@ -104,6 +107,8 @@ void free_data(epi4_ctx* c) {
     dfree(c->T2);
     dfree(c->T3);
     dfree(c->lgam);
+    dfree(c->expl[0]);
+    dfree(c->expl[1]);
     c->loaded = false;
 }
 
@@ -189,6 +194,10 @@ int finish_load(epi4_ctx* c) {
     CU(cudaMalloc(&c->lgam, L.size() * sizeof(double)));
     CU(cudaMemcpyAsync(c->lgam, L.data(), L.size() * sizeof(double), cudaMemcpyHostToDevice, c->stream));
     CU(cudaEventRecord(c->ev[2], c->stream));
+    for (int p = 0; p < 2; ++p) {
+        CU(cudaMalloc(&c->expl[p], (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_SAMPLES));
+        CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
+    }
     CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, c->stream, &c->stats.launches_load));
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(cudaStreamSynchronize(c->stream));

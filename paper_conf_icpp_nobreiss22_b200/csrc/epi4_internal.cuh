@@ -52,6 +52,7 @@ struct DevData {
     const uint32_t* T2;
     const uint32_t* T3;
     const double* lgam;          // M + 2 entries
+    const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
 };
 
 // offset (in uint32 words) of (chunk kc, snp, g, word w) in a chunked plane array
@@ -132,6 +133,8 @@ cudaError_t launch_retile(const uint32_t* rows, int32_t n, int64_t np, int32_t n
                           uint32_t* planes, unsigned int* status, cudaStream_t s, int64_t* launches);
 cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t npad, int32_t nchunks,
                           uint32_t* rows, cudaStream_t s, int64_t* launches);
+cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,
+                          int64_t* launches);
 cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, cudaStream_t s,
                        int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);

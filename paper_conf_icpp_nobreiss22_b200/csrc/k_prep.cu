@@ -162,6 +162,32 @@ cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t
     return cudaGetLastError();
 }
 
+// ---- {0,1}-byte expansion of the planes (operands of the i8 tensor-core pipe) ---------------------
+// expl[kc][snp][g][s] = bit s of plane (kc, snp, g); 16 output bytes per thread.
+__global__ void __launch_bounds__(256) k_expand(const uint32_t* __restrict__ planes, int64_t total16,
+                                                uint8_t* __restrict__ expl) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= total16) return;
+    const int c = (int)(t & 7);                 // 16-byte chunk of the 128-sample row
+    const int64_t rowid = t >> 3;               // (kc, snp, g)
+    const uint32_t word = planes[rowid * EPI4_CHUNK_WORDS + (c >> 1)];
+    const uint32_t half = (word >> (16 * (c & 1))) & 0xFFFFu;
+    uint32_t o[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) o[k] = (((half >> (4 * k)) & 0xFu) * 0x00204081u) & 0x01010101u;
+    reinterpret_cast<uint4*>(expl)[t] = make_uint4(o[0], o[1], o[2], o[3]);
+}
+
+cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,
+                          int64_t* launches) {
+    const int64_t total16 = (int64_t)nchunks * npad * 2 * 8;
+    if (total16 > 0) {
+        k_expand<<<(unsigned)((total16 + 255) / 256), 256, 0, s>>>(planes, total16, expl);
+        if (launches) ++*launches;
+    }
+    return cudaGetLastError();
+}
+
 // ---- lower-order tables ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_pop1(DevData d, uint32_t* __restrict__ T1) {
     const int snp = blockIdx.x * blockDim.x + threadIdx.x;
