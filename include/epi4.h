@@ -109,7 +109,7 @@ int epi4_tables(epi4_ctx* ctx, const uint64_t* quads, int64_t n, uint32_t* count
 int epi4_set_dump(epi4_ctx* ctx, uint32_t* counts_dev);
 
 /* ---- plan --------------------------------------------------------------------
- * Work unit u = (w-block, x): all quads whose first SNP lies in w-block [32*wb, 32*wb+32) and
+ * Work unit u = (w-range, x): all quads whose first SNP lies in [64*wr, 64*wr+64) and
  * whose second SNP is x.  The plan lists this rank's units (static LPT by modelled cost, identical
  * on every rank).  Host-only; usable without a GPU. */
 int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world);
@@ -127,6 +127,10 @@ typedef struct {
     int64_t launches;      /* kernels launched by the last search                  */
     int64_t launches_load; /* kernels launched by the last load                    */
     double executed_macs;  /* MACs issued by the last search's contraction (incl. padding/masking) */
+    double prof[8];        /* diagnostics: [0] exact-K2 evaluations (filter candidates); with opts.reserved[0]
+                              & 8 also summed SM cycles: [1] epilogue busy, [2] epilogue waiting for the
+                              accumulators, [3] producer busy, [4] producer waiting for TMA data,
+                              [5] MMA waiting for operands, [6] TMA waiting for a free stage */
 } epi4_stats;
 
 int epi4_get_stats(epi4_ctx* ctx, epi4_stats* out);

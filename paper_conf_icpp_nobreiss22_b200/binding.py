@@ -39,10 +39,12 @@ class epi4_stats(ctypes.Structure):
     _fields_ = [("ms_pack", ctypes.c_double), ("ms_pop", ctypes.c_double), ("ms_quad", ctypes.c_double),
                 ("ms_merge", ctypes.c_double), ("quads", ctypes.c_int64), ("tiles", ctypes.c_int64),
                 ("launches", ctypes.c_int64), ("launches_load", ctypes.c_int64),
-                ("executed_macs", ctypes.c_double)]
+                ("executed_macs", ctypes.c_double), ("prof", ctypes.c_double * 8)]
 
     def as_dict(self):
-        return {k: getattr(self, k) for k, _ in self._fields_}
+        d = {k: getattr(self, k) for k, _ in self._fields_}
+        d["prof"] = list(self.prof)
+        return d
 
 
 def _load():

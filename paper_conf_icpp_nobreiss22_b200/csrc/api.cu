@@ -44,6 +44,19 @@ void dfree(T*& p) {
     if (p) cudaFree((void*)p);
     p = nullptr;
 }
+
+// grow-only device buffer: reallocates only when a larger size is needed (loads of same-shaped
+// datasets reuse every allocation, so a step does no cudaMalloc/cudaFree)
+template <class T>
+cudaError_t grow(T*& p, size_t& cap, size_t bytes) {
+    if (bytes <= cap && p) return cudaSuccess;
+    if (p) cudaFree((void*)p);
+    p = nullptr;
+    cap = 0;
+    cudaError_t e = cudaMalloc((void**)&p, bytes ? bytes : 16);
+    if (e == cudaSuccess) cap = bytes;
+    return e;
+}
 }  // namespace
 
 struct epi4_ctx {
@@ -59,7 +72,13 @@ struct epi4_ctx {
     uint32_t* planes[2] = {nullptr, nullptr};
     uint32_t *T1 = nullptr, *T2 = nullptr, *T3 = nullptr;
     double* lgam = nullptr;
+    int32_t* lfx = nullptr;
+    int32_t lfx_shift = 0;
     uint8_t* expl[2] = {nullptr, nullptr};
+    size_t cap_planes[2] = {0, 0}, cap_T1 = 0, cap_T2 = 0, cap_T3 = 0, cap_lgam = 0, cap_lfx = 0, cap_expl[2] = {0, 0};
+    unsigned char* scratch = nullptr;     // H2D staging / pack indices
+    std::vector<double> host_L;           // lgamma(n + 1), grown on demand
+    size_t cap_scratch = 0;
     // search workspace
     Unit* d_units = nullptr;
     int64_t* d_prefix = nullptr;
@@ -97,16 +116,23 @@ DevData devdata(const epi4_ctx* c) {
     d.lgam = c->lgam;
     d.expl[0] = c->expl[0];
     d.expl[1] = c->expl[1];
+    d.lfx = c->lfx;
+    d.lfx_n = (int32_t)(c->np[0] + c->np[1] + 2);
+    d.lfx_inv_scale = std::ldexp(1.0, -c->lfx_shift);
+    // 243 table roundings of <= 1/2 unit each, plus slack for the double rounding of the exact K2
+    d.lfx_err = 122.0 * d.lfx_inv_scale + 1e-6;
     return d;
 }
 
-void free_data(epi4_ctx* c) {
+void release_data(epi4_ctx* c) {
+    dfree(c->scratch);
     dfree(c->planes[0]);
     dfree(c->planes[1]);
     dfree(c->T1);
     dfree(c->T2);
     dfree(c->T3);
     dfree(c->lgam);
+    dfree(c->lfx);
     dfree(c->expl[0]);
     dfree(c->expl[1]);
     c->loaded = false;
@@ -120,11 +146,11 @@ struct PlanEntry {
 
 std::vector<PlanEntry> all_units(int32_t n) {
     std::vector<PlanEntry> v;
-    const int32_t nb = (n + EPI4_B - 1) / EPI4_B;
-    for (int32_t wb = 0; wb < nb; ++wb)
-        for (int32_t x = wb * EPI4_B + 1; x <= n - 3; ++x) {
-            const double cost = (double)unit_tiles(n, x, 1);
-            if (cost > 0) v.push_back({{wb, x}, cost});
+    const int32_t nr = (n + EPI4_WR - 1) / EPI4_WR;
+    for (int32_t wr = 0; wr < nr; ++wr)
+        for (int32_t x = wr * EPI4_WR + 1; x <= n - 3; ++x) {
+            const double cost = (double)unit_tiles(n, x);
+            if (cost > 0) v.push_back({{wr, x}, cost});
         }
     return v;
 }
@@ -134,7 +160,7 @@ std::vector<PlanEntry> plan_rank(int32_t n, int32_t rank, int32_t world) {
     // longest processing time first; ties broken by (wb, x) so every rank computes the same plan
     std::stable_sort(v.begin(), v.end(), [](const PlanEntry& a, const PlanEntry& b) {
         if (a.cost != b.cost) return a.cost > b.cost;
-        if (a.u.wb != b.u.wb) return a.u.wb < b.u.wb;
+        if (a.u.wr != b.u.wr) return a.u.wr < b.u.wr;
         return a.u.x < b.u.x;
     });
     if (world <= 1) return v;
@@ -178,24 +204,43 @@ int finish_load(epi4_ctx* c) {
     if (st & EPI4_ST_AA_AND_Aa) return fail(EPI4_EINVAL, "a sample has both AA and Aa bits set");
     // lower-order tables
     const int64_t n = c->n;
-    CU(cudaMalloc(&c->T1, (size_t)n * 4 * sizeof(uint32_t)));
-    CU(cudaMalloc(&c->T2, (size_t)c2(n) * 8 * sizeof(uint32_t)));
+    CU(grow(c->T1, c->cap_T1, (size_t)n * 4 * sizeof(uint32_t)));
+    CU(grow(c->T2, c->cap_T2, (size_t)c2(n) * 8 * sizeof(uint32_t)));
     const size_t t3b = (size_t)c3(n) * 16 * sizeof(uint32_t);
     size_t freeb = 0, totb = 0;
     CU(cudaMemGetInfo(&freeb, &totb));
-    if (t3b + ((size_t)1 << 30) > freeb)
+    if (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
         return fail(EPI4_ENOMEM, "3-way tables need %.1f GB but only %.1f GB of HBM are free (N=%d); "
                     "the windowed T3 path for larger N is not built yet", t3b / 1e9, freeb / 1e9, c->n);
-    CU(cudaMalloc(&c->T3, t3b));
+    CU(grow(c->T3, c->cap_T3, t3b));
     // lgamma table L[k] = lgamma(k + 1) for k in [0, M + 1]
     const int64_t m = c->np[0] + c->np[1];
-    std::vector<double> L((size_t)m + 2);
-    for (int64_t k = 0; k < m + 2; ++k) L[(size_t)k] = std::lgamma((double)k + 1.0);
-    CU(cudaMalloc(&c->lgam, L.size() * sizeof(double)));
-    CU(cudaMemcpyAsync(c->lgam, L.data(), L.size() * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+    std::vector<double>& L = c->host_L;
+    const size_t have = L.size();
+    if (have < (size_t)m + 2) {
+        L.resize((size_t)m + 2);
+        for (size_t k = have; k < L.size(); ++k) L[k] = std::lgamma((double)k + 1.0);
+    }
+    CU(grow(c->lgam, c->cap_lgam, ((size_t)m + 2) * sizeof(double)));
+    CU(cudaMemcpyAsync(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+    // fixed-point copy for the K2 filter: every entry and every K2 (<= L[M + 81], superadditivity of
+    // log n!) must fit in int32 -> shift s = floor(log2((2^31 - 1) / L[M + 81]))
+    {
+        const double kmax = std::lgamma((double)(m + 81) + 1.0);
+        int s = 0;
+        while (s < 30 && std::ldexp(kmax, s + 1) < 2147483647.0) ++s;
+        c->lfx_shift = s;
+        std::vector<int32_t> F((size_t)m + 2);
+        for (size_t k = 0; k < F.size(); ++k) F[k] = (int32_t)std::llrint(std::ldexp(L[k], s));
+        // the double table must be resident before the async copies complete: both copies are
+        // stream-ordered and we synchronize below, so the host vectors outlive them
+        CU(grow(c->lfx, c->cap_lfx, F.size() * sizeof(int32_t)));
+        CU(cudaMemcpyAsync(c->lfx, F.data(), F.size() * sizeof(int32_t), cudaMemcpyHostToDevice, c->stream));
+        CU(cudaStreamSynchronize(c->stream));
+    }
     CU(cudaEventRecord(c->ev[2], c->stream));
     for (int p = 0; p < 2; ++p) {
-        CU(cudaMalloc(&c->expl[p], (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_SAMPLES));
+        CU(grow(c->expl[p], c->cap_expl[p], (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_SAMPLES));
         CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
     }
     CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, c->stream, &c->stats.launches_load));
@@ -209,15 +254,15 @@ int finish_load(epi4_ctx* c) {
 }
 
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
-    free_data(c);
+    c->loaded = false;
     c->n = n;
-    c->npad = (n + EPI4_B - 1) / EPI4_B * EPI4_B;
+    c->npad = (n + EPI4_YR + EPI4_WR - 1) / EPI4_WR * EPI4_WR;
     c->np[0] = n0;
     c->np[1] = n1;
     for (int p = 0; p < 2; ++p) {
         c->nchunks[p] = (int32_t)((c->np[p] + EPI4_CHUNK_SAMPLES - 1) / EPI4_CHUNK_SAMPLES);
         const size_t words = (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_WORDS;
-        CU(cudaMalloc(&c->planes[p], words * sizeof(uint32_t)));
+        CU(grow(c->planes[p], c->cap_planes[p], words * sizeof(uint32_t)));
         CU(cudaMemsetAsync(c->planes[p], 0, words * sizeof(uint32_t), c->stream));
     }
     CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
@@ -277,7 +322,7 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
     c->sm_count = prop.multiProcessorCount;
     cudaError_t e = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaMalloc(&c->d_status, sizeof(unsigned int));
-    if (e == cudaSuccess) e = cudaMalloc(&c->d_counters, 4 * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc(&c->d_counters, 32 * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_k2, EPI4_MAX_TOPK * sizeof(double));
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_idx, EPI4_MAX_TOPK * sizeof(uint64_t));
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_n, sizeof(int32_t));
@@ -295,7 +340,7 @@ void epi4_destroy(epi4_ctx* c) {
     if (!c) return;
     cudaSetDevice(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
-    free_data(c);
+    release_data(c);
     dfree(c->d_units);
     dfree(c->d_prefix);
     dfree(c->d_counters);
@@ -328,24 +373,20 @@ int epi4_load_bits(epi4_ctx* c, const uint32_t* pc, const uint32_t* pk, int32_t 
     if (int r = alloc_planes(c, n_snps, n0, n1)) return r;
     CU(cudaEventRecord(c->ev[0], c->stream));
     const uint32_t* src[2] = {pc, pk};
+    if (ptr_kind != EPI4_PTR_HOST && ptr_kind != EPI4_PTR_DEVICE) return fail(EPI4_EINVAL, "ptr_kind %d", ptr_kind);
+    const size_t words0 = (size_t)2 * n_snps * (size_t)((c->np[0] + 31) / 32);
+    const size_t words1 = (size_t)2 * n_snps * (size_t)((c->np[1] + 31) / 32);
+    if (ptr_kind == EPI4_PTR_HOST) CU(grow(c->scratch, c->cap_scratch, (words0 + words1) * sizeof(uint32_t)));
     for (int p = 0; p < 2; ++p) {
-        const size_t words = (size_t)2 * n_snps * (size_t)((c->np[p] + 31) / 32);
+        const size_t words = p ? words1 : words0;
         const uint32_t* rows = src[p];
-        uint32_t* tmp = nullptr;
         if (ptr_kind == EPI4_PTR_HOST) {
-            CU(cudaMalloc(&tmp, words * sizeof(uint32_t)));
+            uint32_t* tmp = reinterpret_cast<uint32_t*>(c->scratch) + (p ? words0 : 0);
             CU(cudaMemcpyAsync(tmp, src[p], words * sizeof(uint32_t), cudaMemcpyHostToDevice, c->stream));
             rows = tmp;
-        } else if (ptr_kind != EPI4_PTR_DEVICE) {
-            return fail(EPI4_EINVAL, "ptr_kind %d", ptr_kind);
         }
-        cudaError_t e = launch_retile(rows, n_snps, c->np[p], c->npad, c->nchunks[p], c->planes[p], c->d_status,
-                                      c->stream, &c->stats.launches_load);
-        if (tmp) {
-            cudaStreamSynchronize(c->stream);
-            cudaFree(tmp);
-        }
-        CU(e);
+        CU(launch_retile(rows, n_snps, c->np[p], c->npad, c->nchunks[p], c->planes[p], c->d_status, c->stream,
+                         &c->stats.launches_load));
     }
     CU(cudaEventRecord(c->ev[1], c->stream));
     int r = finish_load(c);
@@ -365,18 +406,20 @@ int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, i
     CU(cudaSetDevice(c->device));
     c->stats.launches_load = 0;
     const uint8_t *dg = geno, *dp = phen;
-    uint8_t *tg = nullptr, *tp = nullptr;
-    int32_t* idx = nullptr;   // [m] (idx0 then idx1) + 2 counts
+    // scratch: [pack indices (2m+2) int32][genotypes n*m][phenotypes m] (the last two only for host input)
+    const size_t idx_bytes = ((size_t)(2 * m + 2) * sizeof(int32_t) + 255) & ~(size_t)255;
+    const size_t gbytes = ptr_kind == EPI4_PTR_HOST ? (((size_t)n_snps * m + 255) & ~(size_t)255) + (size_t)m : 0;
+    CU(grow(c->scratch, c->cap_scratch, idx_bytes + gbytes));
+    int32_t* idx = reinterpret_cast<int32_t*>(c->scratch);   // [m] (idx0 then idx1) + 2 counts
     CU(cudaEventRecord(c->ev[0], c->stream));
     if (ptr_kind == EPI4_PTR_HOST) {
-        CU(cudaMalloc(&tg, (size_t)n_snps * m));
-        CU(cudaMalloc(&tp, (size_t)m));
+        uint8_t* tg = c->scratch + idx_bytes;
+        uint8_t* tp = tg + (((size_t)n_snps * m + 255) & ~(size_t)255);
         CU(cudaMemcpyAsync(tg, geno, (size_t)n_snps * m, cudaMemcpyHostToDevice, c->stream));
         CU(cudaMemcpyAsync(tp, phen, (size_t)m, cudaMemcpyHostToDevice, c->stream));
         dg = tg;
         dp = tp;
     }
-    CU(cudaMalloc(&idx, (size_t)(2 * m + 2) * sizeof(int32_t)));
     CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
     // pass 1: split by phenotype (idx0 at [0, m), idx1 at [m, 2m), counts at [2m, 2m+2))
     CU(launch_split_phen(dp, m, idx, idx + m, idx + 2 * m, c->d_status, c->stream, &c->stats.launches_load));
@@ -398,9 +441,6 @@ int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, i
     }
     cudaEventRecord(c->ev[1], c->stream);
     cudaStreamSynchronize(c->stream);
-    cudaFree(idx);
-    if (tg) cudaFree(tg);
-    if (tp) cudaFree(tp);
     if (r) return r;
     r = finish_load(c);
     float ms = 0;
@@ -446,7 +486,7 @@ int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* out, d
         return fail(EPI4_EINVAL, "bad plan arguments");
     std::vector<PlanEntry> v = plan_rank(n_snps, rank, world);
     for (size_t i = 0; i < v.size(); ++i) {
-        out[2 * i] = v[i].u.wb;
+        out[2 * i] = v[i].u.wr;
         out[2 * i + 1] = v[i].u.x;
         if (cost_out) cost_out[i] = v[i].cost;
     }
@@ -466,13 +506,13 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (ub < 0) ub = 0;
     if (ub > ue) ub = ue;
     const int64_t nu = ue - ub;
-    const int32_t zt = quad_zt(c->opts.pipe);
+    const int32_t G = quad_group(c->opts.pipe);
     std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
     std::vector<int64_t> prefix((size_t)std::max<int64_t>(nu, 1));
     int64_t acc = 0;
     for (int64_t i = 0; i < nu; ++i) {
         units[(size_t)i] = plan[(size_t)(ub + i)].u;
-        acc += unit_tiles(c->n, units[(size_t)i].x, zt);
+        acc += unit_tiles(c->n, units[(size_t)i].x, G);
         prefix[(size_t)i] = acc;
     }
     if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
@@ -486,10 +526,11 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
         CU(cudaMemcpyAsync(c->d_units, units.data(), nu * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
         CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), nu * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
     }
-    const int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
+    int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
+    grid = std::max(G, grid / G * G);                 // whole clusters
     if (int r = ensure_lists(c, grid, top_k)) return r;
     CU(cudaMemsetAsync(c->d_list_cnt, 0, (size_t)grid * sizeof(int32_t), c->stream));
-    CU(cudaMemsetAsync(c->d_counters, 0, 4 * sizeof(unsigned long long), c->stream));
+    CU(cudaMemsetAsync(c->d_counters, 0, 32 * sizeof(unsigned long long), c->stream));
     CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
 
     SearchParams sp;
@@ -498,7 +539,6 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.prefix = c->d_prefix;
     sp.nunits = nu;
     sp.ntiles = acc;
-    sp.zt = zt;
     sp.tile_counter = c->d_counters;
     sp.topk = top_k;
     sp.list_k2 = c->d_list_k2;
@@ -507,6 +547,10 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.dump = c->dump;
     sp.status = c->d_status;
     sp.quads_done = c->d_counters + 1;
+    sp.prof = c->d_counters + 16;
+    sp.use_lfx = 0;
+    sp.group = G;
+    sp.debug = c->opts.reserved[0];
 
     c->stats.launches = 0;
     CU(cudaEventRecord(c->ev[2], c->stream));
@@ -518,7 +562,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(launch_merge(sp, grid, c->d_out_k2, c->d_out_idx, c->d_out_n, c->stream, &c->stats.launches));
     int32_t nout = 0;
-    unsigned long long ctr[2] = {0, 0};
+    unsigned long long ctr[32] = {0};
     CU(cudaMemcpyAsync(&nout, c->d_out_n, sizeof nout, cudaMemcpyDeviceToHost, c->stream));
     CU(cudaMemcpyAsync(quads_out, c->d_out_idx, (size_t)top_k * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
     CU(cudaMemcpyAsync(k2_out, c->d_out_k2, (size_t)top_k * sizeof(double), cudaMemcpyDeviceToHost, c->stream));
@@ -531,8 +575,9 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaEventElapsedTime(&ms, c->ev[3], c->ev[4]));
     c->stats.ms_merge = ms;
     c->stats.quads = (int64_t)ctr[1];
-    c->stats.tiles = acc;
-    c->stats.executed_macs = (double)acc * 1024.0 * 16.0 * zt * (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
+    for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)ctr[16 + i];
+    c->stats.tiles = acc * G;
+    c->stats.executed_macs = (double)acc * G * 1024.0 * 16.0 * (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
     *n_out = nout;
     return 0;
 }

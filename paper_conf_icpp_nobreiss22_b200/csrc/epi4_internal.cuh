@@ -1,9 +1,13 @@
 // epi4_internal.cuh — internal declarations shared by the libepi4 translation units.
 //
 // Device data layout in HBM:
-//   planes[p]  : uint32, chunked K-major: [chunk kc][snp (padded to 32)][g = 0 AA, 1 Aa][4 words]
+//   planes[p]  : uint32, chunked K-major: [chunk kc][snp (padded, see npad)][g = 0 AA, 1 Aa][4 words]
 //                one chunk = 128 samples of phenotype p; pad bits are 0 (PAPER.md:L66-68 encoding,
-//                re-tiled so that the 32 SNPs of a block are 1 KiB contiguous per chunk).
+//                re-tiled so that consecutive SNPs are contiguous per chunk).
+//   expl[p]    : uint8 {0,1}, the same planes expanded to one byte per sample, [chunk][row r = 2 snp + g]
+//                [128 bytes] with the UMMA 128-byte swizzle applied in HBM (16-byte piece c of row r stored
+//                at piece c ^ (r & 7)), so a linear bulk copy of 8-row-aligned rows lands in the canonical
+//                K-major SW128 shared-memory layout.
 //   T1[snp][p][2]          popc(P_a(snp))                              (PAPER.md:L85 indivPop)
 //   T2[rank2][p][4]        popc(P_a(i) & P_b(j)), i<j, cell 2a+b       (PAPER.md:L86 pairwPop)
 //   T3[rank3][p][8]        popc(P_a(i) & P_b(j) & P_c(k)), i<j<k, cell 4a+2b+c
@@ -15,7 +19,9 @@
 
 #include "../../include/epi4.h"
 
-#define EPI4_B 32             // SNP block size (32-SNP blocks)
+#define EPI4_B 32             // SNP block size accepted in epi4_opts (32-SNP blocks)
+#define EPI4_WR 64            // w-range of a work unit / rows of the A operand: 64 SNPs x {AA, Aa}
+#define EPI4_YR 16            // y-range of a tile: 16 consecutive SNPs after x
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
 
@@ -46,13 +52,17 @@ struct DevData {
     const uint32_t* planes[2];   // chunked planes per phenotype
     int32_t nchunks[2];          // chunks per phenotype
     int32_t n;                   // SNPs
-    int32_t npad;                // SNPs padded to a multiple of 32 (row count of a chunk / 2)
+    int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
     uint32_t np[2];              // n0, n1
     const uint32_t* T1;
     const uint32_t* T2;
     const uint32_t* T3;
     const double* lgam;          // M + 2 entries
     const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
+    const int32_t* lfx;          // fixed-point lgamma table round(L[n] * 2^lfx_shift), M + 2 entries
+    int32_t lfx_n;
+    double lfx_inv_scale;        // 2^-lfx_shift
+    double lfx_err;              // bound on |acc * 2^-s - K2| (filter slack)
 };
 
 // offset (in uint32 words) of (chunk kc, snp, g, word w) in a chunked plane array
@@ -60,37 +70,33 @@ __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, 
     return ((kc * npad + snp) * 2 + g) * EPI4_CHUNK_WORDS + w;
 }
 
-// A work unit (wb, x): quads with w in block wb (w < x), second SNP x, any y < z after x.
+// A work unit (wr, x): the quads (w, x, y, z) with w in the 64-SNP range [64 wr, 64 wr + 64), w < x,
+// second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + 16) with
+// y0 = x + 1 + 16k, and z in (y0, n); a tile holds 64 x 16 = 1024 (w, y) combinations.
 struct Unit {
-    int32_t wb, x;
+    int32_t wr, x;
 };
 
-// number of tiles of unit (wb,x) when a tile covers ZT consecutive z values:
-// tiles iterate y-blocks yb >= (x+1)/32 and z in [max(x+2, 32*yb+1), n)
-__host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x, int32_t zt) {
+// Tiles are scheduled in groups of G consecutive z of the same (unit, y0) (G = the cluster size of the
+// tensor-core kernel, 1 for the CUDA-core kernel); a group's last members may be past n (dummy tiles).
+__host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x, int32_t G = 1) {
     int64_t t = 0;
-    int32_t nb = (n + EPI4_B - 1) / EPI4_B;
-    for (int32_t yb = (x + 1) / EPI4_B; yb < nb; ++yb) {
-        int32_t zlo = max(x + 2, yb * EPI4_B + 1);
-        if (zlo < n) t += (n - zlo + zt - 1) / zt;
-    }
+    for (int32_t y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) t += (n - y0 - 1 + G - 1) / G;
     return t;
 }
 
-// decode tile t of unit (x) -> (yb, z0)
-__device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int32_t zt, int64_t t, int32_t& yb,
-                                                 int32_t& z0) {
-    int32_t nb = (n + EPI4_B - 1) / EPI4_B;
-    for (yb = (x + 1) / EPI4_B; yb < nb; ++yb) {
-        int32_t zlo = max(x + 2, yb * EPI4_B + 1);
-        int64_t cnt = (zlo < n) ? (n - zlo + zt - 1) / zt : 0;
+// decode group t of unit (x) -> (y0, first z of the group)
+__device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t, int32_t& y0, int32_t& z,
+                                                 int32_t G = 1) {
+    for (y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) {
+        const int64_t cnt = (n - y0 - 1 + G - 1) / G;
         if (t < cnt) {
-            z0 = zlo + (int32_t)t * zt;
+            z = y0 + 1 + (int32_t)t * G;
             return;
         }
         t -= cnt;
     }
-    z0 = n;  // unreachable for valid t
+    z = n;  // unreachable for valid t
 }
 
 // find the unit of a flat tile index by binary search on the inclusive prefix of tile counts
@@ -110,7 +116,6 @@ struct SearchParams {
     const int64_t* prefix;     // inclusive prefix of tiles per unit
     int64_t nunits;
     int64_t ntiles;
-    int32_t zt;                // z values per tile
     unsigned long long* tile_counter;   // dynamic scheduler
     int32_t topk;              // list capacity used (<= EPI4_MAX_TOPK)
     double* list_k2;           // per-CTA lists [grid][topk]
@@ -119,6 +124,10 @@ struct SearchParams {
     uint32_t* dump;            // optional 162 counts per quad indexed by rank4 (NULL = off)
     unsigned int* status;
     unsigned long long* quads_done;   // useful quads evaluated (atomicAdd once per CTA)
+    unsigned long long* prof;  // [16] diagnostics: [0] exact K2 evaluations, [1..] per-role cycle counters
+    int32_t use_lfx;           // fixed-point K2 filter table resident in shared memory
+    int32_t group;             // tiles per scheduling group (= cluster size of the tensor-core kernel)
+    int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA
 };
 
 }  // namespace epi4
@@ -139,7 +148,7 @@ cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T
                        int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_i8tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
-int32_t quad_zt(int32_t pipe);
+int32_t quad_group(int32_t pipe);
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,
                          int32_t* out_n, cudaStream_t s, int64_t* launches);
 cudaError_t launch_tables(const DevData& d, const uint64_t* quads, int64_t n, uint32_t* out, unsigned int* status,

@@ -1,6 +1,7 @@
 // epilogue.cuh — the fused per-quad epilogue shared by every contraction kernel (step a6/a7 of
 // SURVEY.md §8(a)):
-//   (1) assemble the 81 "generalized" counts of a quad w<x<y<z for one phenotype: index
+//   (1) assemble the 81 "generalized" counts of a quad w<x<y<z for one phenotype (in three slabs of 27
+//       along the first SNP, see quad_eval): index
 //       27α+9β+3γ+δ with α..δ in {0 = AA, 1 = Aa, 2 = '*' (any genotype)}:
 //         no '*'     -> the 16 counts of the 4-way contraction
 //         one '*'    -> 3-way tables T3 of the other three SNPs
@@ -20,131 +21,153 @@
 
 namespace epi4 {
 
-// lower-order values of one quad (w<x<y<z) for both phenotypes
-struct LowOrder {
-    uint32_t t3[2][4][8];   // [p][wxy, wxz, wyz, xyz][4a+2b+c]
-    uint32_t t2[2][6][4];   // [p][wx, wy, wz, xy, xz, yz][2a+b]
-    uint32_t t1[2][4][2];   // [p][w, x, y, z][a]
-};
+// ---- lower-order table access (both phenotypes of an entry are adjacent) ----------------------------
+// T3 entry of (i<j<k): 16 uint32 = [p][4a+2b+c];  T2 entry of (i<j): 8 uint32 = [p][2a+b];  T1[snp]: [p][a].
+__device__ __forceinline__ uint4 t3_half(const DevData& d, int i, int j, int k, int p, int a) {
+    // the 4 cells with first genotype a of phenotype p
+    return __ldg(reinterpret_cast<const uint4*>(d.T3 + rank3(i, j, k) * 16 + p * 8 + a * 4));
+}
+__device__ __forceinline__ uint2 t2_row(const DevData& d, int i, int j, int p, int a) {
+    return __ldg(reinterpret_cast<const uint2*>(d.T2 + rank2(i, j) * 8 + p * 4 + a * 2));
+}
+__device__ __forceinline__ uint4 t2_all(const DevData& d, int i, int j, int p) {
+    return __ldg(reinterpret_cast<const uint4*>(d.T2 + rank2(i, j) * 8 + p * 4));
+}
+__device__ __forceinline__ uint2 t1_all(const DevData& d, int i, int p) {
+    return __ldg(reinterpret_cast<const uint2*>(d.T1 + (int64_t)i * 4 + p * 2));
+}
+__device__ __forceinline__ uint32_t u4(const uint4& v, int k) { return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w; }
+__device__ __forceinline__ uint32_t u2(const uint2& v, int k) { return k == 0 ? v.x : v.y; }
 
-__device__ __forceinline__ void load8(const uint32_t* p, uint32_t (&v)[8]) {
-    uint4 a = __ldg(reinterpret_cast<const uint4*>(p));
-    uint4 b = __ldg(reinterpret_cast<const uint4*>(p) + 1);
-    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
-}
-__device__ __forceinline__ void load4(const uint32_t* p, uint32_t (&v)[4]) {
-    uint4 a = __ldg(reinterpret_cast<const uint4*>(p));
-    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
-}
-__device__ __forceinline__ void load_t3(const DevData& d, int i, int j, int k, int slot, LowOrder& lo) {
-    const uint32_t* p = d.T3 + rank3(i, j, k) * 16;
-    load8(p, lo.t3[0][slot]);
-    load8(p + 8, lo.t3[1][slot]);
-}
-__device__ __forceinline__ void load_t2(const DevData& d, int i, int j, int slot, LowOrder& lo) {
-    const uint32_t* p = d.T2 + rank2(i, j) * 8;
-    load4(p, lo.t2[0][slot]);
-    load4(p + 4, lo.t2[1][slot]);
-}
-__device__ __forceinline__ void load_t1(const DevData& d, int i, int slot, LowOrder& lo) {
-    const uint32_t* p = d.T1 + (int64_t)i * 4;
-    uint4 a = __ldg(reinterpret_cast<const uint4*>(p));
-    lo.t1[0][slot][0] = a.x; lo.t1[0][slot][1] = a.y; lo.t1[1][slot][0] = a.z; lo.t1[1][slot][1] = a.w;
-}
-__device__ __forceinline__ void load_low(const DevData& d, int w, int x, int y, int z, LowOrder& lo) {
-    load_t3(d, w, x, y, 0, lo);
-    load_t3(d, w, x, z, 1, lo);
-    load_t3(d, w, y, z, 2, lo);
-    load_t3(d, x, y, z, 3, lo);
-    load_t2(d, w, x, 0, lo);
-    load_t2(d, w, y, 1, lo);
-    load_t2(d, w, z, 2, lo);
-    load_t2(d, x, y, 3, lo);
-    load_t2(d, x, z, 4, lo);
-    load_t2(d, y, z, 5, lo);
-    load_t1(d, w, 0, lo);
-    load_t1(d, x, 1, lo);
-    load_t1(d, y, 2, lo);
-    load_t1(d, z, 3, lo);
-}
-
-// (1) generalized counts of phenotype p; c16[8a+4b+2c+d] = 4-way counts with a..d in {0,1}
+// Slab decomposition along the first SNP (w) of the quad.  For α in {0, 1, '*'} the slab
+// S_α[β][γ][δ] = G[α][β][γ][δ] holds 27 generalized counts (digits in {0, 1, 2 = '*'}):
+//   slab '*' (w marginalised): T3(x,y,z), T2 of (x,y),(x,z),(y,z), T1 of x,y,z and n_p;
+//   slab α in {0,1}:           the 4-way counts c16[α...], T3 of (w,x,y),(w,x,z),(w,y,z), T2 of (w,.),
+//                              T1(w) — all restricted to genotype α of w.
+// Möbius on the remaining three axes gives the cells r[α][...] for α = 0, 1; and, because the
+// recovery is linear, r[2][...] = M3(S_*) - M3(S_0) - M3(S_1)  (PAPER.md:L126 applied on axis w).
+// Cells therefore come out a-major, i.e. in canonical order c = 27a + 9b + 3c + d.
 template <int P>
-__device__ __forceinline__ void fill_generalized(int (&g)[81], const uint32_t (&c16)[16], const LowOrder& lo,
-                                                 uint32_t np) {
+__device__ __forceinline__ void fill_slab_star(int (&g)[27], const DevData& d, int x, int y, int z) {
+    const uint4 txyz0 = t3_half(d, x, y, z, P, 0), txyz1 = t3_half(d, x, y, z, P, 1);
+    const uint4 pxy = t2_all(d, x, y, P), pxz = t2_all(d, x, z, P), pyz = t2_all(d, y, z, P);
+    const uint2 sx = t1_all(d, x, P), sy = t1_all(d, y, P), sz = t1_all(d, z, P);
 #pragma unroll
-    for (int c = 0; c < 81; ++c) {
-        const int a = c / 27, b = (c / 9) % 3, e = (c / 3) % 3, f = c % 3;
-        const int ns = (a == 2) + (b == 2) + (e == 2) + (f == 2);
+    for (int c = 0; c < 27; ++c) {
+        const int b = c / 9, e = (c / 3) % 3, f = c % 3;
+        const int ns = (b == 2) + (e == 2) + (f == 2);
         uint32_t v;
-        if (ns == 0) {
-            v = c16[a * 8 + b * 4 + e * 2 + f];
-        } else if (ns == 1) {
-            if (f == 2) v = lo.t3[P][0][a * 4 + b * 2 + e];        // (w,x,y)
-            else if (e == 2) v = lo.t3[P][1][a * 4 + b * 2 + f];   // (w,x,z)
-            else if (b == 2) v = lo.t3[P][2][a * 4 + e * 2 + f];   // (w,y,z)
-            else v = lo.t3[P][3][b * 4 + e * 2 + f];               // (x,y,z)
+        if (ns == 0) v = b ? u4(txyz1, e * 2 + f) : u4(txyz0, e * 2 + f);
+        else if (ns == 1) {
+            if (f == 2) v = u4(pxy, b * 2 + e);
+            else if (e == 2) v = u4(pxz, b * 2 + f);
+            else v = u4(pyz, e * 2 + f);
         } else if (ns == 2) {
-            if (e == 2 && f == 2) v = lo.t2[P][0][a * 2 + b];      // (w,x)
-            else if (b == 2 && f == 2) v = lo.t2[P][1][a * 2 + e]; // (w,y)
-            else if (b == 2 && e == 2) v = lo.t2[P][2][a * 2 + f]; // (w,z)
-            else if (a == 2 && f == 2) v = lo.t2[P][3][b * 2 + e]; // (x,y)
-            else if (a == 2 && e == 2) v = lo.t2[P][4][b * 2 + f]; // (x,z)
-            else v = lo.t2[P][5][e * 2 + f];                       // (y,z)
-        } else if (ns == 3) {
-            if (a != 2) v = lo.t1[P][0][a];
-            else if (b != 2) v = lo.t1[P][1][b];
-            else if (e != 2) v = lo.t1[P][2][e];
-            else v = lo.t1[P][3][f];
+            if (b != 2) v = u2(sx, b);
+            else if (e != 2) v = u2(sy, e);
+            else v = u2(sz, f);
         } else {
-            v = np;
+            v = d.np[P];
+        }
+        g[c] = (int)v;
+    }
+}
+template <int P, int A>
+__device__ __forceinline__ void fill_slab_w(int (&g)[27], const uint32_t (&c16)[16], const DevData& d, int w, int x,
+                                            int y, int z) {
+    const uint4 twxy = t3_half(d, w, x, y, P, A), twxz = t3_half(d, w, x, z, P, A), twyz = t3_half(d, w, y, z, P, A);
+    const uint2 pwx = t2_row(d, w, x, P, A), pwy = t2_row(d, w, y, P, A), pwz = t2_row(d, w, z, P, A);
+    const uint2 sw = t1_all(d, w, P);
+#pragma unroll
+    for (int c = 0; c < 27; ++c) {
+        const int b = c / 9, e = (c / 3) % 3, f = c % 3;
+        const int ns = (b == 2) + (e == 2) + (f == 2);
+        uint32_t v;
+        if (ns == 0) v = c16[A * 8 + b * 4 + e * 2 + f];
+        else if (ns == 1) {
+            if (f == 2) v = u4(twxy, b * 2 + e);
+            else if (e == 2) v = u4(twxz, b * 2 + f);
+            else v = u4(twyz, e * 2 + f);
+        } else if (ns == 2) {
+            if (b != 2) v = u2(pwx, b);
+            else if (e != 2) v = u2(pwy, e);
+            else v = u2(pwz, f);
+        } else {
+            v = u2(sw, A);
         }
         g[c] = (int)v;
     }
 }
 
-// (2) aa recovery, axis by axis (216 subtractions)
-__device__ __forceinline__ void mobius(int (&g)[81]) {
+// aa recovery on the three axes of a slab (strides 9, 3, 1): 3 x 9 x 2 = 54 subtractions
+__device__ __forceinline__ void mobius3(int (&g)[27]) {
 #pragma unroll
-    for (int ax = 0; ax < 4; ++ax) {
-        const int s = ax == 0 ? 27 : ax == 1 ? 9 : ax == 2 ? 3 : 1;
+    for (int ax = 0; ax < 3; ++ax) {
+        const int s = ax == 0 ? 9 : ax == 1 ? 3 : 1;
 #pragma unroll
-        for (int c = 0; c < 81; ++c)
+        for (int c = 0; c < 27; ++c)
             if (((c / s) % 3) == 2) g[c] = g[c] - g[c - s] - g[c - 2 * s];
     }
 }
 
-// (3) K2 in canonical order; explicit round-to-nearest adds so nothing can be reassociated
-__device__ __forceinline__ double k2_score(const int (&g0)[81], const int (&g1)[81], const double* __restrict__ L) {
-    double k2 = 0.0;
+// Per-quad evaluation in canonical cell order.  FIX: fixed-point K2 filter sum with the smem table
+// lfx; DBL: exact K2 in double, t_c = (L[r+1] - L[r0]) - L[r1], K2 += t_c, c = 0..80
+// (reading #4); DUMP: write the 2 x 81 cells (controls first).
+template <bool FIX, bool DBL, bool DUMP>
+__device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y, int z, const uint32_t (&c0)[16],
+                                          const uint32_t (&c1)[16], const int32_t* lfx, uint32_t& acc, double& k2,
+                                          uint32_t* dump) {
+    int R0[27], R1[27];
+    fill_slab_star<0>(R0, d, x, y, z);
+    fill_slab_star<1>(R1, d, x, y, z);
+    mobius3(R0);
+    mobius3(R1);
+    uint32_t a0 = 0, a1 = 0;
+    double kk = 0.0;
+    auto consume = [&](const int (&T0)[27], const int (&T1)[27], int base) {
 #pragma unroll
-    for (int c = 0; c < 81; ++c) {
-        const int r0 = g0[c], r1 = g1[c];
-        const double t = __dsub_rn(__dsub_rn(__ldg(L + (r0 + r1 + 1)), __ldg(L + r0)), __ldg(L + r1));
-        k2 = __dadd_rn(k2, t);
+        for (int c = 0; c < 27; ++c) {
+            const int r0 = T0[c], r1 = T1[c];
+            if (FIX) {
+                const uint32_t t = (uint32_t)lfx[r0 + r1 + 1] - (uint32_t)lfx[r0] - (uint32_t)lfx[r1];
+                if (c & 1) a1 += t; else a0 += t;
+            }
+            if (DBL) {
+                const double t = __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1));
+                kk = __dadd_rn(kk, t);
+            }
+            if (DUMP) {
+                dump[base + c] = (uint32_t)r0;
+                dump[81 + base + c] = (uint32_t)r1;
+            }
+        }
+    };
+#pragma unroll
+    for (int a = 0; a < 2; ++a) {
+        int T0[27], T1[27];
+        if (a == 0) { fill_slab_w<0, 0>(T0, c0, d, w, x, y, z); fill_slab_w<1, 0>(T1, c1, d, w, x, y, z); }
+        else        { fill_slab_w<0, 1>(T0, c0, d, w, x, y, z); fill_slab_w<1, 1>(T1, c1, d, w, x, y, z); }
+        mobius3(T0);
+        mobius3(T1);
+        consume(T0, T1, 27 * a);
+#pragma unroll
+        for (int c = 0; c < 27; ++c) { R0[c] -= T0[c]; R1[c] -= T1[c]; }
     }
-    return k2;
+    consume(R0, R1, 54);
+    acc = a0 + a1;
+    k2 = kk;
 }
 
-// full epilogue for one quad given its 2 x 16 contraction counts; optionally dumps the 162 counts
-__device__ __forceinline__ double score_quad(const DevData& d, int w, int x, int y, int z,
-                                             const uint32_t (&c0)[16], const uint32_t (&c1)[16],
-                                             uint32_t* dump_row) {
-    LowOrder lo;
-    load_low(d, w, x, y, z, lo);
-    int g0[81], g1[81];
-    fill_generalized<0>(g0, c0, lo, d.np[0]);
-    fill_generalized<1>(g1, c1, lo, d.np[1]);
-    mobius(g0);
-    mobius(g1);
-    if (dump_row) {
-#pragma unroll
-        for (int c = 0; c < 81; ++c) {
-            dump_row[c] = (uint32_t)g0[c];
-            dump_row[81 + c] = (uint32_t)g1[c];
-        }
-    }
-    return k2_score(g0, g1, d.lgam);
+// exact K2 of one quad (double, canonical order); optionally dumps its 162 cells.  Not inlined: in the
+// tensor-core epilogue it runs only for filter candidates, so its registers must not add to the hot loop's.
+static __device__ __noinline__ double score_quad(const DevData& d, int w, int x, int y, int z,
+                                          const uint32_t (&c0)[16], const uint32_t (&c1)[16],
+                                          uint32_t* dump_row) {
+    uint32_t acc;
+    double k2;
+    if (dump_row) quad_eval<false, true, true>(d, w, x, y, z, c0, c1, nullptr, acc, k2, dump_row);
+    else quad_eval<false, true, false>(d, w, x, y, z, c0, c1, nullptr, acc, k2, nullptr);
+    return k2;
 }
 
 // ---------------------------------------------------------------------------------------------

@@ -163,19 +163,21 @@ cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t
 }
 
 // ---- {0,1}-byte expansion of the planes (operands of the i8 tensor-core pipe) ---------------------
-// expl[kc][snp][g][s] = bit s of plane (kc, snp, g); 16 output bytes per thread.
+// expl[kc][r = 2 snp + g][128 B]: byte s of row r = bit s of plane (kc, snp, g); 16-byte piece c stored
+// at piece c ^ (r & 7) (UMMA SW128 pattern, rows are 128 B so the 8-row groups are 1 KiB aligned).
 __global__ void __launch_bounds__(256) k_expand(const uint32_t* __restrict__ planes, int64_t total16,
                                                 uint8_t* __restrict__ expl) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= total16) return;
-    const int c = (int)(t & 7);                 // 16-byte chunk of the 128-sample row
-    const int64_t rowid = t >> 3;               // (kc, snp, g)
+    const int c = (int)(t & 7);                 // 16-byte piece of the 128-sample row
+    const int64_t rowid = t >> 3;               // (kc, snp, g) = (kc, r)
     const uint32_t word = planes[rowid * EPI4_CHUNK_WORDS + (c >> 1)];
     const uint32_t half = (word >> (16 * (c & 1))) & 0xFFFFu;
     uint32_t o[4];
 #pragma unroll
     for (int k = 0; k < 4; ++k) o[k] = (((half >> (4 * k)) & 0xFu) * 0x00204081u) & 0x01010101u;
-    reinterpret_cast<uint4*>(expl)[t] = make_uint4(o[0], o[1], o[2], o[3]);
+    const int sw = c ^ (int)(rowid & 7);
+    reinterpret_cast<uint4*>(expl)[rowid * 8 + sw] = make_uint4(o[0], o[1], o[2], o[3]);
 }
 
 cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,

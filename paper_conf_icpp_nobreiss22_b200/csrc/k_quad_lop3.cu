@@ -1,6 +1,6 @@
 // k_quad_lop3.cu — CUDA-core contraction (EPI4_PIPE_LOP3): AND + POPC on bit planes.
 //
-// The cross-check pipe of SURVEY.md §8(a) a5: for each tile (w-block wb, x, y-block yb, z) the 32 x 32
+// The cross-check pipe of SURVEY.md §8(a) a5: for each tile (w-range wr, x, y-range y0, z) the 64 x 16
 // (w, y) combinations are counted directly: for each 32-sample word, the pair rows
 // (w,x,a,b) = P_a(w) & P_b(x) ("combine") are ANDed with the pair columns
 // (y,z,c,d) and popcounted (3 ANDs + POPC per sample and genotype).  This is the
@@ -8,7 +8,7 @@
 // no native b1 tensor op, so this pipe runs on the integer ALUs.  The fused
 // epilogue (epilogue.cuh) recovers the aa cells, scores K2 and updates the CTA's top-k list.
 //
-// CTA = 256 threads; thread (i = tid%32, jg = tid/32) owns quads (32wb+i, x, 32yb+jg+8m, z), m<4.
+// CTA = 256 threads; thread (i = tid%64, jg = tid/64) owns quads (64wr+i, x, y0+jg+4m, z), m<4.
 #include "epilogue.cuh"
 
 namespace epi4 {
@@ -36,11 +36,11 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
         if (tile >= sp.ntiles) break;
         const int64_t u = find_unit(sp.prefix, sp.nunits, tile);
         const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);
-        const int32_t wb = sp.units[u].wb, x = sp.units[u].x;
-        int32_t yb, z;
-        unit_tile_decode(d.n, x, 1, t, yb, z);
-        const int i = tid & 31, jg = tid >> 5;
-        const int w = wb * EPI4_B + i;
+        const int32_t wr = sp.units[u].wr, x = sp.units[u].x;
+        int32_t y0, z;
+        unit_tile_decode(d.n, x, t, y0, z, 1);
+        const int i = tid & 63, jg = tid >> 6;
+        const int w = wr * EPI4_WR + i;
 
         uint32_t cnt[2][LOP3_Q][16];
 #pragma unroll
@@ -66,10 +66,10 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
                 const uint32_t zv[2][4] = {{z0.x, z0.y, z0.z, z0.w}, {z1.x, z1.y, z1.z, z1.w}};
 #pragma unroll
                 for (int m = 0; m < LOP3_Q; ++m) {
-                    const int y = yb * EPI4_B + jg + 8 * m;
-                    const uint4 y0 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, y, 0, 0)));
-                    const uint4 y1 = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, y, 1, 0)));
-                    const uint32_t yv[2][4] = {{y0.x, y0.y, y0.z, y0.w}, {y1.x, y1.y, y1.z, y1.w}};
+                    const int y = y0 + jg + 4 * m;
+                    const uint4 ya = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, y, 0, 0)));
+                    const uint4 yb = __ldg(reinterpret_cast<const uint4*>(P + plane_off(kc, d.npad, y, 1, 0)));
+                    const uint32_t yv[2][4] = {{ya.x, ya.y, ya.z, ya.w}, {yb.x, yb.y, yb.z, yb.w}};
 #pragma unroll
                     for (int wd = 0; wd < 4; ++wd) {
                         uint32_t wx[4], yz[4];
@@ -97,7 +97,7 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
                 for (int c = 0; c < 16; ++c) s_cnt[((p * LOP3_Q + m) * 16 + c) * LOP3_THREADS + tid] = cnt[p][m][c];
 
         for (int m = 0; m < LOP3_Q; ++m) {
-            const int y = yb * EPI4_B + jg + 8 * m;
+            const int y = y0 + jg + 4 * m;
             const bool valid = (w < x) && (y > x) && (y < z);
             double key = 0.0;
             uint64_t idx = 0;

@@ -1,27 +1,28 @@
 // k_quad_tc.cu — the hot kernel: 4-way contraction on the 5th-generation tensor cores
 // (tcgen05.mma kind::i8, {0,1} operands, s32 accumulators in TMEM) with the fused epilogue.
 //
-// What it computes: for a tile (w-block wb, x, y-block yb, z) the
-// 128 x 128 matrix C_p[(w,x,a,b)][(y,z,c,d)] = sum over samples s of phenotype p of
-// P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]   — the 16 non-aa genotype counts of the 32 x 32 quads
-// (w, x, y, z), for controls and for cases (tensorOp_4way, "a matrix with 16
-// values per each quad").  Rows are pair products of the w-block with x and columns pair products of
-// the y-block with z (the paper's `combine`), built on chip.
+// What it computes: for a tile (w-range wr, x, y-range y0, z) and each
+// phenotype p the 128 x 128 matrix
+//     C_p[(w, a)][(y, b, c, d)] = sum over samples s of phenotype p of P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]
+// for the 64 SNPs w of the range and the 16 SNPs y = y0..y0+15: the 16 non-aa genotype counts of the
+// 64 x 16 quads (w, x, y, z) ("a matrix with 16 values per each quad").
+// Factorisation: the paper ANDs SNP pairs into both operands (combine);
+// here the A operand is the raw single-SNP planes (w, a) — copied from HBM by the TMA engine, no on-chip
+// production at all — and x is folded into the B operand, whose columns are triple products
+// P_b(x) & P_c(y) & P_d(z) built by two producer warps.  This halves the operand bytes that must be written
+// by threads (the LSU was the bottleneck of pair x pair tiles).
+// Why i8: sm_100a has no native binary tensor op (ptxas emulates mma.sync ...b1.and.popc with legacy IMMA,
+// SURVEY.md App. C); AND+POPC becomes an integer MAC on {0,1} bytes, exact in s32.
 //
-// Why i8: sm_100a has no native binary (b1) tensor op — ptxas emulates
-// mma.sync ...b1.and.popc with legacy IMMA — so the AND+POPC of the paper becomes an
-// integer MAC on {0,1} bytes: AND(a,b) = a*b and POPC = the K-sum, exact in s32.
-//
-// Warp roles (CTA = 8 warps, 1 CTA per SM, persistent, static tile stride):
-//   warp 0      : TMEM allocation (512 columns) + one elected thread issuing tcgen05.mma
-//   warps 1..3  : producers — per 128-sample chunk, AND the pre-expanded {0,1} byte planes of the single
-//                 SNPs into the A (pair rows) and B (pair columns) tiles, stored K-major with the 128-byte
-//                 swizzle (UMMA canonical SW128 layout), then fence.proxy.async + mbarrier arrive
-//   warps 4..7  : epilogue — tcgen05.ld the control and case accumulators, 4x4 lane transposes so that
-//                 one thread holds one quad's 2 x 16 counts, then the shared epilogue (aa recovery,
-//                 K2 in double, top-k; epilogue.cuh)
-// Pipelines: smem ring of STAGES x (A 16 KiB + B 16 KiB) (full/empty mbarriers); TMEM double buffer
-// (2 x [128 ctrl | 128 case] columns) between MMA and epilogue (tmem_full/tmem_empty mbarriers).
+// Warp roles (CTA = 12 warps, 1 CTA per SM, persistent, static tile stride):
+//   warp 0      : TMEM allocation (512 columns) + one thread running a non-blocking event loop that issues
+//                 the TMA bulk copies of a stage (A: 64 SNPs x 2 planes x 128 samples = 16 KiB, pre-swizzled
+//                 in HBM; the 16 y planes, x and z) and the tcgen05.mma of ready stages
+//   warps 1..3  : producers — B[(y,b,c,d)] = x_b & z_d & y_c per 16-byte piece, stored K-major SW128
+//   warps 4..11 : epilogue — tcgen05.ld of the control and case accumulators, pairwise lane exchange so one
+//                 thread holds one quad's 2 x 16 counts, then the shared epilogue (epilogue.cuh)
+// Pipelines: STAGES x {A, B, singles} (sfull: TMA bytes landed, full: B produced, empty: MMA done);
+// TMEM double buffer (2 x [128 ctrl | 128 case] columns) between MMA and epilogue.
 #include "epilogue.cuh"
 
 namespace epi4 {
@@ -29,11 +30,21 @@ namespace epi4 {
 namespace tc {
 constexpr int M = 128, N = 128;          // UMMA shape (cta_group::1), K = 32 bytes per instruction
 constexpr int KCH = EPI4_CHUNK_SAMPLES;  // 128 samples (bytes) per pipeline stage
-constexpr int STAGES = 4;
-constexpr int A_BYTES = M * KCH, B_BYTES = N * KCH, STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int PROD_WARPS = 3, EPI_WARPS = 4;
-constexpr int THREADS = 32 * (1 + PROD_WARPS + EPI_WARPS);
+constexpr int A_BYTES = M * KCH, B_BYTES = N * KCH;
+constexpr int SY_OFF = A_BYTES + B_BYTES, SY_BYTES = 2 * EPI4_YR * KCH;   // 16 y SNPs x 2 planes
+constexpr int SX_OFF = SY_OFF + SY_BYTES, SZ_OFF = SX_OFF + 2 * KCH;
+constexpr int STAGE_BYTES = ((SZ_OFF + 2 * KCH) + 1023) / 1024 * 1024;
+constexpr int TX_BYTES = A_BYTES + SY_BYTES + 4 * KCH;                      // bytes the TMA brings per stage
+// warp 0: MMA issuer; warp 1: TMA issuer; warps 2-3: producers (alternating stages); warps 4-11:
+// epilogue.  384 threads keep 168 registers per thread (above 384 ptxas drops to 128).
+constexpr int PROD_WARPS = 2, EPI_WARPS = 8;
+constexpr int PROD_WARP0 = 2, EPI_WARP0 = 4;
+constexpr int PROD_THREADS = 32 * PROD_WARPS;
+constexpr int THREADS = 384;
 constexpr int TMEM_COLS = 512;
+constexpr int CLUSTER = 2;                 // CTAs sharing A, the y slab and x through TMA multicast
+                                           // (2 packs all 148 SMs; 4 strands SMs of the 18-SM GPCs)
+constexpr int SHARED_TX = A_BYTES + SY_BYTES + 2 * KCH;   // multicast by the cluster leader
 // instruction descriptor: D s32 (bits 4-5 = 2), A/B u8 (0), K-major, N>>3 at bit 17, M>>4 at bit 24
 constexpr uint32_t IDESC = (2u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }  // namespace tc
@@ -50,6 +61,15 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
         "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok)
         : "r"(smem_u32(bar)), "r"(parity)
         : "memory");
@@ -129,35 +149,109 @@ __device__ __forceinline__ void quad_transpose(const uint32_t (&v)[16], uint32_t
         }
 }
 
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_id_x() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t nclusters_x() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%nclusterid.x;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 struct TileInfo {
-    int32_t wb, x, yb, z;
+    int32_t wr, x, y0, z;
 };
-__device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t tile) {
-    const int64_t u = find_unit(sp.prefix, sp.nunits, tile);
-    const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);
+// group -> this CTA's tile: the cluster's CTA of rank r takes z = first z of the group + r (>= n: dummy)
+__device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t group) {
+    const int64_t u = find_unit(sp.prefix, sp.nunits, group);
+    const int64_t t = group - (u ? sp.prefix[u - 1] : 0);
     TileInfo ti;
-    ti.wb = sp.units[u].wb;
+    ti.wr = sp.units[u].wr;
     ti.x = sp.units[u].x;
-    unit_tile_decode(sp.d.n, ti.x, 1, t, ti.yb, ti.z);
+    unit_tile_decode(sp.d.n, ti.x, t, ti.y0, ti.z, tc::CLUSTER);
+    ti.z += (int32_t)cluster_rank();
     return ti;
 }
 
+// iterator over the (tile, phenotype, chunk) steps of this CTA
+struct StepIt {
+    int64_t tile;
+    TileInfo ti;
+    int p, kc;
+    __device__ __forceinline__ void init(const SearchParams& sp) {
+        tile = cluster_id_x();
+        p = 0;
+        kc = 0;
+        if (tile < sp.ntiles) ti = decode_tile(sp, tile);
+    }
+    __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
+    __device__ __forceinline__ void next(const SearchParams& sp) {
+        if (++kc == sp.d.nchunks[p]) {
+            kc = 0;
+            if (++p == 2) {
+                p = 0;
+                tile += nclusters_x();
+                if (tile < sp.ntiles) ti = decode_tile(sp, tile);
+            }
+        }
+    }
+};
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t tx) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(tx) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s_mc(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint16_t mask) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "h"(mask)
+        : "memory");
+}
+// arrive (when this thread's prior MMAs complete) on the same-offset mbarrier of every CTA in `mask`
+__device__ __forceinline__ void mma_commit_mc(uint64_t* bar, uint16_t mask) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                     smem_u32(bar)),
+                 "h"(mask)
+                 : "memory");
+}
+
+template <int STAGES>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
     extern __shared__ unsigned char smem_raw[];
-    __shared__ __align__(8) uint64_t full_bar[tc::STAGES], empty_bar[tc::STAGES];
+    __shared__ __align__(8) uint64_t sfull_bar[STAGES], full_bar[STAGES], empty_bar[STAGES];
     __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2];
     __shared__ uint32_t s_tmem;
-    // 1024-aligned operand ring, then the top-k state
+    // 1024-aligned stage ring, then the fixed-point lgamma table, then the top-k state
     const uint32_t raw = smem_u32(smem_raw);
     unsigned char* ring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-    TopKSmem tk = topk_carve(ring + tc::STAGES * tc::STAGE_BYTES, sp.topk);
+    int32_t* s_lfx = reinterpret_cast<int32_t*>(ring + STAGES * tc::STAGE_BYTES);
+    const int lfx_words = sp.use_lfx ? ((sp.d.lfx_n + 3) & ~3) : 0;
+    TopKSmem tk = topk_carve(reinterpret_cast<unsigned char*>(s_lfx + lfx_words), sp.topk);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const DevData& d = sp.d;
     if (tid == 0) {
-        for (int s = 0; s < tc::STAGES; ++s) {
-            mbar_init(&full_bar[s], tc::PROD_WARPS);
-            mbar_init(&empty_bar[s], 1);
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(&sfull_bar[s], 1);
+            mbar_init(&full_bar[s], 1);          // one producer warp builds a stage's B tile
+            mbar_init(&empty_bar[s], tc::CLUSTER);   // every CTA's MMA must release a stage
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&tfull_bar[b], 1);
@@ -171,11 +265,15 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);
+    for (int e = tid; e < lfx_words; e += tc::THREADS) s_lfx[e] = e < d.lfx_n ? __ldg(d.lfx + e) : 0;
     tc_fence_before();
-    __syncthreads();
+    cluster_sync_all();                  // barrier inits visible cluster-wide before any multicast
     tc_fence_after();
+    const bool leader = cluster_rank() == 0;
+    const uint16_t cmask = (uint16_t)((1u << tc::CLUSTER) - 1);
+    const int64_t first_group = cluster_id_x(), group_stride = nclusters_x();
     const uint32_t tmem = s_tmem;
-    const int nch0 = d.nchunks[0], nch1 = d.nchunks[1];
+    const int64_t chunk_stride = (int64_t)d.npad * 2 * tc::KCH;   // bytes of one chunk of expl
 
     if (warp == 0) {
         // ===================== MMA issuer =====================
@@ -183,7 +281,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
             int stage = 0;
             uint32_t phase = 0;
             int it = 0;
-            for (int64_t tile = blockIdx.x; tile < sp.ntiles; tile += gridDim.x, ++it) {
+            const bool timing = (sp.debug & 8) != 0;
+            long long t_wait = 0;
+            for (int64_t tile = first_group; tile < sp.ntiles; tile += group_stride, ++it) {
                 const int buf = it & 1;
                 const uint32_t tphase = (uint32_t)((it >> 1) & 1);
                 mbar_wait(&tempty_bar[buf], tphase ^ 1u);   // epilogue drained this buffer
@@ -191,128 +291,264 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
                     const uint32_t dcol = tmem + (uint32_t)(buf * 256 + p * 128);
-                    const int nch = p ? nch1 : nch0;
+                    const int nch = d.nchunks[p];
                     for (int kc = 0; kc < nch; ++kc) {
+                        const long long t0 = timing ? clock64() : 0;
+                        mbar_wait(&sfull_bar[stage], phase);
                         mbar_wait(&full_bar[stage], phase);
+                        if (timing) t_wait += clock64() - t0;
                         tc_fence_after();
                         const uint32_t a0 = smem_u32(ring + stage * tc::STAGE_BYTES);
                         const uint32_t b0 = a0 + tc::A_BYTES;
+                        if (!(sp.debug & 4)) {
 #pragma unroll
-                        for (int k = 0; k < tc::KCH / 32; ++k)
-                            mma_i8(dcol, sw128_desc(a0 + 32 * k), sw128_desc(b0 + 32 * k), (kc | k) != 0);
-                        mma_commit(&empty_bar[stage]);          // frees the smem slot when these MMAs finish
-                        if (++stage == tc::STAGES) { stage = 0; phase ^= 1u; }
+                            for (int k = 0; k < tc::KCH / 32; ++k)
+                                mma_i8(dcol, sw128_desc(a0 + 32 * k), sw128_desc(b0 + 32 * k), (kc | k) != 0);
+                        }
+                        mma_commit_mc(&empty_bar[stage], cmask);  // frees the stage in every CTA of the cluster
+                        if (++stage == STAGES) { stage = 0; phase ^= 1u; }
                     }
                 }
                 mma_commit(&tfull_bar[buf]);                    // accumulators of this tile are ready
             }
+            if (timing) atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
         }
         __syncwarp();
-    } else if (warp <= tc::PROD_WARPS) {
-        // ===================== producers =====================
-        const int pt = tid - 32;                  // 0..95
-        const int c = pt & 7;                     // 16-byte chunk of the 128-byte K row (fixed per thread)
-        const int u0 = pt >> 3;                   // 0..11
-        int stage = 0;
-        uint32_t phase = 0;
-        for (int64_t tile = blockIdx.x; tile < sp.ntiles; tile += gridDim.x) {
-            const TileInfo ti = decode_tile(sp, tile);
-#pragma unroll 1
-            for (int p = 0; p < 2; ++p) {
-                const uint8_t* E = d.expl[p];
-                const int nch = p ? nch1 : nch0;
-                for (int kc = 0; kc < nch; ++kc) {
-                    mbar_wait(&empty_bar[stage], phase ^ 1u);
-                    unsigned char* sa = ring + stage * tc::STAGE_BYTES;
-                    unsigned char* sb = sa + tc::A_BYTES;
-                    const uint8_t* Ek = E + (int64_t)kc * d.npad * 2 * tc::KCH;
-                    const uint4 x0 = __ldg(reinterpret_cast<const uint4*>(Ek + (ti.x * 2 + 0) * tc::KCH) + c);
-                    const uint4 x1 = __ldg(reinterpret_cast<const uint4*>(Ek + (ti.x * 2 + 1) * tc::KCH) + c);
-                    const uint4 z0 = __ldg(reinterpret_cast<const uint4*>(Ek + (ti.z * 2 + 0) * tc::KCH) + c);
-                    const uint4 z1 = __ldg(reinterpret_cast<const uint4*>(Ek + (ti.z * 2 + 1) * tc::KCH) + c);
-#pragma unroll 2
-                    for (int ua = u0; ua < 64; ua += 12) {
-                        // A unit (i, a) -> rows i*4 + a*2 + b; B unit (j, cc) -> columns j*4 + cc*2 + dd
-                        const int i = ua >> 1, a = ua & 1;
-                        const uint4 wv = __ldg(reinterpret_cast<const uint4*>(Ek + ((ti.wb * EPI4_B + i) * 2 + a) * tc::KCH) + c);
-                        const uint4 yv = __ldg(reinterpret_cast<const uint4*>(Ek + ((ti.yb * EPI4_B + i) * 2 + a) * tc::KCH) + c);
-                        const int r0 = i * 4 + a * 2;
-                        *reinterpret_cast<uint4*>(sa + sw128_off(r0, c)) = and4(wv, x0);
-                        *reinterpret_cast<uint4*>(sa + sw128_off(r0 + 1, c)) = and4(wv, x1);
-                        *reinterpret_cast<uint4*>(sb + sw128_off(r0, c)) = and4(yv, z0);
-                        *reinterpret_cast<uint4*>(sb + sw128_off(r0 + 1, c)) = and4(yv, z1);
-                    }
-                    fence_proxy_async();                  // generic-proxy stores -> visible to the tensor core
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&full_bar[stage]);
-                    if (++stage == tc::STAGES) { stage = 0; phase ^= 1u; }
+    } else if (warp == 1) {
+        // ===================== TMA issuer =====================
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t phase = 0;
+            StepIt st;
+            st.init(sp);
+            const bool timing = (sp.debug & 8) != 0;
+            long long t_wait = 0;
+            for (; st.valid(sp); st.next(sp)) {
+                const long long t0 = timing ? clock64() : 0;
+                mbar_wait(&empty_bar[stage], phase ^ 1u);
+                if (timing) t_wait += clock64() - t0;
+                unsigned char* sbase = ring + stage * tc::STAGE_BYTES;
+                const uint8_t* E = d.expl[st.p] + (int64_t)st.kc * chunk_stride;
+                mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
+                if (leader) {
+                    // A, the y slab and x are the same for the whole cluster: one L2 read, multicast
+                    bulk_g2s_mc(sbase, E + (int64_t)st.ti.wr * EPI4_WR * 2 * tc::KCH, tc::A_BYTES, &sfull_bar[stage], cmask);
+                    bulk_g2s_mc(sbase + tc::SY_OFF, E + (int64_t)st.ti.y0 * 2 * tc::KCH, tc::SY_BYTES, &sfull_bar[stage], cmask);
+                    bulk_g2s_mc(sbase + tc::SX_OFF, E + (int64_t)st.ti.x * 2 * tc::KCH, 2 * tc::KCH, &sfull_bar[stage], cmask);
                 }
+                const int zc = st.ti.z < d.n ? st.ti.z : d.n - 1;   // dummy tile: any valid row
+                bulk_g2s(sbase + tc::SZ_OFF, E + (int64_t)zc * 2 * tc::KCH, 2 * tc::KCH, &sfull_bar[stage]);
+                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
             }
+            if (timing) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
         }
-    } else {
+        __syncwarp();
+    } else if (warp >= tc::PROD_WARP0 && warp < tc::PROD_WARP0 + tc::PROD_WARPS) {
+        // ===================== producers =====================
+        // Producer warp j builds the whole B tile of every step s with s % PROD_WARPS == j, so the warps'
+        // per-stage latencies (shared loads, fence.proxy.async, barrier arrive) overlap.  Lane: 16-byte
+        // piece cc = lane & 7 of the 128-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k.
+        // B[n = 8 y_local + 4b + 2c + d] = x_b & z_d & y_c (rows of smem singles keep the HBM swizzle:
+        // piece cc of absolute row r sits at piece cc ^ (r & 7)).
+        const int pw = warp - tc::PROD_WARP0;
+        const int cc = lane & 7;
+        const int cpl = (lane >> 3) & 1;
+        const bool skip = (sp.debug & 1) != 0;
+        StepIt st;
+        st.init(sp);
+        const bool timing = (sp.debug & 8) != 0;
+        long long t_wait = 0, t_busy = 0;
+        for (int64_t step = 0; st.valid(sp); st.next(sp), ++step) {
+            if ((int)(step % tc::PROD_WARPS) != pw) continue;
+            const int stage = (int)(step % STAGES);
+            const uint32_t phase = (uint32_t)((step / STAGES) & 1);
+            const long long t0 = timing ? clock64() : 0;
+            mbar_wait(&sfull_bar[stage], phase);
+            const long long t1 = timing ? clock64() : 0;
+            t_wait += t1 - t0;
+            if (!skip) {
+                unsigned char* sbase = ring + stage * tc::STAGE_BYTES;
+                unsigned char* sb = sbase + tc::A_BYTES;
+                const int x = st.ti.x, z = st.ti.z, y0 = st.ti.y0;
+                const uint4 x0 = *reinterpret_cast<const uint4*>(sbase + tc::SX_OFF + ((cc ^ ((2 * x) & 7)) << 4));
+                const uint4 x1 = *reinterpret_cast<const uint4*>(sbase + tc::SX_OFF + 128 + ((cc ^ ((2 * x + 1) & 7)) << 4));
+                const uint4 z0 = *reinterpret_cast<const uint4*>(sbase + tc::SZ_OFF + ((cc ^ ((2 * z) & 7)) << 4));
+                const uint4 z1 = *reinterpret_cast<const uint4*>(sbase + tc::SZ_OFF + 128 + ((cc ^ ((2 * z + 1) & 7)) << 4));
+                const uint4 xz[4] = {and4(x0, z0), and4(x0, z1), and4(x1, z0), and4(x1, z1)};   // [b*2 + d]
+                uint4 yv[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int rr = 2 * ((lane >> 4) + 2 * k) + cpl;        // row inside the y slab
+                    const int ra = 2 * y0 + rr;                            // absolute row (for the swizzle)
+                    yv[k] = *reinterpret_cast<const uint4*>(sbase + tc::SY_OFF + rr * 128 + ((cc ^ (ra & 7)) << 4));
+                }
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int yl = (lane >> 4) + 2 * k;
+#pragma unroll
+                    for (int bd = 0; bd < 4; ++bd) {
+                        const int n = yl * 8 + (bd >> 1) * 4 + cpl * 2 + (bd & 1);
+                        *reinterpret_cast<uint4*>(sb + sw128_off(n, cc)) = and4(yv[k], xz[bd]);
+                    }
+                }
+                fence_proxy_async();                      // generic-proxy stores -> visible to the tensor core
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&full_bar[stage]);
+            if (timing) t_busy += clock64() - t1;
+        }
+        if (timing && lane == 0) {
+            atomicAdd(sp.prof + 3, (unsigned long long)t_busy);
+            atomicAdd(sp.prof + 4, (unsigned long long)t_wait);
+        }
+    } else if (warp >= tc::EPI_WARP0) {
         // ===================== epilogue =====================
-        const int q = warp & 3;                   // TMEM lane quadrant this warp may access
-        const int row = q * 32 + lane;            // = i*4 + ab
-        const int i = row >> 2, t = row & 3;
-        unsigned long long my_quads = 0;
+        // lane quadrant q holds rows 32q..32q+31 = (w_local, a) with w_local = row/2; a 16-column group g
+        // holds y_local = 2g, 2g+1 x (b, c, d).  Lanes a=0/a=1 swap halves so that lane a owns the quad
+        // y_local = 2g + a with all 16 counts c16[8a' + 4b + 2c + d].
+        const int ew = warp - tc::EPI_WARP0;           // 0..7
+        const int q = warp & 3;                         // TMEM lane quadrant this warp may access
+        const int h = ew >> 2;                          // two warps per quadrant split the column groups
+        const int row = q * 32 + lane;
+        const int wl = row >> 1, a = row & 1;
+        unsigned long long my_quads = 0, n_exact = 0;
+        long long t_wait = 0, t_busy = 0;
+        const bool timing = (sp.debug & 8) != 0;
         int it = 0;
-        for (int64_t tile = blockIdx.x; tile < sp.ntiles; tile += gridDim.x, ++it) {
+        for (int64_t tile = first_group; tile < sp.ntiles; tile += group_stride, ++it) {
             const TileInfo ti = decode_tile(sp, tile);
             const int buf = it & 1;
             const uint32_t tphase = (uint32_t)((it >> 1) & 1);
+            const long long t0 = timing ? clock64() : 0;
             mbar_wait(&tfull_bar[buf], tphase);
+            const long long t1 = timing ? clock64() : 0;
+            t_wait += t1 - t0;
             tc_fence_after();
-            const int w = ti.wb * EPI4_B + i;
+            const int w = ti.wr * EPI4_WR + wl;
             const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * 256);
 #pragma unroll 1
-            for (int g = 0; g < 8; ++g) {
+            for (int g = h; g < 8; g += 2) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(tbase + 16 * g, v0);
                 tmem_ld16(tbase + 128 + 16 * g, v1);
                 tmem_wait_ld();
-                if (g == 7) {
+                if (g + 2 >= 8) {
                     tc_fence_before();
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&tempty_bar[buf]);
                 }
                 uint32_t c0[16], c1[16];
-                quad_transpose(v0, c0);
-                quad_transpose(v1, c1);
-                const int y = ti.yb * EPI4_B + 4 * g + t;
-                const bool valid = (w < ti.x) && (ti.x < y) && (y < ti.z);
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    // send my values for the other lane's quad, keep mine
+                    const uint32_t s0 = a ? v0[k] : v0[8 + k], s1 = a ? v1[k] : v1[8 + k];
+                    const uint32_t r0 = __shfl_xor_sync(0xffffffffu, s0, 1);
+                    const uint32_t r1 = __shfl_xor_sync(0xffffffffu, s1, 1);
+                    // lane a keeps c16[8a + k] = its own v[8a + k] and takes c16[8(1-a) + k] from the partner
+                    c0[k] = a ? r0 : v0[k];
+                    c0[8 + k] = a ? v0[8 + k] : r0;
+                    c1[k] = a ? r1 : v1[k];
+                    c1[8 + k] = a ? v1[8 + k] : r1;
+                }
+                const int y = ti.y0 + 2 * g + a;
+                const bool valid = (w < ti.x) && (y < ti.z) && (ti.z < d.n) && !(sp.debug & 2);
                 double key = 0.0;
                 uint64_t idx = 0;
+                bool offer = false;
                 if (valid) {
                     uint32_t* dump = sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
-                    key = score_quad(d, w, ti.x, y, ti.z, c0, c1, dump);
+                    offer = true;
+                    if (dump) {
+                        key = score_quad(d, w, ti.x, y, ti.z, c0, c1, dump);
+                    } else if (sp.use_lfx) {
+                        // exact-bounded fixed-point filter; only possible top-k members get the exact K2
+                        uint32_t acc;
+                        double dummy;
+                        quad_eval<true, false, false>(d, w, ti.x, y, ti.z, c0, c1, s_lfx, acc, dummy, nullptr);
+                        const double thr = *reinterpret_cast<volatile double*>(tk.thr);
+                        offer = (double)(int32_t)acc * d.lfx_inv_scale - d.lfx_err <= thr;
+                        if (offer) {
+                            key = score_quad(d, w, ti.x, y, ti.z, c0, c1, nullptr);
+                            ++n_exact;
+                        }
+                    } else {
+                        key = score_quad(d, w, ti.x, y, ti.z, c0, c1, nullptr);
+                    }
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;
                 }
-                warp_offer(tk, valid, key, idx);
+                warp_offer(tk, offer, key, idx);
+            }
+            if (timing) t_busy += clock64() - t1;
+        }
+        unsigned long long v = my_quads, ne = n_exact;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            v += __shfl_xor_sync(0xffffffffu, v, o);
+            ne += __shfl_xor_sync(0xffffffffu, ne, o);
+        }
+        if (lane == 0) {
+            atomicAdd(sp.quads_done, v);
+            atomicAdd(sp.prof + 0, ne);
+            if (timing) {
+                atomicAdd(sp.prof + 1, (unsigned long long)t_busy);
+                atomicAdd(sp.prof + 2, (unsigned long long)t_wait);
             }
         }
-        unsigned long long v = my_quads;
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        if (lane == 0) atomicAdd(sp.quads_done, v);
     }
     tc_fence_before();
-    __syncthreads();
+    cluster_sync_all();                  // no CTA leaves while cluster peers may still signal it
     tc_fence_after();
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tc::TMEM_COLS));
     topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
 }
 
-int32_t quad_zt(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? 1 : 1; }
-
-cudaError_t launch_quad_i8tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches) {
-    const size_t smem = 1024 + (size_t)tc::STAGES * tc::STAGE_BYTES + topk_smem_bytes(sp.topk);
-    cudaError_t e = cudaFuncSetAttribute(k_quad_i8tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+template <int STAGES>
+static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
+    cudaError_t e = cudaFuncSetAttribute(k_quad_i8tc<STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    k_quad_i8tc<<<grid, tc::THREADS, smem, s>>>(sp);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(tc::THREADS);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = tc::CLUSTER;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_quad_i8tc<STAGES>, sp);
+}
+
+int32_t quad_group(int32_t pipe) { return pipe == EPI4_PIPE_I8TC ? tc::CLUSTER : 1; }
+
+cudaError_t launch_quad_i8tc(const SearchParams& sp_in, int32_t grid, cudaStream_t s, int64_t* launches) {
+    SearchParams sp = sp_in;
+    grid = grid / tc::CLUSTER * tc::CLUSTER;
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024;   // alignment + static smem slack
+    const size_t lfx_bytes = (size_t)((sp.d.lfx_n + 3) & ~3) * sizeof(int32_t);
+    // most pipeline stages that fit; the fixed-point K2 filter table in smem is preferred, falling back to
+    // exact-only scoring when it cannot fit with at least 2 stages
+    int st = 0;
+    for (int pass = 0; pass < 2 && !st; ++pass) {
+        sp.use_lfx = pass == 0 && sp.d.lfx != nullptr && !(sp.debug & 16);   // debug 16: no table, more stages
+        for (int cand = 5; cand >= 2 && !st; --cand)
+            if (fixed + (size_t)cand * tc::STAGE_BYTES + (sp.use_lfx ? lfx_bytes : 0) <= (size_t)optin) st = cand;
+    }
+    if (!st) return cudaErrorInvalidConfiguration;
+    const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + (sp.use_lfx ? lfx_bytes : 0) + topk_smem_bytes(sp.topk);
+    cudaError_t e = st == 5 ? launch_cfg<5>(sp, smem, grid, s)
+                  : st == 4 ? launch_cfg<4>(sp, smem, grid, s)
+                  : st == 3 ? launch_cfg<3>(sp, smem, grid, s)
+                            : launch_cfg<2>(sp, smem, grid, s);
     if (launches) ++*launches;
-    return cudaGetLastError();
+    return e;
 }
 
 }  // namespace epi4
