@@ -37,14 +37,19 @@ constexpr int STAGE_BYTES = ((SZ_OFF + 2 * KCH) + 1023) / 1024 * 1024;
 constexpr int TX_BYTES = A_BYTES + SY_BYTES + 4 * KCH;                      // bytes the TMA brings per stage
 // warp 0: MMA issuer; warp 1: TMA issuer; warps 2-3: producers (alternating stages); warps 4-11:
 // epilogue.  384 threads keep 168 registers per thread (above 384 ptxas drops to 128).
-constexpr int PROD_WARPS = 2, EPI_WARPS = 8;
-constexpr int PROD_WARP0 = 2, EPI_WARP0 = 4;
-constexpr int PROD_THREADS = 32 * PROD_WARPS;
-constexpr int THREADS = 384;
+#ifndef EPI4_TC_PROD_WARPS
+#define EPI4_TC_PROD_WARPS 2
+#endif
+#ifndef EPI4_TC_EPI_WARPS
+#define EPI4_TC_EPI_WARPS 8
+#endif
+constexpr int PROD_WARPS = EPI4_TC_PROD_WARPS, EPI_WARPS = EPI4_TC_EPI_WARPS;   // EPI_WARPS: 4 or 8
+constexpr int PROD_WARP0 = 2, EPI_WARP0 = 2 + PROD_WARPS;
+constexpr int THREADS = 32 * (2 + PROD_WARPS + EPI_WARPS);
+constexpr int EPI_SPLIT = EPI_WARPS / 4;   // warps per TMEM lane quadrant (they alternate 16-column groups)
 constexpr int TMEM_COLS = 512;
 constexpr int CLUSTER = 2;                 // CTAs sharing A, the y slab and x through TMA multicast
                                            // (2 packs all 148 SMs; 4 strands SMs of the 18-SM GPCs)
-constexpr int SHARED_TX = A_BYTES + SY_BYTES + 2 * KCH;   // multicast by the cluster leader
 // instruction descriptor: D s32 (bits 4-5 = 2), A/B u8 (0), K-major, N>>3 at bit 17, M>>4 at bit 24
 constexpr uint32_t IDESC = (2u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }  // namespace tc
@@ -345,11 +350,14 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         __syncwarp();
     } else if (warp >= tc::PROD_WARP0 && warp < tc::PROD_WARP0 + tc::PROD_WARPS) {
         // ===================== producers =====================
-        // Producer warp j builds the whole B tile of every step s with s % PROD_WARPS == j, so the warps'
+        // Producer warp j builds the whole B tile of every step s with s % PW == j, so the warps'
         // per-stage latencies (shared loads, fence.proxy.async, barrier arrive) overlap.  Lane: 16-byte
         // piece cc = lane & 7 of the 128-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k.
         // B[n = 8 y_local + 4b + 2c + d] = x_b & z_d & y_c (rows of smem singles keep the HBM swizzle:
         // piece cc of absolute row r sits at piece cc ^ (r & 7)).
+        // A warp's successive uses of a stage must be exactly one mbarrier phase apart (parity waits alias
+        // otherwise), so the number of active producer warps must divide STAGES.
+        constexpr int PW = (STAGES % tc::PROD_WARPS == 0) ? tc::PROD_WARPS : (STAGES % 2 == 0 ? 2 : 1);
         const int pw = warp - tc::PROD_WARP0;
         const int cc = lane & 7;
         const int cpl = (lane >> 3) & 1;
@@ -359,7 +367,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         const bool timing = (sp.debug & 8) != 0;
         long long t_wait = 0, t_busy = 0;
         for (int64_t step = 0; st.valid(sp); st.next(sp), ++step) {
-            if ((int)(step % tc::PROD_WARPS) != pw) continue;
+            if ((int)(step % PW) != pw) continue;     // warps with pw >= PW stay idle
             const int stage = (int)(step % STAGES);
             const uint32_t phase = (uint32_t)((step / STAGES) & 1);
             const long long t0 = timing ? clock64() : 0;
@@ -408,7 +416,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         // y_local = 2g + a with all 16 counts c16[8a' + 4b + 2c + d].
         const int ew = warp - tc::EPI_WARP0;           // 0..7
         const int q = warp & 3;                         // TMEM lane quadrant this warp may access
-        const int h = ew >> 2;                          // two warps per quadrant split the column groups
+        const int h = ew >> 2;                          // warps of one quadrant split the column groups
         const int row = q * 32 + lane;
         const int wl = row >> 1, a = row & 1;
         unsigned long long my_quads = 0, n_exact = 0;
@@ -427,12 +435,12 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
             const int w = ti.wr * EPI4_WR + wl;
             const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * 256);
 #pragma unroll 1
-            for (int g = h; g < 8; g += 2) {
+            for (int g = h; g < 8; g += tc::EPI_SPLIT) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(tbase + 16 * g, v0);
                 tmem_ld16(tbase + 128 + 16 * g, v1);
                 tmem_wait_ld();
-                if (g + 2 >= 8) {
+                if (g + tc::EPI_SPLIT >= 8) {
                     tc_fence_before();
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&tempty_bar[buf]);
