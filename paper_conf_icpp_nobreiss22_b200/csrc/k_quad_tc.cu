@@ -188,20 +188,25 @@ __device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t 
     return ti;
 }
 
-// iterator over the (tile, phenotype, chunk) steps of this CTA
+// iterator over the (tile, phenotype, chunk) steps of this CTA.  The per-phenotype chunk counts are held
+// in registers: indexing the kernel-parameter arrays with a runtime index spilled the parameter block to
+// the local-memory stack (L1 is mostly carved out for smem, so each step paid an L2 round trip).
 struct StepIt {
     int64_t tile;
     TileInfo ti;
     int p, kc;
+    int nch0, nch1;
     __device__ __forceinline__ void init(const SearchParams& sp) {
         tile = cluster_id_x();
         p = 0;
         kc = 0;
+        nch0 = sp.d.nchunks[0];
+        nch1 = sp.d.nchunks[1];
         if (tile < sp.ntiles) ti = decode_tile(sp, tile);
     }
     __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
     __device__ __forceinline__ void next(const SearchParams& sp) {
-        if (++kc == sp.d.nchunks[p]) {
+        if (++kc == (p ? nch1 : nch0)) {
             kc = 0;
             if (++p == 2) {
                 p = 0;
@@ -279,6 +284,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
     const int64_t first_group = cluster_id_x(), group_stride = nclusters_x();
     const uint32_t tmem = s_tmem;
     const int64_t chunk_stride = (int64_t)d.npad * 2 * tc::KCH;   // bytes of one chunk of expl
+    const int nch0_r = d.nchunks[0], nch1_r = d.nchunks[1];      // (no runtime-indexed parameter arrays)
+    const uint8_t* const expl0 = d.expl[0];
+    const uint8_t* const expl1 = d.expl[1];
 
     if (warp == 0) {
         // ===================== MMA issuer =====================
@@ -296,7 +304,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
                     const uint32_t dcol = tmem + (uint32_t)(buf * 256 + p * 128);
-                    const int nch = d.nchunks[p];
+                    const int nch = p ? nch1_r : nch0_r;
                     for (int kc = 0; kc < nch; ++kc) {
                         const long long t0 = timing ? clock64() : 0;
                         mbar_wait(&sfull_bar[stage], phase);
@@ -321,19 +329,32 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         __syncwarp();
     } else if (warp == 1) {
         // ===================== TMA issuer =====================
-        if (lane == 0) {
-            int stage = 0;
-            uint32_t phase = 0;
+        // TL lanes issue alternating steps in lockstep (lane l: steps l, l+TL, ...), each with its own stage
+        // and barrier: one thread issuing every step paid each instruction latency serially (~290 cycles per
+        // step, measured with debug & 64), which bounded the whole pipeline.  TL divides STAGES, so a lane's
+        // successive uses of a stage are one mbarrier phase apart.
+        constexpr int TL = 1;   // 2 lanes helped the pipeline-only case but not the full kernel (measured)
+        if (lane < TL) {
             StepIt st;
             st.init(sp);
+            int64_t step = 0;
+            for (int k = 0; k < lane && st.valid(sp); ++k, ++step) st.next(sp);
             const bool timing = (sp.debug & 8) != 0;
             long long t_wait = 0;
-            for (; st.valid(sp); st.next(sp)) {
+            while (st.valid(sp)) {
+                const int stage = (int)(step % STAGES);
+                const uint32_t phase = (uint32_t)((step / STAGES) & 1);
                 const long long t0 = timing ? clock64() : 0;
                 mbar_wait(&empty_bar[stage], phase ^ 1u);
                 if (timing) t_wait += clock64() - t0;
                 unsigned char* sbase = ring + stage * tc::STAGE_BYTES;
-                const uint8_t* E = d.expl[st.p] + (int64_t)st.kc * chunk_stride;
+                const uint8_t* E = (st.p ? expl1 : expl0) + (int64_t)st.kc * chunk_stride;
+                if (sp.debug & 128) {                 // diagnostics: no copies (MMA on stale smem)
+                    mbar_arrive(&sfull_bar[stage]);
+                    for (int k = 0; k < TL && st.valid(sp); ++k) st.next(sp);
+                    step += TL;
+                    continue;
+                }
                 mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
                 if (leader) {
                     // A, the y slab and x are the same for the whole cluster: one L2 read, multicast
@@ -343,7 +364,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
                 }
                 const int zc = st.ti.z < d.n ? st.ti.z : d.n - 1;   // dummy tile: any valid row
                 bulk_g2s(sbase + tc::SZ_OFF, E + (int64_t)zc * 2 * tc::KCH, 2 * tc::KCH, &sfull_bar[stage]);
-                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+                for (int k = 0; k < TL && st.valid(sp); ++k) st.next(sp);
+                step += TL;
             }
             if (timing) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
         }
