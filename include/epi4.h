@@ -109,7 +109,7 @@ int epi4_tables(epi4_ctx* ctx, const uint64_t* quads, int64_t n, uint32_t* count
 int epi4_set_dump(epi4_ctx* ctx, uint32_t* counts_dev);
 
 /* ---- plan --------------------------------------------------------------------
- * Work unit u = (w-range, x): all quads whose first SNP lies in [64*wr, 64*wr+64) and
+ * Work unit u = (w-range, x): all quads whose first SNP lies in [128*wr, 128*wr+128) and
  * whose second SNP is x.  The plan lists this rank's units (static LPT by modelled cost, identical
  * on every rank).  Host-only; usable without a GPU. */
 int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world);

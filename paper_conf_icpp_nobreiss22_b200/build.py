@@ -12,6 +12,8 @@ LIB = os.path.join(HERE, "libepi4.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-O2", "--expt-relaxed-constexpr"]
+if os.environ.get("EPI4_PROF"):   # instrumented build: per-role cycle counters + debug-64 pipeline trace
+    FLAGS.append("-DEPI4_PROF=1")
 
 
 def sources():

@@ -146,9 +146,9 @@ struct PlanEntry {
 
 std::vector<PlanEntry> all_units(int32_t n) {
     std::vector<PlanEntry> v;
-    const int32_t nr = (n + EPI4_WR - 1) / EPI4_WR;
+    const int32_t nr = (n + EPI4_WP - 1) / EPI4_WP;
     for (int32_t wr = 0; wr < nr; ++wr)
-        for (int32_t x = wr * EPI4_WR + 1; x <= n - 3; ++x) {
+        for (int32_t x = wr * EPI4_WP + 1; x <= n - 3; ++x) {
             const double cost = (double)unit_tiles(n, x);
             if (cost > 0) v.push_back({{wr, x}, cost});
         }
@@ -256,7 +256,7 @@ int finish_load(epi4_ctx* c) {
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
     c->loaded = false;
     c->n = n;
-    c->npad = (n + EPI4_YR + EPI4_WR - 1) / EPI4_WR * EPI4_WR;
+    c->npad = (n + EPI4_YR + EPI4_WP - 1) / EPI4_WP * EPI4_WP;
     c->np[0] = n0;
     c->np[1] = n1;
     for (int p = 0; p < 2; ++p) {
@@ -506,13 +506,13 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (ub < 0) ub = 0;
     if (ub > ue) ub = ue;
     const int64_t nu = ue - ub;
-    const int32_t G = quad_group(c->opts.pipe);
+    const int32_t G = quad_split(c->opts.pipe);
     std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
     std::vector<int64_t> prefix((size_t)std::max<int64_t>(nu, 1));
     int64_t acc = 0;
     for (int64_t i = 0; i < nu; ++i) {
         units[(size_t)i] = plan[(size_t)(ub + i)].u;
-        acc += unit_tiles(c->n, units[(size_t)i].x, G);
+        acc += unit_tiles(c->n, units[(size_t)i].x) * G;
         prefix[(size_t)i] = acc;
     }
     if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
@@ -527,7 +527,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
         CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), nu * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
     }
     int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
-    grid = std::max(G, grid / G * G);                 // whole clusters
+    grid = std::max(2, grid / 2 * 2);                 // whole CTA pairs
     if (int r = ensure_lists(c, grid, top_k)) return r;
     CU(cudaMemsetAsync(c->d_list_cnt, 0, (size_t)grid * sizeof(int32_t), c->stream));
     CU(cudaMemsetAsync(c->d_counters, 0, 32 * sizeof(unsigned long long), c->stream));
@@ -549,7 +549,6 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.quads_done = c->d_counters + 1;
     sp.prof = c->d_counters + 16;
     sp.use_lfx = 0;
-    sp.group = G;
     sp.debug = c->opts.reserved[0];
 
     c->stats.launches = 0;
@@ -576,8 +575,8 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     c->stats.ms_merge = ms;
     c->stats.quads = (int64_t)ctr[1];
     for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)ctr[16 + i];
-    c->stats.tiles = acc * G;
-    c->stats.executed_macs = (double)acc * G * 1024.0 * 16.0 * (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
+    c->stats.tiles = acc / G;
+    c->stats.executed_macs = (double)(acc / G) * 2048.0 * 16.0 * (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
     *n_out = nout;
     return 0;
 }

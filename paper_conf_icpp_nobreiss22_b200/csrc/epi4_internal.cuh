@@ -20,7 +20,8 @@
 #include "../../include/epi4.h"
 
 #define EPI4_B 32             // SNP block size accepted in epi4_opts (32-SNP blocks)
-#define EPI4_WR 64            // w-range of a work unit / rows of the A operand: 64 SNPs x {AA, Aa}
+#define EPI4_WR 64            // w-range of one CTA / rows of its A operand: 64 SNPs x {AA, Aa}
+#define EPI4_WP 128           // w-range of a work unit (a CTA pair: two 64-SNP halves)
 #define EPI4_YR 16            // y-range of a tile: 16 consecutive SNPs after x
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
@@ -70,28 +71,26 @@ __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, 
     return ((kc * npad + snp) * 2 + g) * EPI4_CHUNK_WORDS + w;
 }
 
-// A work unit (wr, x): the quads (w, x, y, z) with w in the 64-SNP range [64 wr, 64 wr + 64), w < x,
-// second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + 16) with
-// y0 = x + 1 + 16k, and z in (y0, n); a tile holds 64 x 16 = 1024 (w, y) combinations.
+// A work unit (wp, x): the quads (w, x, y, z) with w in the 128-SNP range [128 wp, 128 wp + 128), w < x,
+// second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + 16) with y0 = x + 1 + 16k,
+// and z in (y0, n); a tile holds 128 x 16 (w, y) combinations, split into the two 64-SNP halves of the
+// w-range (the two CTAs of a tensor-core cluster, or two tiles of the CUDA-core kernel).
 struct Unit {
-    int32_t wr, x;
+    int32_t wr, x;   // wr = 128-SNP w-range index
 };
 
-// Tiles are scheduled in groups of G consecutive z of the same (unit, y0) (G = the cluster size of the
-// tensor-core kernel, 1 for the CUDA-core kernel); a group's last members may be past n (dummy tiles).
-__host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x, int32_t G = 1) {
+__host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x) {
     int64_t t = 0;
-    for (int32_t y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) t += (n - y0 - 1 + G - 1) / G;
+    for (int32_t y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) t += n - y0 - 1;
     return t;
 }
 
-// decode group t of unit (x) -> (y0, first z of the group)
-__device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t, int32_t& y0, int32_t& z,
-                                                 int32_t G = 1) {
+// decode tile t of unit (x) -> (y0, z)
+__device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t, int32_t& y0, int32_t& z) {
     for (y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) {
-        const int64_t cnt = (n - y0 - 1 + G - 1) / G;
+        const int64_t cnt = n - y0 - 1;
         if (t < cnt) {
-            z = y0 + 1 + (int32_t)t * G;
+            z = y0 + 1 + (int32_t)t;
             return;
         }
         t -= cnt;
@@ -126,7 +125,7 @@ struct SearchParams {
     unsigned long long* quads_done;   // useful quads evaluated (atomicAdd once per CTA)
     unsigned long long* prof;  // [16] diagnostics: [0] exact K2 evaluations, [1..] per-role cycle counters
     int32_t use_lfx;           // fixed-point K2 filter table resident in shared memory
-    int32_t group;             // tiles per scheduling group (= cluster size of the tensor-core kernel)
+
     int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA
 };
 
@@ -148,7 +147,7 @@ cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T
                        int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_i8tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
-int32_t quad_group(int32_t pipe);
+int32_t quad_split(int32_t pipe);
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,
                          int32_t* out_n, cudaStream_t s, int64_t* launches);
 cudaError_t launch_tables(const DevData& d, const uint64_t* quads, int64_t n, uint32_t* out, unsigned int* status,

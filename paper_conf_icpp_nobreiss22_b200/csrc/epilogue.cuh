@@ -99,6 +99,42 @@ __device__ __forceinline__ void fill_slab_w(int (&g)[27], const uint32_t (&c16)[
     }
 }
 
+// Slab α = aa of w, before recovery: S_*[c] - S_0[c] - S_1[c] (the generalized counts restricted to w = aa).
+// Because the recovery is linear, M3 of it is r[2][...] (PAPER.md:L126 applied on axis w); computing it from
+// the raw tables (instead of keeping M3(S_*), M3(S_0), M3(S_1) alive) holds one slab per phenotype at a time.
+template <int P>
+__device__ __forceinline__ void fill_slab_aa(int (&g)[27], const uint32_t (&c16)[16], const DevData& d, int w, int x,
+                                             int y, int z) {
+    const uint4 txyz0 = t3_half(d, x, y, z, P, 0), txyz1 = t3_half(d, x, y, z, P, 1);
+    const uint4 pxy = t2_all(d, x, y, P), pxz = t2_all(d, x, z, P), pyz = t2_all(d, y, z, P);
+    const uint2 sx = t1_all(d, x, P), sy = t1_all(d, y, P), sz = t1_all(d, z, P);
+    const uint4 twxy0 = t3_half(d, w, x, y, P, 0), twxy1 = t3_half(d, w, x, y, P, 1);
+    const uint4 twxz0 = t3_half(d, w, x, z, P, 0), twxz1 = t3_half(d, w, x, z, P, 1);
+    const uint4 twyz0 = t3_half(d, w, y, z, P, 0), twyz1 = t3_half(d, w, y, z, P, 1);
+    const uint4 pwx = t2_all(d, w, x, P), pwy = t2_all(d, w, y, P), pwz = t2_all(d, w, z, P);
+    const uint2 sw = t1_all(d, w, P);
+#pragma unroll
+    for (int c = 0; c < 27; ++c) {
+        const int b = c / 9, e = (c / 3) % 3, f = c % 3;
+        const int ns = (b == 2) + (e == 2) + (f == 2);
+        uint32_t v;
+        if (ns == 0) {
+            v = (b ? u4(txyz1, e * 2 + f) : u4(txyz0, e * 2 + f)) - c16[b * 4 + e * 2 + f] - c16[8 + b * 4 + e * 2 + f];
+        } else if (ns == 1) {
+            if (f == 2) v = u4(pxy, b * 2 + e) - u4(twxy0, b * 2 + e) - u4(twxy1, b * 2 + e);
+            else if (e == 2) v = u4(pxz, b * 2 + f) - u4(twxz0, b * 2 + f) - u4(twxz1, b * 2 + f);
+            else v = u4(pyz, e * 2 + f) - u4(twyz0, e * 2 + f) - u4(twyz1, e * 2 + f);
+        } else if (ns == 2) {
+            if (b != 2) v = u2(sx, b) - u4(pwx, b) - u4(pwx, 2 + b);
+            else if (e != 2) v = u2(sy, e) - u4(pwy, e) - u4(pwy, 2 + e);
+            else v = u2(sz, f) - u4(pwz, f) - u4(pwz, 2 + f);
+        } else {
+            v = d.np[P] - sw.x - sw.y;
+        }
+        g[c] = (int)v;
+    }
+}
+
 // aa recovery on the three axes of a slab (strides 9, 3, 1): 3 x 9 x 2 = 54 subtractions
 __device__ __forceinline__ void mobius3(int (&g)[27]) {
 #pragma unroll
@@ -110,18 +146,14 @@ __device__ __forceinline__ void mobius3(int (&g)[27]) {
     }
 }
 
-// Per-quad evaluation in canonical cell order.  FIX: fixed-point K2 filter sum with the smem table
-// lfx; DBL: exact K2 in double, t_c = (L[r+1] - L[r0]) - L[r1], K2 += t_c, c = 0..80
+// Per-quad evaluation in canonical cell order, one slab (27 cells x 2 phenotypes) at a time:
+// α = AA (cells 0..26), Aa (27..53), aa (54..80).  FIX: fixed-point K2 filter sum with the smem table lfx
+// (DESIGN.md §5); DBL: exact K2 in double, t_c = (L[r+1] - L[r0]) - L[r1], K2 += t_c, c = 0..80
 // (reading #4); DUMP: write the 2 x 81 cells (controls first).
 template <bool FIX, bool DBL, bool DUMP>
 __device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y, int z, const uint32_t (&c0)[16],
                                           const uint32_t (&c1)[16], const int32_t* lfx, uint32_t& acc, double& k2,
                                           uint32_t* dump) {
-    int R0[27], R1[27];
-    fill_slab_star<0>(R0, d, x, y, z);
-    fill_slab_star<1>(R1, d, x, y, z);
-    mobius3(R0);
-    mobius3(R1);
     uint32_t a0 = 0, a1 = 0;
     double kk = 0.0;
     auto consume = [&](const int (&T0)[27], const int (&T1)[27], int base) {
@@ -143,17 +175,15 @@ __device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y,
         }
     };
 #pragma unroll
-    for (int a = 0; a < 2; ++a) {
+    for (int a = 0; a < 3; ++a) {
         int T0[27], T1[27];
         if (a == 0) { fill_slab_w<0, 0>(T0, c0, d, w, x, y, z); fill_slab_w<1, 0>(T1, c1, d, w, x, y, z); }
-        else        { fill_slab_w<0, 1>(T0, c0, d, w, x, y, z); fill_slab_w<1, 1>(T1, c1, d, w, x, y, z); }
+        else if (a == 1) { fill_slab_w<0, 1>(T0, c0, d, w, x, y, z); fill_slab_w<1, 1>(T1, c1, d, w, x, y, z); }
+        else { fill_slab_aa<0>(T0, c0, d, w, x, y, z); fill_slab_aa<1>(T1, c1, d, w, x, y, z); }
         mobius3(T0);
         mobius3(T1);
         consume(T0, T1, 27 * a);
-#pragma unroll
-        for (int c = 0; c < 27; ++c) { R0[c] -= T0[c]; R1[c] -= T1[c]; }
     }
-    consume(R0, R1, 54);
     acc = a0 + a1;
     k2 = kk;
 }

@@ -1,55 +1,69 @@
 // k_quad_tc.cu — the hot kernel: 4-way contraction on the 5th-generation tensor cores
-// (tcgen05.mma kind::i8, {0,1} operands, s32 accumulators in TMEM) with the fused epilogue.
+// (tcgen05.mma.cta_group::2.kind::i8, {0,1} operands, s32 accumulators in TMEM) with the fused epilogue.
 //
-// What it computes: for a tile (w-range wr, x, y-range y0, z) and each
-// phenotype p the 128 x 128 matrix
+// What it computes: for a tile (w-range pair wp, x, y-range y0, z) and each
+// phenotype p the 256 x 128 matrix
 //     C_p[(w, a)][(y, b, c, d)] = sum over samples s of phenotype p of P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]
-// for the 64 SNPs w of the range and the 16 SNPs y = y0..y0+15: the 16 non-aa genotype counts of the
-// 64 x 16 quads (w, x, y, z) ("a matrix with 16 values per each quad").
-// Factorisation (DESIGN.md §4): the paper ANDs SNP pairs into both operands (combine, PAPER.md:L89, L116);
-// here the A operand is the raw single-SNP planes (w, a) — copied from HBM by the TMA engine, no on-chip
-// production at all — and x is folded into the B operand, whose columns are triple products
-// P_b(x) & P_c(y) & P_d(z) built by two producer warps.  This halves the operand bytes that must be written
-// by threads (the LSU was the bottleneck of pair x pair tiles).
+// for the 128 SNPs w of the range pair and the 16 SNPs y = y0..y0+15: the 16 non-aa genotype counts of the
+// 128 x 16 quads (w, x, y, z) ("a matrix with 16 values per each quad").
+// Factorisation (DESIGN.md §5): the paper ANDs SNP pairs into both operands (combine, PAPER.md:L89, L116);
+// here the A operand is the raw single-SNP planes (w, a), copied from HBM by the TMA engine, and x is folded
+// into the B operand, whose columns are triple products P_b(x) & P_c(y) & P_d(z) built on chip.
 // Why i8: sm_100a has no native binary tensor op (ptxas emulates mma.sync ...b1.and.popc with legacy IMMA,
 // SURVEY.md App. C); AND+POPC becomes an integer MAC on {0,1} bytes, exact in s32.
+// Why 2-CTA: a 1-CTA M=128 N=128 i8 MMA issues every ~97 cycles (5.4K MAC/clk/SM); cta_group::2 with
+// M=256 N=128 issues every 64 cycles, the full 8.2K MAC/clk/SM (tools/probe_mma.cu, profiles/).
 //
-// Warp roles (CTA = 12 warps, 1 CTA per SM, persistent, static tile stride):
-//   warp 0      : TMEM allocation (512 columns) + one thread running a non-blocking event loop that issues
-//                 the TMA bulk copies of a stage (A: 64 SNPs x 2 planes x 128 samples = 16 KiB, pre-swizzled
-//                 in HBM; the 16 y planes, x and z) and the tcgen05.mma of ready stages
-//   warps 1..3  : producers — B[(y,b,c,d)] = x_b & z_d & y_c per 16-byte piece, stored K-major SW128
-//   warps 4..11 : epilogue — tcgen05.ld of the control and case accumulators, pairwise lane exchange so one
-//                 thread holds one quad's 2 x 16 counts, then the shared epilogue (epilogue.cuh)
-// Pipelines: STAGES x {A, B, singles} (sfull: TMA bytes landed, full: B produced, empty: MMA done);
-// TMEM double buffer (2 x [128 ctrl | 128 case] columns) between MMA and epilogue.
+// CTA pair (cluster of 2): CTA r holds the A rows of w-range 2wp + r (64 SNPs x {AA, Aa}) and builds the
+// B columns of y = y0 + 8r .. y0 + 8r + 7; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
+// receives its 128 rows x all 128 columns and its epilogue scores its 64 x 16 quads.
+// Warp roles (each CTA: 12 warps, 1 CTA per SM, persistent, static tile stride over clusters):
+//   warp 0      : TMEM allocation (cta_group::2, 512 columns); leader: one thread issuing tcgen05.mma
+//   warp 1      : one thread issuing the TMA bulk copies of the CTA's stage (A 16 KiB pre-swizzled in HBM,
+//                 its 8 y planes, x, z)
+//   warps 2..3  : producers (alternating steps) — the CTA's half of B, x_b & z_d & y_c per 16-byte piece,
+//                 K-major SW128; each then arrives on the leader's `full` barrier
+//   warps 4..11 : epilogue — tcgen05.ld of the control and case accumulators, lane-pair exchange so one
+//                 thread holds one quad's 2 x 16 counts, the shared epilogue (epilogue.cuh); then an
+//                 arrival on the leader's `tempty` barrier
+// Pipelines: STAGES x {A, B half, singles} per CTA (sfull: own TMA landed; full @leader: both B halves built;
+// empty: leader's MMA commit, multicast to both CTAs); TMEM double buffer 2 x [128 ctrl | 128 case].
+#include <cstdio>
+#include <cstdlib>
+#include <type_traits>
 #include "epilogue.cuh"
 
 namespace epi4 {
 
 namespace tc {
-constexpr int M = 128, N = 128;          // UMMA shape (cta_group::1), K = 32 bytes per instruction
+constexpr int M = 256, N = 128;          // UMMA shape (cta_group::2), K = 32 bytes per instruction
 constexpr int KCH = EPI4_CHUNK_SAMPLES;  // 128 samples (bytes) per pipeline stage
-constexpr int A_BYTES = M * KCH, B_BYTES = N * KCH;
-constexpr int SY_OFF = A_BYTES + B_BYTES, SY_BYTES = 2 * EPI4_YR * KCH;   // 16 y SNPs x 2 planes
-constexpr int SX_OFF = SY_OFF + SY_BYTES, SZ_OFF = SX_OFF + 2 * KCH;
-constexpr int STAGE_BYTES = ((SZ_OFF + 2 * KCH) + 1023) / 1024 * 1024;
-constexpr int TX_BYTES = A_BYTES + SY_BYTES + 4 * KCH;                      // bytes the TMA brings per stage
-// warp 0: MMA issuer; warp 1: TMA issuer; warps 2-3: producers (alternating stages); warps 4-11:
-// epilogue.  384 threads keep 168 registers per thread (above 384 ptxas drops to 128).
-#ifndef EPI4_TC_PROD_WARPS
-#define EPI4_TC_PROD_WARPS 2
+constexpr int A_BYTES = 128 * KCH;       // this CTA's 128 A rows
+constexpr int B_BYTES = (N / 2) * KCH;   // this CTA's 64 B columns
+constexpr int YH = EPI4_YR / 2;          // y SNPs per CTA
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 24 KiB, 1024-aligned
+constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per stage
+// singles (x, z, y-half planes of one step) prefetched by each producer warp with cp.async into its own ring
+constexpr int SX_OFF = 0, SZ_OFF = 2 * KCH, SY_OFF = 4 * KCH;
+constexpr int SGL_BYTES = (4 + 2 * YH) * KCH;              // 20 rows x 128 B
+#ifndef EPI4_PF
+#define EPI4_PF 1
 #endif
-#ifndef EPI4_TC_EPI_WARPS
-#define EPI4_TC_EPI_WARPS 8
+constexpr int PF = EPI4_PF;                                // prefetch distance (own steps)
+constexpr int SGL_SLOTS = PF + 1;
+#ifndef EPI4_PROD_WARPS
+#define EPI4_PROD_WARPS 3
 #endif
-constexpr int PROD_WARPS = EPI4_TC_PROD_WARPS, EPI_WARPS = EPI4_TC_EPI_WARPS;   // EPI_WARPS: 4 or 8
-constexpr int PROD_WARP0 = 2, EPI_WARP0 = 2 + PROD_WARPS;
-constexpr int THREADS = 32 * (2 + PROD_WARPS + EPI_WARPS);
-constexpr int EPI_SPLIT = EPI_WARPS / 4;   // warps per TMEM lane quadrant (they alternate 16-column groups)
+constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
+constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate steps (one thread cannot hide
+                                         // its own wait/bookkeeping latency behind the blocking MMA issue)
+constexpr int TMA_WARP = MMA_WARPS, PROD_WARP0 = TMA_WARP + 1, EPI_WARP0 = PROD_WARP0 + PROD_WARPS;
+constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 448 with 3 producer warps: 128 registers
+constexpr int MAX_STAGES = 12;
+constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
+constexpr int STAGE_Q = PROD_WARPS / gcd_c(PROD_WARPS, MMA_WARPS) * MMA_WARPS;   // stage counts: multiples
 constexpr int TMEM_COLS = 512;
-constexpr int CLUSTER = 2;                 // CTAs sharing A, the y slab and x through TMA multicast
-                                           // (2 packs all 148 SMs; 4 strands SMs of the 18-SM GPCs)
+constexpr int CLUSTER = 2;
 // instruction descriptor: D s32 (bits 4-5 = 2), A/B u8 (0), K-major, N>>3 at bit 17, M>>4 at bit 24
 constexpr uint32_t IDESC = (2u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }  // namespace tc
@@ -59,22 +73,25 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)_
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
 }
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(smem_u32(bar)) : "memory");
+__device__ __forceinline__ void mbar_arrive_local(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+// arrive on the same-offset barrier of cluster CTA `cta`.  Release at CTA scope (the CUTLASS remote-arrive
+// form): a cluster-scope release compiles to a GPU-wide memory barrier that waits for the thread's in-flight
+// cp.async prefetches (~1000 cycles per step, measured with debug 64).  What the peer consumes is this CTA's
+// own shared memory, read by the tensor core after fence.proxy.async; CTA-scope completion covers it.
+__device__ __forceinline__ void mbar_arrive_cluster(uint64_t* bar, uint32_t cta) {
+    uint32_t remote;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(smem_u32(bar)), "r"(cta));
+    asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(remote) : "memory");
+}
+// CTA-scope acquire: a cluster-scope acquire compiles to an L1 invalidate (CCTL.IVALL) after every successful
+// poll, which evicts the epilogue's cached tables; no waiter here reads peer data through L1 (the tensor core
+// reads the peer's operands through the async proxy, ordered by the producer's fence.proxy.async + release).
 __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
         "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(ok)
-        : "r"(smem_u32(bar)), "r"(parity)
-        : "memory");
-    return ok != 0;
-}
-__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
-    uint32_t ok;
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok)
         : "r"(smem_u32(bar)), "r"(parity)
         : "memory");
@@ -88,6 +105,21 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         if (clock64() - t0 > 40000000000LL) __trap();
     }
 }
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t tx) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(tx) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -101,18 +133,20 @@ __device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
     d |= (uint64_t)2 << 61;                 // SWIZZLE_128B
     return d;
 }
-
-__device__ __forceinline__ void mma_i8(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t acc) {
+// D[tmem] (+)= A[smem, both CTAs] . B[smem, both CTAs]^T for the CTA pair; issued by the leader only
+__device__ __forceinline__ void mma2_i8(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t acc) {
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %4, p;\n\t}" ::"r"(d_tmem),
+        "tcgen05.mma.cta_group::2.kind::i8 [%0], %1, %2, %4, p;\n\t}" ::"r"(d_tmem),
         "l"(adesc), "l"(bdesc), "r"(acc), "r"(tc::IDESC));
 }
-__device__ __forceinline__ void mma_commit(uint64_t* bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+// arrive (when the leader's prior MMAs complete) on the same-offset barrier of both CTAs of the pair
+__device__ __forceinline__ void mma2_commit_mc(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                     smem_u32(bar)),
+                 "h"((uint16_t)3)
                  : "memory");
 }
-
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
@@ -121,39 +155,31 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
         : "r"(taddr));
 }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+// zero 16 columns of this warp's 32 TMEM lanes
+__device__ __forceinline__ void tmem_zero16(uint32_t taddr) {
+    const uint32_t z = 0;
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(taddr),
+        "r"(z)
+        : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // byte offset of (row r, 16-byte chunk c) inside a K-major SW128 tile of 128-byte rows
 __device__ __forceinline__ uint32_t sw128_off(int r, int c) {
     return (uint32_t)((r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4));
 }
-
 __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x & b.x, a.y & b.y, a.z & b.z, a.w & b.w); }
 
-// 4x4 transpose inside each group of 4 lanes.  In: lane t (t = lane & 3) holds v[4*jj + cd] = its row
-// (ab = t) for quads jj = 0..3.  Out: lane t holds w[4*ab + cd] of quad jj = t.
-__device__ __forceinline__ void quad_transpose(const uint32_t (&v)[16], uint32_t (&w)[16]) {
-    const int t = threadIdx.x & 3;
-    uint32_t r[4][4];   // r[k][cd]: value received in round k (k = 0: own diagonal)
-#pragma unroll
-    for (int cd = 0; cd < 4; ++cd) {
-        r[0][cd] = t == 0 ? v[cd] : t == 1 ? v[4 + cd] : t == 2 ? v[8 + cd] : v[12 + cd];
-#pragma unroll
-        for (int k = 1; k < 4; ++k) {
-            const int jj = t ^ k;   // send my row's value for quad jj to lane jj
-            const uint32_t s = jj == 0 ? v[cd] : jj == 1 ? v[4 + cd] : jj == 2 ? v[8 + cd] : v[12 + cd];
-            r[k][cd] = __shfl_xor_sync(0xffffffffu, s, k);
-        }
-    }
-    // w[ab][cd] came in round k = ab ^ t
-#pragma unroll
-    for (int ab = 0; ab < 4; ++ab)
-#pragma unroll
-        for (int cd = 0; cd < 4; ++cd) {
-            const int k = ab ^ t;
-            w[ab * 4 + cd] = k == 0 ? r[0][cd] : k == 1 ? r[1][cd] : k == 2 ? r[2][cd] : r[3][cd];
-        }
+// one lane of the (converged) warp returns true
+__device__ __forceinline__ bool elect_one() {
+    uint32_t pred = 0;
+    asm volatile(
+        "{\n\t.reg .b32 rx;\n\t.reg .pred px;\n\telect.sync rx|px, %1;\n\t@px mov.s32 %0, 1;\n\t}"
+        : "+r"(pred)
+        : "r"(0xffffffffu));
+    return pred != 0;
 }
-
 __device__ __forceinline__ uint32_t cluster_rank() {
     uint32_t r;
     asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
@@ -174,23 +200,20 @@ __device__ __forceinline__ void cluster_sync_all() {
 }
 
 struct TileInfo {
-    int32_t wr, x, y0, z;
+    int32_t wp, x, y0, z;
 };
-// group -> this CTA's tile: the cluster's CTA of rank r takes z = first z of the group + r (>= n: dummy)
-__device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t group) {
-    const int64_t u = find_unit(sp.prefix, sp.nunits, group);
-    const int64_t t = group - (u ? sp.prefix[u - 1] : 0);
+__device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t tile) {
+    const int64_t u = find_unit(sp.prefix, sp.nunits, tile);
+    const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);
     TileInfo ti;
-    ti.wr = sp.units[u].wr;
+    ti.wp = sp.units[u].wr;
     ti.x = sp.units[u].x;
-    unit_tile_decode(sp.d.n, ti.x, t, ti.y0, ti.z, tc::CLUSTER);
-    ti.z += (int32_t)cluster_rank();
+    unit_tile_decode(sp.d.n, ti.x, t, ti.y0, ti.z);
     return ti;
 }
 
-// iterator over the (tile, phenotype, chunk) steps of this CTA.  The per-phenotype chunk counts are held
-// in registers: indexing the kernel-parameter arrays with a runtime index spilled the parameter block to
-// the local-memory stack (L1 is mostly carved out for smem, so each step paid an L2 round trip).
+// iterator over the (tile, phenotype, chunk) steps of this cluster; advance(k) moves k steps ahead.
+// Chunk counts live in registers (runtime indexing of kernel-parameter arrays spills the parameter block).
 struct StepIt {
     int64_t tile;
     TileInfo ti;
@@ -205,267 +228,336 @@ struct StepIt {
         if (tile < sp.ntiles) ti = decode_tile(sp, tile);
     }
     __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
-    __device__ __forceinline__ void next(const SearchParams& sp) {
-        if (++kc == (p ? nch1 : nch0)) {
-            kc = 0;
+    __device__ __forceinline__ void advance(const SearchParams& sp, int k) {
+        kc += k;
+        if (kc < (p ? nch1 : nch0)) return;
+        const int64_t t0 = tile;
+        while (kc >= (p ? nch1 : nch0)) {
+            kc -= p ? nch1 : nch0;
             if (++p == 2) {
                 p = 0;
                 tile += nclusters_x();
-                if (tile < sp.ntiles) ti = decode_tile(sp, tile);
             }
         }
+        if (tile != t0 && tile < sp.ntiles) ti = decode_tile(sp, tile);
     }
 };
 
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t tx) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(tx) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                     smem_u32(dst)),
-                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
-                 : "memory");
-}
-
-__device__ __forceinline__ void bulk_g2s_mc(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint16_t mask) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(
-            smem_u32(dst)),
-        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "h"(mask)
-        : "memory");
-}
-// arrive (when this thread's prior MMAs complete) on the same-offset mbarrier of every CTA in `mask`
-__device__ __forceinline__ void mma_commit_mc(uint64_t* bar, uint16_t mask) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
-                     smem_u32(bar)),
-                 "h"(mask)
-                 : "memory");
-}
+// Compile-time instrumentation (build with -DEPI4_PROF=1): per-role cycle counters in prof[1..7] and, with
+// debug bit 64, a per-step event trace of cluster 0 printed at exit (tools/trace_view.py).
+#ifndef EPI4_PROF
+#define EPI4_PROF 0
+#endif
+#if EPI4_PROF
+constexpr int TR_STEPS = 96, TR_EV = 14;
+__device__ long long g_trace[2][TR_EV][TR_STEPS];
+#define TRACE(ev, step)                                                                                    \
+    do {                                                                                                   \
+        if (tracing && (step) < TR_STEPS) g_trace[rank][ev][(step)] = clock64() - t_base;                   \
+    } while (0)
+#define PCLK() clock64()
+#else
+#define TRACE(ev, step) do { } while (0)
+#define PCLK() 0LL
+#endif
 
 template <int STAGES>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
+    static_assert(STAGES % tc::STAGE_Q == 0, "a producer's / issuer's successive uses of a stage must be one phase apart");
     extern __shared__ unsigned char smem_raw[];
     __shared__ __align__(8) uint64_t sfull_bar[STAGES], full_bar[STAGES], empty_bar[STAGES];
     __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2];
     __shared__ uint32_t s_tmem;
-    // 1024-aligned stage ring, then the fixed-point lgamma table, then the top-k state
+    // 1024-aligned stage ring, the producers' singles rings, the fixed-point lgamma table, the top-k state
+    // (same offsets in both CTAs of the pair: the MMA addresses the peer's operands at the same offsets)
     const uint32_t raw = smem_u32(smem_raw);
     unsigned char* ring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-    int32_t* s_lfx = reinterpret_cast<int32_t*>(ring + STAGES * tc::STAGE_BYTES);
+    unsigned char* sgl_ring = ring + STAGES * tc::STAGE_BYTES;   // [PROD_WARPS][SGL_SLOTS][SGL_BYTES]
+    int32_t* s_lfx = reinterpret_cast<int32_t*>(sgl_ring + tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES);
     const int lfx_words = sp.use_lfx ? ((sp.d.lfx_n + 3) & ~3) : 0;
     TopKSmem tk = topk_carve(reinterpret_cast<unsigned char*>(s_lfx + lfx_words), sp.topk);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const DevData& d = sp.d;
+    const uint32_t rank = cluster_rank();
+    const bool leader = rank == 0;
     if (tid == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&sfull_bar[s], 1);
-            mbar_init(&full_bar[s], 1);          // one producer warp builds a stage's B tile
-            mbar_init(&empty_bar[s], tc::CLUSTER);   // every CTA's MMA must release a stage
+            mbar_init(&full_bar[s], tc::CLUSTER);         // (leader) one producer arrival per CTA
+            mbar_init(&empty_bar[s], 1);                  // the leader's MMA commit
         }
         for (int b = 0; b < 2; ++b) {
-            mbar_init(&tfull_bar[b], 1);
-            mbar_init(&tempty_bar[b], tc::EPI_WARPS);
+            mbar_init(&tfull_bar[b], tc::MMA_WARPS);      // each issuer's commit after its last step
+            mbar_init(&tempty_bar[b], tc::CLUSTER * tc::EPI_WARPS);   // (leader) every epilogue warp of the pair
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 0) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&s_tmem)),
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&s_tmem)),
                      "r"(tc::TMEM_COLS));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
     }
     topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);
     for (int e = tid; e < lfx_words; e += tc::THREADS) s_lfx[e] = e < d.lfx_n ? __ldg(d.lfx + e) : 0;
+    // Accumulators are zeroed by the epilogue after it reads them (and once here), so every MMA accumulates:
+    // the two issuers' MMAs into one tile may then complete in any order.
+    __syncthreads();                     // TMEM address visible
+    if (warp >= tc::EPI_WARP0) {
+        const int ew = warp - tc::EPI_WARP0, q = warp & 3, h = ew >> 2;
+        const uint32_t tq = s_tmem + ((uint32_t)(q * 32) << 16);
+        for (int col = 16 * h; col < tc::TMEM_COLS; col += 32) tmem_zero16(tq + (uint32_t)col);
+        tmem_wait_st();
+    }
     tc_fence_before();
-    cluster_sync_all();                  // barrier inits visible cluster-wide before any multicast
+    cluster_sync_all();                  // barrier inits and TMEM allocation visible to the pair
     tc_fence_after();
-    const bool leader = cluster_rank() == 0;
-    const uint16_t cmask = (uint16_t)((1u << tc::CLUSTER) - 1);
-    const int64_t first_group = cluster_id_x(), group_stride = nclusters_x();
     const uint32_t tmem = s_tmem;
+#if EPI4_PROF
+    const bool tracing = (sp.debug & 64) && cluster_id_x() == 0;
+    const long long t_base = clock64();
+#endif
+    const int64_t first_tile = cluster_id_x(), tile_stride = nclusters_x();
     const int64_t chunk_stride = (int64_t)d.npad * 2 * tc::KCH;   // bytes of one chunk of expl
-    const int nch0_r = d.nchunks[0], nch1_r = d.nchunks[1];      // (no runtime-indexed parameter arrays)
+    const int nch0_r = d.nchunks[0], nch1_r = d.nchunks[1];
     const uint8_t* const expl0 = d.expl[0];
     const uint8_t* const expl1 = d.expl[1];
 
-    if (warp == 0) {
-        // ===================== MMA issuer =====================
-        if (lane == 0) {
-            int stage = 0;
-            uint32_t phase = 0;
-            int it = 0;
-            const bool timing = (sp.debug & 8) != 0;
+    if (warp < tc::MMA_WARPS) {
+        // ===================== MMA issuers (leader CTA) =====================
+        // Issuer m takes the steps s with s % MMA_WARPS == m.  The whole warp runs the loop (warp-uniform
+        // control flow keeps the descriptors in uniform registers); one elected lane issues.  Descriptors are
+        // precomputed once: per MMA only a 64-bit add (tools/probe_mma3.cu).  Every MMA accumulates (the
+        // epilogue re-zeroes the accumulators), so the two issuers' MMAs commute.
+        if (leader) {
+            const int m = warp;
+            const uint32_t ring_s = smem_u32(ring);
+            const uint64_t adesc0 = sw128_desc(ring_s), bdesc0 = sw128_desc(ring_s + tc::A_BYTES);
+            int stage = m;
+            uint32_t phase = 0, soff = (uint32_t)m * (tc::STAGE_BYTES >> 4);
+            int it = 0, gstep = 0;
             long long t_wait = 0;
-            for (int64_t tile = first_group; tile < sp.ntiles; tile += group_stride, ++it) {
+            const bool do_mma = !(sp.debug & 4);
+            for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
                 const int buf = it & 1;
                 const uint32_t tphase = (uint32_t)((it >> 1) & 1);
-                mbar_wait(&tempty_bar[buf], tphase ^ 1u);   // epilogue drained this buffer
+                mbar_wait(&tempty_bar[buf], tphase ^ 1u);   // both CTAs' epilogues drained this buffer
                 tc_fence_after();
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
                     const uint32_t dcol = tmem + (uint32_t)(buf * 256 + p * 128);
                     const int nch = p ? nch1_r : nch0_r;
-                    for (int kc = 0; kc < nch; ++kc) {
-                        const long long t0 = timing ? clock64() : 0;
-                        mbar_wait(&sfull_bar[stage], phase);
-                        mbar_wait(&full_bar[stage], phase);
-                        if (timing) t_wait += clock64() - t0;
+#pragma unroll 1
+                    for (int kc = 0; kc < nch; ++kc, ++gstep) {
+                        if ((gstep & (tc::MMA_WARPS - 1)) != m) continue;
+                        const long long t0 = PCLK();
+                        if (lane == 0) TRACE(12, gstep);
+                        mbar_wait(&full_bar[stage], phase);         // both B halves built, both A halves landed
+                        t_wait += PCLK() - t0;
+                        if (lane == 0) TRACE(10, gstep);
                         tc_fence_after();
-                        const uint32_t a0 = smem_u32(ring + stage * tc::STAGE_BYTES);
-                        const uint32_t b0 = a0 + tc::A_BYTES;
-                        if (!(sp.debug & 4)) {
+                        if (elect_one()) {
+                            if (do_mma) {
 #pragma unroll
-                            for (int k = 0; k < tc::KCH / 32; ++k)
-                                mma_i8(dcol, sw128_desc(a0 + 32 * k), sw128_desc(b0 + 32 * k), (kc | k) != 0);
+                                for (int k = 0; k < tc::KCH / 32; ++k)
+                                    mma2_i8(dcol, adesc0 + soff + 2 * k, bdesc0 + soff + 2 * k, 1u);
+                            }
+                            mma2_commit_mc(&empty_bar[stage]);      // frees the stage in both CTAs
                         }
-                        mma_commit_mc(&empty_bar[stage], cmask);  // frees the stage in every CTA of the cluster
-                        if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+                        __syncwarp();
+                        if (lane == 0) TRACE(11, gstep);
+                        soff += tc::MMA_WARPS * (tc::STAGE_BYTES >> 4);
+                        stage += tc::MMA_WARPS;
+                        if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; soff -= STAGES * (tc::STAGE_BYTES >> 4); }
                     }
                 }
-                mma_commit(&tfull_bar[buf]);                    // accumulators of this tile are ready
+                if (elect_one()) mma2_commit_mc(&tfull_bar[buf]);   // this issuer's MMAs of the tile are done
+                __syncwarp();
             }
-            if (timing) atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
+            if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
         }
         __syncwarp();
-    } else if (warp == 1) {
-        // ===================== TMA issuer =====================
-        // TL lanes issue alternating steps in lockstep (lane l: steps l, l+TL, ...), each with its own stage
-        // and barrier: one thread issuing every step paid each instruction latency serially (~290 cycles per
-        // step, measured with debug & 64), which bounded the whole pipeline.  TL divides STAGES, so a lane's
-        // successive uses of a stage are one mbarrier phase apart.
-        constexpr int TL = 1;   // 2 lanes helped the pipeline-only case but not the full kernel (measured)
-        if (lane < TL) {
+    } else if (warp == tc::TMA_WARP) {
+        // ===================== TMA issuer: this CTA's A (16 KiB per step) =====================
+        // whole warp runs the loop (uniform operands), one elected lane issues
+        {
+            int stage = 0;
+            uint32_t phase = 0;
             StepIt st;
             st.init(sp);
-            int64_t step = 0;
-            for (int k = 0; k < lane && st.valid(sp); ++k, ++step) st.next(sp);
-            const bool timing = (sp.debug & 8) != 0;
             long long t_wait = 0;
-            while (st.valid(sp)) {
-                const int stage = (int)(step % STAGES);
-                const uint32_t phase = (uint32_t)((step / STAGES) & 1);
-                const long long t0 = timing ? clock64() : 0;
+            const uint32_t ring_s = smem_u32(ring);
+            for (int gstep = 0; st.valid(sp); st.advance(sp, 1), ++gstep) {
+                const long long t0 = PCLK();
                 mbar_wait(&empty_bar[stage], phase ^ 1u);
-                if (timing) t_wait += clock64() - t0;
-                unsigned char* sbase = ring + stage * tc::STAGE_BYTES;
+                t_wait += PCLK() - t0;
+                if (lane == 0) TRACE(0, gstep);
                 const uint8_t* E = (st.p ? expl1 : expl0) + (int64_t)st.kc * chunk_stride;
-                if (sp.debug & 128) {                 // diagnostics: no copies (MMA on stale smem)
-                    mbar_arrive(&sfull_bar[stage]);
-                    for (int k = 0; k < TL && st.valid(sp); ++k) st.next(sp);
-                    step += TL;
-                    continue;
+                const int64_t wrow = (int64_t)(st.ti.wp * 2 + (int)rank) * EPI4_WR * 2;   // first A row
+                if (elect_one()) {
+                    mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                                 ::"r"(ring_s + (uint32_t)(stage * tc::STAGE_BYTES)), "l"(E + wrow * tc::KCH),
+                                 "r"((uint32_t)tc::A_BYTES), "r"(smem_u32(&sfull_bar[stage]))
+                                 : "memory");
                 }
-                mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
-                if (leader) {
-                    // A, the y slab and x are the same for the whole cluster: one L2 read, multicast
-                    bulk_g2s_mc(sbase, E + (int64_t)st.ti.wr * EPI4_WR * 2 * tc::KCH, tc::A_BYTES, &sfull_bar[stage], cmask);
-                    bulk_g2s_mc(sbase + tc::SY_OFF, E + (int64_t)st.ti.y0 * 2 * tc::KCH, tc::SY_BYTES, &sfull_bar[stage], cmask);
-                    bulk_g2s_mc(sbase + tc::SX_OFF, E + (int64_t)st.ti.x * 2 * tc::KCH, 2 * tc::KCH, &sfull_bar[stage], cmask);
-                }
-                const int zc = st.ti.z < d.n ? st.ti.z : d.n - 1;   // dummy tile: any valid row
-                bulk_g2s(sbase + tc::SZ_OFF, E + (int64_t)zc * 2 * tc::KCH, 2 * tc::KCH, &sfull_bar[stage]);
-                for (int k = 0; k < TL && st.valid(sp); ++k) st.next(sp);
-                step += TL;
+                __syncwarp();
+                if (lane == 0) TRACE(1, gstep);
+                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
             }
-            if (timing) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
+            if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
         }
-        __syncwarp();
-    } else if (warp >= tc::PROD_WARP0 && warp < tc::PROD_WARP0 + tc::PROD_WARPS) {
+    } else if (warp < tc::EPI_WARP0) {
         // ===================== producers =====================
-        // Producer warp j builds the whole B tile of every step s with s % PW == j, so the warps'
-        // per-stage latencies (shared loads, fence.proxy.async, barrier arrive) overlap.  Lane: 16-byte
-        // piece cc = lane & 7 of the 128-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k.
-        // B[n = 8 y_local + 4b + 2c + d] = x_b & z_d & y_c (rows of smem singles keep the HBM swizzle:
-        // piece cc of absolute row r sits at piece cc ^ (r & 7)).
-        // A warp's successive uses of a stage must be exactly one mbarrier phase apart (parity waits alias
-        // otherwise), so the number of active producer warps must divide STAGES.
-        constexpr int PW = (STAGES % tc::PROD_WARPS == 0) ? tc::PROD_WARPS : (STAGES % 2 == 0 ? 2 : 1);
+        // Producer warp j builds this CTA's B half of every step s with s % PROD_WARPS == j.  Its singles
+        // (x, z and the CTA's 8 y SNPs: 20 rows of 128 B, pre-swizzled in HBM) are prefetched PF own steps
+        // ahead with cp.async into the warp's private ring.  Lane: 16-byte piece cc = lane & 7 of the
+        // 128-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k (k = 0..3);
+        // B[n = 8 y_local + 4b + 2c + d] = x_b & y_c & z_d.  The warp waits for its CTA's A (sfull) before
+        // arriving on the leader's `full` barrier, so `full` also certifies the follower's A.
         const int pw = warp - tc::PROD_WARP0;
-        const int cc = lane & 7;
-        const int cpl = (lane >> 3) & 1;
-        const bool skip = (sp.debug & 1) != 0;
-        StepIt st;
+        const int cc = lane & 7, cpl = (lane >> 3) & 1, yq = lane >> 4;
+        const bool build = !(sp.debug & 1);
+        unsigned char* my_sgl = sgl_ring + pw * tc::SGL_SLOTS * tc::SGL_BYTES;
+        // store offsets inside the B half for bd = 2b + d (y_local = yq; + 2048 per k)
+        uint32_t boff[4];
+#pragma unroll
+        for (int bd = 0; bd < 4; ++bd) {
+            const int n7 = (bd >> 1) * 4 + cpl * 2 + (bd & 1);
+            boff[bd] = (uint32_t)(yq * 1024 + n7 * 128 + ((cc ^ n7) << 4));
+        }
+        // this lane's 5 pieces of a singles slot: piece 0 = x|z row piece, pieces 1..4 = y rows
+        const int pxz = lane < 16 ? lane * 16 : (lane - 16) * 16;     // byte offset inside the x or z rows
+        long long t_wait = 0, t_busy = 0, t_arr = 0;
+        StepIt st, pre;
         st.init(sp);
-        const bool timing = (sp.debug & 8) != 0;
-        long long t_wait = 0, t_busy = 0;
-        for (int64_t step = 0; st.valid(sp); st.next(sp), ++step) {
-            if ((int)(step % PW) != pw) continue;     // warps with pw >= PW stay idle
-            const int stage = (int)(step % STAGES);
-            const uint32_t phase = (uint32_t)((step / STAGES) & 1);
-            const long long t0 = timing ? clock64() : 0;
-            mbar_wait(&sfull_bar[stage], phase);
-            const long long t1 = timing ? clock64() : 0;
+        st.advance(sp, pw);
+        pre = st;
+        auto prefetch = [&](int slot, const StepIt& it) {
+            if (it.valid(sp)) {
+                const uint8_t* E = (it.p ? expl1 : expl0) + (int64_t)it.kc * chunk_stride;
+                unsigned char* dst = my_sgl + slot * tc::SGL_BYTES;
+                const uint8_t* srcxz = E + (int64_t)(lane < 16 ? it.ti.x : it.ti.z) * 2 * tc::KCH + pxz;
+                cp_async16(dst + lane * 16, srcxz);
+                const uint8_t* srcy = E + (int64_t)(it.ti.y0 + tc::YH * (int)rank) * 2 * tc::KCH + lane * 16;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) cp_async16(dst + tc::SY_OFF + k * 512 + lane * 16, srcy + k * 512);
+            }
+            cp_async_commit();                                    // (an empty group past the end)
+        };
+#pragma unroll 1
+        for (int k = 0; k < tc::PF; ++k) {
+            prefetch(k, pre);
+            pre.advance(sp, tc::PROD_WARPS);
+        }
+        int slot = 0, stage = pw;
+        uint32_t phase = 0;
+        for (int step = pw; st.valid(sp); step += tc::PROD_WARPS) {
+            if (lane == 0) TRACE(2, step);
+            prefetch(slot == 0 ? tc::PF : slot - 1, pre);         // slot (slot + PF) % (PF + 1)
+            pre.advance(sp, tc::PROD_WARPS);
+            cp_async_wait<tc::PF>();                              // this step's singles landed (own lane)
+            __syncwarp();                                         // ... and every lane's
+            if (lane == 0) TRACE(3, step);
+            const long long t0 = PCLK();
+            mbar_wait(&empty_bar[stage], phase ^ 1u);             // B slot free (MMA of step - STAGES done)
+            const long long t1 = PCLK();
             t_wait += t1 - t0;
-            if (!skip) {
-                unsigned char* sbase = ring + stage * tc::STAGE_BYTES;
-                unsigned char* sb = sbase + tc::A_BYTES;
-                const int x = st.ti.x, z = st.ti.z, y0 = st.ti.y0;
-                const uint4 x0 = *reinterpret_cast<const uint4*>(sbase + tc::SX_OFF + ((cc ^ ((2 * x) & 7)) << 4));
-                const uint4 x1 = *reinterpret_cast<const uint4*>(sbase + tc::SX_OFF + 128 + ((cc ^ ((2 * x + 1) & 7)) << 4));
-                const uint4 z0 = *reinterpret_cast<const uint4*>(sbase + tc::SZ_OFF + ((cc ^ ((2 * z) & 7)) << 4));
-                const uint4 z1 = *reinterpret_cast<const uint4*>(sbase + tc::SZ_OFF + 128 + ((cc ^ ((2 * z + 1) & 7)) << 4));
+            if (lane == 0) TRACE(4, step);
+            if (build) {
+                const unsigned char* sg = my_sgl + slot * tc::SGL_BYTES;
+                unsigned char* sb = ring + stage * tc::STAGE_BYTES + tc::A_BYTES;
+                const int x = st.ti.x, zc = st.ti.z, y0h = st.ti.y0 + tc::YH * (int)rank;
+                // singles keep the HBM swizzle: piece cc of absolute row r sits at piece cc ^ (r & 7)
+                const uint4 x0 = *reinterpret_cast<const uint4*>(sg + tc::SX_OFF + ((cc ^ ((2 * x) & 7)) << 4));
+                const uint4 x1 = *reinterpret_cast<const uint4*>(sg + tc::SX_OFF + 128 + ((cc ^ ((2 * x + 1) & 7)) << 4));
+                const uint4 z0 = *reinterpret_cast<const uint4*>(sg + tc::SZ_OFF + ((cc ^ ((2 * zc) & 7)) << 4));
+                const uint4 z1 = *reinterpret_cast<const uint4*>(sg + tc::SZ_OFF + 128 + ((cc ^ ((2 * zc + 1) & 7)) << 4));
+                const unsigned char* ybase = sg + tc::SY_OFF + (2 * yq + cpl) * 128;
+                const int ra0 = 2 * y0h + 2 * yq + cpl;                        // absolute row of k = 0
+                const uint32_t yo0 = (uint32_t)((cc ^ (ra0 & 7)) << 4), yo1 = (uint32_t)((cc ^ ((ra0 + 4) & 7)) << 4);
+                uint4 yv[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                    yv[k] = *reinterpret_cast<const uint4*>(ybase + k * 512 + ((k & 1) ? yo1 : yo0));
+                if (lane == 0) TRACE(5, step);
                 const uint4 xz[4] = {and4(x0, z0), and4(x0, z1), and4(x1, z0), and4(x1, z1)};   // [b*2 + d]
-                uint4 yv[8];
 #pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    const int rr = 2 * ((lane >> 4) + 2 * k) + cpl;        // row inside the y slab
-                    const int ra = 2 * y0 + rr;                            // absolute row (for the swizzle)
-                    yv[k] = *reinterpret_cast<const uint4*>(sbase + tc::SY_OFF + rr * 128 + ((cc ^ (ra & 7)) << 4));
-                }
+                for (int k = 0; k < 4; ++k)
 #pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    const int yl = (lane >> 4) + 2 * k;
-#pragma unroll
-                    for (int bd = 0; bd < 4; ++bd) {
-                        const int n = yl * 8 + (bd >> 1) * 4 + cpl * 2 + (bd & 1);
-                        *reinterpret_cast<uint4*>(sb + sw128_off(n, cc)) = and4(yv[k], xz[bd]);
-                    }
-                }
+                    for (int bd = 0; bd < 4; ++bd)
+                        *reinterpret_cast<uint4*>(sb + boff[bd] + k * 2048) = and4(yv[k], xz[bd]);
+                if (lane == 0) TRACE(6, step);
                 fence_proxy_async();                      // generic-proxy stores -> visible to the tensor core
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&full_bar[stage]);
-            if (timing) t_busy += clock64() - t1;
+            const long long t2 = PCLK();
+            if (lane == 0) {
+                TRACE(7, step);
+                mbar_wait(&sfull_bar[stage], phase);      // this CTA's A landed
+                TRACE(8, step);
+                if (leader) mbar_arrive_local(&full_bar[stage]);
+                else mbar_arrive_cluster(&full_bar[stage], 0);           // the leader's barrier
+                TRACE(9, step);
+            }
+            __syncwarp();
+            if (EPI4_PROF) {
+                const long long t3 = PCLK();
+                t_busy += t3 - t1;
+                t_arr += t3 - t2;
+            }
+            st.advance(sp, tc::PROD_WARPS);
+            if (++slot == tc::SGL_SLOTS) slot = 0;
+            stage += tc::PROD_WARPS;
+            if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; }
         }
-        if (timing && lane == 0) {
+        cp_async_wait<0>();
+        if (EPI4_PROF && lane == 0) {
             atomicAdd(sp.prof + 3, (unsigned long long)t_busy);
             atomicAdd(sp.prof + 4, (unsigned long long)t_wait);
+            atomicAdd(sp.prof + 7, (unsigned long long)t_arr);
         }
-    } else if (warp >= tc::EPI_WARP0) {
+    } else {
         // ===================== epilogue =====================
         // lane quadrant q holds rows 32q..32q+31 = (w_local, a) with w_local = row/2; a 16-column group g
         // holds y_local = 2g, 2g+1 x (b, c, d).  Lanes a=0/a=1 swap halves so that lane a owns the quad
         // y_local = 2g + a with all 16 counts c16[8a' + 4b + 2c + d].
         const int ew = warp - tc::EPI_WARP0;           // 0..7
         const int q = warp & 3;                         // TMEM lane quadrant this warp may access
-        const int h = ew >> 2;                          // warps of one quadrant split the column groups
+        const int h = ew >> 2;                          // two warps per quadrant split the column groups
         const int row = q * 32 + lane;
         const int wl = row >> 1, a = row & 1;
         unsigned long long my_quads = 0, n_exact = 0;
         long long t_wait = 0, t_busy = 0;
-        const bool timing = (sp.debug & 8) != 0;
+        const bool score = !(sp.debug & 2);
         int it = 0;
-        for (int64_t tile = first_group; tile < sp.ntiles; tile += group_stride, ++it) {
+        for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
             const TileInfo ti = decode_tile(sp, tile);
             const int buf = it & 1;
             const uint32_t tphase = (uint32_t)((it >> 1) & 1);
-            const long long t0 = timing ? clock64() : 0;
+            const long long t0 = PCLK();
             mbar_wait(&tfull_bar[buf], tphase);
-            const long long t1 = timing ? clock64() : 0;
+            const long long t1 = PCLK();
             t_wait += t1 - t0;
             tc_fence_after();
-            const int w = ti.wr * EPI4_WR + wl;
+            const int w = (ti.wp * 2 + (int)rank) * EPI4_WR + wl;
             const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * 256);
 #pragma unroll 1
-            for (int g = h; g < 8; g += tc::EPI_SPLIT) {
+            for (int g = h; g < 8; g += 2) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(tbase + 16 * g, v0);
                 tmem_ld16(tbase + 128 + 16 * g, v1);
                 tmem_wait_ld();
-                if (g + tc::EPI_SPLIT >= 8) {
+                tmem_zero16(tbase + 16 * g);              // ready for the next tile's accumulation
+                tmem_zero16(tbase + 128 + 16 * g);
+                if (g + 2 >= 8) {
+                    tmem_wait_st();
                     tc_fence_before();
                     __syncwarp();
-                    if (lane == 0) mbar_arrive(&tempty_bar[buf]);
+                    if (lane == 0) {
+                        if (leader) mbar_arrive_local(&tempty_bar[buf]);
+                        else mbar_arrive_cluster(&tempty_bar[buf], 0);   // the leader's barrier
+                    }
                 }
                 uint32_t c0[16], c1[16];
 #pragma unroll
@@ -481,7 +573,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
                     c1[8 + k] = a ? v1[8 + k] : r1;
                 }
                 const int y = ti.y0 + 2 * g + a;
-                const bool valid = (w < ti.x) && (y < ti.z) && (ti.z < d.n) && !(sp.debug & 2);
+                const bool valid = (w < ti.x) && (y < ti.z) && score;
                 double key = 0.0;
                 uint64_t idx = 0;
                 bool offer = false;
@@ -509,7 +601,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
                 }
                 warp_offer(tk, offer, key, idx);
             }
-            if (timing) t_busy += clock64() - t1;
+            t_busy += PCLK() - t1;
         }
         unsigned long long v = my_quads, ne = n_exact;
 #pragma unroll
@@ -520,18 +612,28 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         if (lane == 0) {
             atomicAdd(sp.quads_done, v);
             atomicAdd(sp.prof + 0, ne);
-            if (timing) {
+            if (EPI4_PROF) {
                 atomicAdd(sp.prof + 1, (unsigned long long)t_busy);
                 atomicAdd(sp.prof + 2, (unsigned long long)t_wait);
             }
         }
     }
     tc_fence_before();
-    cluster_sync_all();                  // no CTA leaves while cluster peers may still signal it
+    cluster_sync_all();                  // no CTA leaves while its peer may still signal it / read its smem
     tc_fence_after();
     if (warp == 0)
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tc::TMEM_COLS));
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tc::TMEM_COLS));
     topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
+#if EPI4_PROF
+    if (tracing && tid == 0) {
+        for (int k = 0; k < TR_STEPS; ++k)
+            printf("TR %u %d %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld\n", rank, k,
+                   g_trace[rank][0][k], g_trace[rank][1][k], g_trace[rank][2][k], g_trace[rank][3][k],
+                   g_trace[rank][4][k], g_trace[rank][5][k], g_trace[rank][6][k], g_trace[rank][7][k],
+                   g_trace[rank][8][k], g_trace[rank][9][k], g_trace[rank][10][k], g_trace[rank][11][k],
+                   g_trace[rank][12][k], g_trace[rank][13][k]);
+    }
+#endif
 }
 
 template <int STAGES>
@@ -553,7 +655,9 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     return cudaLaunchKernelEx(&cfg, k_quad_i8tc<STAGES>, sp);
 }
 
-int32_t quad_group(int32_t pipe) { return pipe == EPI4_PIPE_I8TC ? tc::CLUSTER : 1; }
+// tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
+// cluster (1 tile); the CUDA-core kernel processes them as 2 tiles
+int32_t quad_split(int32_t pipe) { return pipe == EPI4_PIPE_I8TC ? 1 : 2; }
 
 cudaError_t launch_quad_i8tc(const SearchParams& sp_in, int32_t grid, cudaStream_t s, int64_t* launches) {
     SearchParams sp = sp_in;
@@ -561,22 +665,37 @@ cudaError_t launch_quad_i8tc(const SearchParams& sp_in, int32_t grid, cudaStream
     int dev = 0, optin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024;   // alignment + static smem slack
+    const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024 +   // alignment + static smem slack
+                         (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES;
     const size_t lfx_bytes = (size_t)((sp.d.lfx_n + 3) & ~3) * sizeof(int32_t);
-    // most pipeline stages that fit; the fixed-point K2 filter table in smem is preferred, falling back to
-    // exact-only scoring when it cannot fit with at least 2 stages
+    // most pipeline stages that fit (a multiple of the producer warp count: each warp takes every
+    // PROD_WARPS-th step); the fixed-point K2 filter table in smem is preferred, falling back to exact-only
+    // scoring when it cannot fit with the minimum ring
     int st = 0;
     for (int pass = 0; pass < 2 && !st; ++pass) {
-        sp.use_lfx = pass == 0 && sp.d.lfx != nullptr && !(sp.debug & 16);   // debug 16: no table, more stages
-        for (int cand = 5; cand >= 2 && !st; --cand)
+        sp.use_lfx = pass == 0 && sp.d.lfx != nullptr && !(sp.debug & 16);   // debug 16: no table
+        for (int cand = tc::MAX_STAGES / tc::STAGE_Q * tc::STAGE_Q; cand >= tc::STAGE_Q && !st; cand -= tc::STAGE_Q)
             if (fixed + (size_t)cand * tc::STAGE_BYTES + (sp.use_lfx ? lfx_bytes : 0) <= (size_t)optin) st = cand;
     }
     if (!st) return cudaErrorInvalidConfiguration;
-    const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + (sp.use_lfx ? lfx_bytes : 0) + topk_smem_bytes(sp.topk);
-    cudaError_t e = st == 5 ? launch_cfg<5>(sp, smem, grid, s)
-                  : st == 4 ? launch_cfg<4>(sp, smem, grid, s)
-                  : st == 3 ? launch_cfg<3>(sp, smem, grid, s)
-                            : launch_cfg<2>(sp, smem, grid, s);
+    const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES +
+                        (sp.use_lfx ? lfx_bytes : 0) + topk_smem_bytes(sp.topk);
+    if (getenv("EPI4_VERBOSE"))
+        fprintf(stderr, "k_quad_i8tc: %d producer warps, %d stages, lfx %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
+                sp.use_lfx, smem, grid);
+    cudaError_t e = cudaErrorInvalidConfiguration;
+    auto go = [&](auto S) {
+        constexpr int v = decltype(S)::value;
+        if constexpr (v % tc::STAGE_Q == 0)
+            if (st == v) e = launch_cfg<v>(sp, smem, grid, s);
+    };
+    go(std::integral_constant<int, 2>{});
+    go(std::integral_constant<int, 3>{});
+    go(std::integral_constant<int, 4>{});
+    go(std::integral_constant<int, 6>{});
+    go(std::integral_constant<int, 8>{});
+    go(std::integral_constant<int, 9>{});
+    go(std::integral_constant<int, 12>{});
     if (launches) ++*launches;
     return e;
 }
