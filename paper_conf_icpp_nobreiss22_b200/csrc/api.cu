@@ -106,6 +106,8 @@ DevData devdata(const epi4_ctx* c) {
     d.planes[1] = c->planes[1];
     d.nchunks[0] = c->nchunks[0];
     d.nchunks[1] = c->nchunks[1];
+    d.nchunks4[0] = (c->nchunks[0] + 1) / 2;
+    d.nchunks4[1] = (c->nchunks[1] + 1) / 2;
     d.n = c->n;
     d.npad = c->npad;
     d.np[0] = (uint32_t)c->np[0];
@@ -240,7 +242,7 @@ int finish_load(epi4_ctx* c) {
     }
     CU(cudaEventRecord(c->ev[2], c->stream));
     for (int p = 0; p < 2; ++p) {
-        CU(grow(c->expl[p], c->cap_expl[p], (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_SAMPLES));
+        CU(grow(c->expl[p], c->cap_expl[p], (size_t)((c->nchunks[p] + 1) / 2) * c->npad * 2 * 128));   // fp4 rows
         CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
     }
     CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, c->stream, &c->stats.launches_load));
@@ -256,7 +258,7 @@ int finish_load(epi4_ctx* c) {
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
     c->loaded = false;
     c->n = n;
-    c->npad = (n + EPI4_YR + EPI4_WP - 1) / EPI4_WP * EPI4_WP;
+    c->npad = (n + EPI4_YR + EPI4_WP - 1) / EPI4_WP * EPI4_WP;   // rows past n read as zero planes
     c->np[0] = n0;
     c->np[1] = n1;
     for (int p = 0; p < 2; ++p) {
@@ -506,13 +508,16 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (ub < 0) ub = 0;
     if (ub > ue) ub = ue;
     const int64_t nu = ue - ub;
-    const int32_t G = quad_split(c->opts.pipe);
+    if (c->opts.pipe != EPI4_PIPE_LOP3 && std::max(c->np[0], c->np[1]) > ((int64_t)1 << 24))
+        return fail(EPI4_EINVAL, "tensor-core pipe: fp32 accumulators are exact up to 2^24 samples per phenotype "
+                                 "(%lld, %lld); use EPI4_PIPE_LOP3", (long long)c->np[0], (long long)c->np[1]);
+    const int32_t G = quad_split(c->opts.pipe), YR = quad_yr(c->opts.pipe);
     std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
     std::vector<int64_t> prefix((size_t)std::max<int64_t>(nu, 1));
     int64_t acc = 0;
     for (int64_t i = 0; i < nu; ++i) {
         units[(size_t)i] = plan[(size_t)(ub + i)].u;
-        acc += unit_tiles(c->n, units[(size_t)i].x) * G;
+        acc += unit_tiles(c->n, units[(size_t)i].x, YR) * G;
         prefix[(size_t)i] = acc;
     }
     if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
@@ -576,7 +581,12 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     c->stats.quads = (int64_t)ctr[1];
     for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)ctr[16 + i];
     c->stats.tiles = acc / G;
-    c->stats.executed_macs = (double)(acc / G) * 2048.0 * 16.0 * (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
+    // MACs the contraction executes: 128 (w, a) rows x 8 YR columns per tile and sample (the tensor-core
+    // operands run over whole 256-sample fp4 chunks, the CUDA-core kernel over 128-sample chunks)
+    const double ksamples = c->opts.pipe == EPI4_PIPE_LOP3
+                                ? (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES
+                                : (double)((c->nchunks[0] + 1) / 2 + (c->nchunks[1] + 1) / 2) * 256.0;
+    c->stats.executed_macs = (double)(acc / G) * 128.0 * 8.0 * YR * ksamples;
     *n_out = nout;
     return 0;
 }

@@ -22,7 +22,8 @@
 #define EPI4_B 32             // SNP block size accepted in epi4_opts (32-SNP blocks)
 #define EPI4_WR 64            // w-range of one CTA / rows of its A operand: 64 SNPs x {AA, Aa}
 #define EPI4_WP 128           // w-range of a work unit (a CTA pair: two 64-SNP halves)
-#define EPI4_YR 16            // y-range of a tile: 16 consecutive SNPs after x
+#define EPI4_YR 16            // y-range of a CUDA-core (LOP3) tile: 16 consecutive SNPs after x
+#define EPI4_YR_TC 14         // y-range of a tensor-core tile (N = 112 = 14 x 8 columns; TMEM budget, k_quad_tc.cu)
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
 
@@ -51,7 +52,8 @@ __host__ __device__ __forceinline__ uint64_t pack_quad(int i, int j, int k, int 
 // Everything a kernel needs to read the dataset and the lower-order tables.
 struct DevData {
     const uint32_t* planes[2];   // chunked planes per phenotype
-    int32_t nchunks[2];          // chunks per phenotype
+    int32_t nchunks[2];          // 128-sample chunks per phenotype
+    int32_t nchunks4[2];         // 256-sample fp4 chunks per phenotype (rows of expl)
     int32_t n;                   // SNPs
     int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
     uint32_t np[2];              // n0, n1
@@ -72,22 +74,24 @@ __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, 
 }
 
 // A work unit (wp, x): the quads (w, x, y, z) with w in the 128-SNP range [128 wp, 128 wp + 128), w < x,
-// second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + 16) with y0 = x + 1 + 16k,
-// and z in (y0, n); a tile holds 128 x 16 (w, y) combinations, split into the two 64-SNP halves of the
-// w-range (the two CTAs of a tensor-core cluster, or two tiles of the CUDA-core kernel).
+// second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + yr) with y0 = x + 1 + yr k,
+// and z in (y0, n); a tile holds 128 x yr (w, y) combinations (yr = 14 tensor core, 16 CUDA core), split into
+// the two 64-SNP halves of the w-range (the two CTAs of a tensor-core cluster, or two tiles of the CUDA-core
+// kernel).
 struct Unit {
     int32_t wr, x;   // wr = 128-SNP w-range index
 };
 
-__host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x) {
+__host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x, int32_t yr = EPI4_YR) {
     int64_t t = 0;
-    for (int32_t y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) t += n - y0 - 1;
+    for (int32_t y0 = x + 1; y0 <= n - 2; y0 += yr) t += n - y0 - 1;
     return t;
 }
 
-// decode tile t of unit (x) -> (y0, z)
-__device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t, int32_t& y0, int32_t& z) {
-    for (y0 = x + 1; y0 <= n - 2; y0 += EPI4_YR) {
+// decode tile t of unit (x) -> (y0, z), y-range yr
+__device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t, int32_t& y0, int32_t& z,
+                                                 int32_t yr = EPI4_YR) {
+    for (y0 = x + 1; y0 <= n - 2; y0 += yr) {
         const int64_t cnt = n - y0 - 1;
         if (t < cnt) {
             z = y0 + 1 + (int32_t)t;
@@ -147,7 +151,8 @@ cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T
                        int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_i8tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
-int32_t quad_split(int32_t pipe);
+int32_t quad_split(int32_t pipe);   // tiles per unit tile (CUDA-core kernel: the two 64-SNP halves)
+int32_t quad_yr(int32_t pipe);      // y-range of a tile
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,
                          int32_t* out_n, cudaStream_t s, int64_t* launches);
 cudaError_t launch_tables(const DevData& d, const uint64_t* quads, int64_t n, uint32_t* out, unsigned int* status,

@@ -165,26 +165,41 @@ cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t
 // ---- {0,1}-byte expansion of the planes (operands of the i8 tensor-core pipe) ---------------------
 // expl[kc][r = 2 snp + g][128 B]: byte s of row r = bit s of plane (kc, snp, g); 16-byte piece c stored
 // at piece c ^ (r & 7) (UMMA SW128 pattern, rows are 128 B so the 8-row groups are 1 KiB aligned).
-__global__ void __launch_bounds__(256) k_expand(const uint32_t* __restrict__ planes, int64_t total16,
-                                                uint8_t* __restrict__ expl) {
+// Tensor-core operand planes: E2M1 nibbles (1.0 = 0x2 for a set bit, 0 otherwise), two samples per byte
+// (sample 2j in the low nibble of byte j), 256 samples = one 128-byte K-major row per fp4 chunk C (the 128-sample
+// plane chunks 2C and 2C+1; a missing odd chunk reads as zeros).  Layout [C][row r = 2 snp + g][128 B] with
+// the UMMA 128-byte swizzle applied: 16-byte piece cc of row r stored at piece cc ^ (r & 7).
+__global__ void __launch_bounds__(256) k_expand(const uint32_t* __restrict__ planes, int32_t npad, int32_t nchunks,
+                                                int64_t total16, uint8_t* __restrict__ expl) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= total16) return;
-    const int c = (int)(t & 7);                 // 16-byte piece of the 128-sample row
-    const int64_t rowid = t >> 3;               // (kc, snp, g) = (kc, r)
-    const uint32_t word = planes[rowid * EPI4_CHUNK_WORDS + (c >> 1)];
-    const uint32_t half = (word >> (16 * (c & 1))) & 0xFFFFu;
+    const int cc = (int)(t & 7);                 // 16-byte piece (32 samples) of the 256-sample row
+    const int64_t rowid = t >> 3;                // (C, r)
+    const int64_t rows = (int64_t)npad * 2;
+    const int64_t C = rowid / rows, r = rowid - C * rows;
+    const int64_t c128 = 2 * C + (cc >> 2);
+    const uint32_t word = c128 < nchunks ? planes[(c128 * rows + r) * EPI4_CHUNK_WORDS + (cc & 3)] : 0u;
     uint32_t o[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) o[k] = (((half >> (4 * k)) & 0xFu) * 0x00204081u) & 0x01010101u;
-    const int sw = c ^ (int)(rowid & 7);
+    for (int k = 0; k < 4; ++k) {
+        uint32_t v = 0;
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+            v |= ((word >> (8 * k + 2 * b)) & 1u) << (8 * b + 1);
+            v |= ((word >> (8 * k + 2 * b + 1)) & 1u) << (8 * b + 5);
+        }
+        o[k] = v;
+    }
+    const int sw = cc ^ (int)(r & 7);
     reinterpret_cast<uint4*>(expl)[rowid * 8 + sw] = make_uint4(o[0], o[1], o[2], o[3]);
 }
 
 cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,
                           int64_t* launches) {
-    const int64_t total16 = (int64_t)nchunks * npad * 2 * 8;
+    const int64_t nc4 = (nchunks + 1) / 2;
+    const int64_t total16 = nc4 * npad * 2 * 8;
     if (total16 > 0) {
-        k_expand<<<(unsigned)((total16 + 255) / 256), 256, 0, s>>>(planes, total16, expl);
+        k_expand<<<(unsigned)((total16 + 255) / 256), 256, 0, s>>>(planes, npad, nchunks, total16, expl);
         if (launches) ++*launches;
     }
     return cudaGetLastError();

@@ -39,7 +39,7 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
         const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);   // = 2 * unit tile + half
         const int32_t wr = sp.units[u].wr * 2 + (int32_t)(t & 1), x = sp.units[u].x;
         int32_t y0, z;
-        unit_tile_decode(d.n, x, t >> 1, y0, z);
+        unit_tile_decode(d.n, x, t >> 1, y0, z, EPI4_YR);
         const int i = tid & 63, jg = tid >> 6;
         const int w = wr * EPI4_WR + i;
 

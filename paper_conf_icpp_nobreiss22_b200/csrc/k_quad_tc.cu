@@ -1,33 +1,39 @@
 // k_quad_tc.cu — the hot kernel: 4-way contraction on the 5th-generation tensor cores
-// (tcgen05.mma.cta_group::2.kind::i8, {0,1} operands, s32 accumulators in TMEM) with the fused epilogue.
+// (tcgen05.mma.cta_group::2.kind::mxf4, E2M1 {0, 1.0} operands, fp32 accumulators in TMEM) with the fused
+// epilogue.
 //
 // What it computes: for a tile (w-range pair wp, x, y-range y0, z) and each
-// phenotype p the 256 x 128 matrix
+// phenotype p the 256 x 112 matrix
 //     C_p[(w, a)][(y, b, c, d)] = sum over samples s of phenotype p of P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]
-// for the 128 SNPs w of the range pair and the 16 SNPs y = y0..y0+15: the 16 non-aa genotype counts of the
-// 128 x 16 quads (w, x, y, z) ("a matrix with 16 values per each quad").
+// for the 128 SNPs w of the range pair and the 14 SNPs y = y0..y0+13: the 16 non-aa genotype counts of the
+// 128 x 14 quads (w, x, y, z) ("a matrix with 16 values per each quad").
 // Factorisation: the paper ANDs SNP pairs into both operands (combine);
 // here the A operand is the raw single-SNP planes (w, a), copied from HBM by the TMA engine, and x is folded
 // into the B operand, whose columns are triple products P_b(x) & P_c(y) & P_d(z) built on chip.
-// Why i8: sm_100a has no native binary tensor op (ptxas emulates mma.sync ...b1.and.popc with legacy IMMA,
-// SURVEY.md App. C); AND+POPC becomes an integer MAC on {0,1} bytes, exact in s32.
-// Why 2-CTA: a 1-CTA M=128 N=128 i8 MMA issues every ~97 cycles (5.4K MAC/clk/SM); cta_group::2 with
-// M=256 N=128 issues every 64 cycles, the full 8.2K MAC/clk/SM (tools/probe_mma.cu, profiles/).
+// Why block-scaled FP4: sm_100a has no native binary tensor op (ptxas emulates mma.sync ...b1.and.popc with
+// legacy IMMA).  A set bit is the E2M1 value 1.0 (nibble 0x2), so AND of packed nibbles
+// is the product, and with all E8M0 block scales = 1 the MMA sums exact small integers: the fp32 accumulator
+// is exact up to 2^24 per phenotype (host check; tools/probe_mxf4.cu: 0 mismatches, counts to 76800).
+// kind::mxf4 runs M=256 N=128 K=64 in 64 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the
+// operand bytes (2 samples per byte).
+// Why 2-CTA: a 1-CTA M=128 MMA issues every ~97 cycles whatever N; cta_group::2 reaches the full rate.
+// Why N = 112: TMEM holds 2 buffers x 2 phenotypes x 112 fp32 columns (448) plus the scale factors.
 //
 // CTA pair (cluster of 2): CTA r holds the A rows of w-range 2wp + r (64 SNPs x {AA, Aa}) and builds the
-// B columns of y = y0 + 8r .. y0 + 8r + 7; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
-// receives its 128 rows x all 128 columns and its epilogue scores its 64 x 16 quads.
-// Warp roles (each CTA: 12 warps, 1 CTA per SM, persistent, static tile stride over clusters):
-//   warp 0      : TMEM allocation (cta_group::2, 512 columns); leader: one thread issuing tcgen05.mma
-//   warp 1      : one thread issuing the TMA bulk copies of the CTA's stage (A 16 KiB pre-swizzled in HBM,
-//                 its 8 y planes, x, z)
-//   warps 2..3  : producers (alternating steps) — the CTA's half of B, x_b & z_d & y_c per 16-byte piece,
-//                 K-major SW128; each then arrives on the leader's `full` barrier
-//   warps 4..11 : epilogue — tcgen05.ld of the control and case accumulators, lane-pair exchange so one
-//                 thread holds one quad's 2 x 16 counts, the shared epilogue (epilogue.cuh); then an
-//                 arrival on the leader's `tempty` barrier
-// Pipelines: STAGES x {A, B half, singles} per CTA (sfull: own TMA landed; full @leader: both B halves built;
-// empty: leader's MMA commit, multicast to both CTAs); TMEM double buffer 2 x [128 ctrl | 128 case].
+// B columns of y = y0 + 7r .. y0 + 7r + 6; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
+// receives its 128 rows x all 112 columns and its epilogue scores its 64 x 14 quads.
+// Warp roles (each CTA: 15 warps, 1 CTA per SM, persistent, static tile stride over clusters):
+//   warps 0..1  : leader — MMA issuers (alternating steps, one elected lane each); follower — warp 0 relays
+//                 "A landed" to the leader's `full` barrier; warp 0 also allocates TMEM (cta_group::2)
+//   warps 2..3  : TMA issuers (alternating steps): the CTA's A, 16 KiB per step, pre-swizzled in HBM
+//   warps 4..6  : producers (every 3rd step each) — the CTA's half of B, x_b & y_c & z_d per 16-byte piece,
+//                 K-major SW128, from singles prefetched with cp.async; then an arrival on the leader's `full`
+//   warps 7..14 : epilogue — tcgen05.ld of the control and case accumulators, lane-pair exchange so one
+//                 thread holds one quad's 2 x 16 counts, re-zeroing of the accumulators, the shared epilogue
+//                 (epilogue.cuh); an arrival on the leader's `tempty` barrier
+// Pipelines: STAGES x {A, B half} per CTA (sfull: own TMA landed; full @leader: both B halves built and the
+// follower's A landed; empty: the issuer's MMA commit, multicast to both CTAs); TMEM double buffer
+// 2 x [112 ctrl | 112 case].  One step = one 256-sample fp4 chunk of one phenotype = 4 MMAs.
 #include <cstdio>
 #include <cstdlib>
 #include <type_traits>
@@ -36,16 +42,17 @@
 namespace epi4 {
 
 namespace tc {
-constexpr int M = 256, N = 128;          // UMMA shape (cta_group::2), K = 32 bytes per instruction
-constexpr int KCH = EPI4_CHUNK_SAMPLES;  // 128 samples (bytes) per pipeline stage
-constexpr int A_BYTES = 128 * KCH;       // this CTA's 128 A rows
-constexpr int B_BYTES = (N / 2) * KCH;   // this CTA's 64 B columns
-constexpr int YH = EPI4_YR / 2;          // y SNPs per CTA
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 24 KiB, 1024-aligned
+constexpr int M = 256, N = 8 * EPI4_YR_TC;   // UMMA shape (cta_group::2), K = 64 fp4 = 32 bytes per instruction
+constexpr int ROWB = 128;                // bytes of one K-major operand row per stage (256 fp4 samples)
+constexpr int A_BYTES = 128 * ROWB;      // this CTA's 128 A rows
+constexpr int B_ROWS = N / 2;            // this CTA's 56 B columns
+constexpr int B_BYTES = (B_ROWS + 7) / 8 * 1024;
+constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (7)
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 23 KiB, 1024-aligned
 constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per stage
-// singles (x, z, y-half planes of one step) prefetched by each producer warp with cp.async into its own ring
-constexpr int SX_OFF = 0, SZ_OFF = 2 * KCH, SY_OFF = 4 * KCH;
-constexpr int SGL_BYTES = (4 + 2 * YH) * KCH;              // 20 rows x 128 B
+// singles (x, z and 8 y rows-pairs of one step) prefetched by each producer warp with cp.async into its ring
+constexpr int SX_OFF = 0, SZ_OFF = 2 * ROWB, SY_OFF = 4 * ROWB;
+constexpr int SGL_BYTES = (4 + 16) * ROWB;                 // 20 rows x 128 B
 #ifndef EPI4_PF
 #define EPI4_PF 1
 #endif
@@ -57,15 +64,22 @@ constexpr int SGL_SLOTS = PF + 1;
 constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
 constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate steps (one thread cannot hide
                                          // its own wait/bookkeeping latency behind the blocking MMA issue)
-constexpr int TMA_WARP = MMA_WARPS, PROD_WARP0 = TMA_WARP + 1, EPI_WARP0 = PROD_WARP0 + PROD_WARPS;
-constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 448 with 3 producer warps: 128 registers
+constexpr int TMA_WARPS = 2;             // a bulk-copy issue blocks its thread ~150-200 cycles: two warps alternate
+constexpr int TMA_WARP0 = MMA_WARPS, PROD_WARP0 = TMA_WARP0 + TMA_WARPS, EPI_WARP0 = PROD_WARP0 + PROD_WARPS;
+constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 480 with 3 producer warps: 128 registers
 constexpr int MAX_STAGES = 12;
 constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
-constexpr int STAGE_Q = PROD_WARPS / gcd_c(PROD_WARPS, MMA_WARPS) * MMA_WARPS;   // stage counts: multiples
+constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
+constexpr int STAGE_Q = lcm_c(lcm_c(PROD_WARPS, MMA_WARPS), TMA_WARPS);   // stage counts: multiples
 constexpr int TMEM_COLS = 512;
+constexpr int ACC_COLS = 4 * N;          // [buf][p] accumulators: columns buf * 2N + p * N
+constexpr int SF_COL = 480;              // scale factors (all E8M0 0x7F = 1.0): columns 480..511, every lane
+static_assert(ACC_COLS <= SF_COL, "TMEM: accumulators overlap the scale factors");
+constexpr int NG = N / 16;               // 16-column groups of an accumulator (7)
 constexpr int CLUSTER = 2;
-// instruction descriptor: D s32 (bits 4-5 = 2), A/B u8 (0), K-major, N>>3 at bit 17, M>>4 at bit 24
-constexpr uint32_t IDESC = (2u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+// block-scaled instruction descriptor: A/B E2M1 (format 1 at bits 7 and 10), K-major, N>>3 at bit 17,
+// scale format E8M0 (bit 23), M>>4 at bit 24, scale-factor ids 0, K = 64 (bit 31 = 0)
+constexpr uint32_t IDESC = (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
 }  // namespace tc
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -133,12 +147,13 @@ __device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
     d |= (uint64_t)2 << 61;                 // SWIZZLE_128B
     return d;
 }
-// D[tmem] (+)= A[smem, both CTAs] . B[smem, both CTAs]^T for the CTA pair; issued by the leader only
-__device__ __forceinline__ void mma2_i8(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t acc) {
+// D[tmem] (+)= A[smem, both CTAs] . B[smem, both CTAs]^T for the CTA pair, E2M1 x E2M1 with the block
+// scales at sf (TMEM); issued by the leader only
+__device__ __forceinline__ void mma2_mxf4(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t sf) {
     asm volatile(
-        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %3, 0;\n\t"
-        "tcgen05.mma.cta_group::2.kind::i8 [%0], %1, %2, %4, p;\n\t}" ::"r"(d_tmem),
-        "l"(adesc), "l"(bdesc), "r"(acc), "r"(tc::IDESC));
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, 1, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::mxf4.block_scale.block32 [%0], %1, %2, %3, [%4], [%4], p;\n\t}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(tc::IDESC), "r"(sf));
 }
 // arrive (when the leader's prior MMAs complete) on the same-offset barrier of both CTAs of the pair
 __device__ __forceinline__ void mma2_commit_mc(uint64_t* bar) {
@@ -155,14 +170,14 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
         : "r"(taddr));
 }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
-// zero 16 columns of this warp's 32 TMEM lanes
-__device__ __forceinline__ void tmem_zero16(uint32_t taddr) {
-    const uint32_t z = 0;
+// fill 16 columns of this warp's 32 TMEM lanes with one 32-bit value
+__device__ __forceinline__ void tmem_fill16(uint32_t taddr, uint32_t v) {
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(taddr),
-        "r"(z)
+        "r"(v)
         : "memory");
 }
+__device__ __forceinline__ void tmem_zero16(uint32_t taddr) { tmem_fill16(taddr, 0u); }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // byte offset of (row r, 16-byte chunk c) inside a K-major SW128 tile of 128-byte rows
@@ -208,7 +223,7 @@ __device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t 
     TileInfo ti;
     ti.wp = sp.units[u].wr;
     ti.x = sp.units[u].x;
-    unit_tile_decode(sp.d.n, ti.x, t, ti.y0, ti.z);
+    unit_tile_decode(sp.d.n, ti.x, t, ti.y0, ti.z, EPI4_YR_TC);
     return ti;
 }
 
@@ -223,11 +238,13 @@ struct StepIt {
         tile = cluster_id_x();
         p = 0;
         kc = 0;
-        nch0 = sp.d.nchunks[0];
-        nch1 = sp.d.nchunks[1];
+        nch0 = sp.d.nchunks4[0];
+        nch1 = sp.d.nchunks4[1];
         if (tile < sp.ntiles) ti = decode_tile(sp, tile);
     }
     __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
+    // physical chunk of this step (a tile-dependent rotation of the K loop was measured slower: r01 notes)
+    __device__ __forceinline__ int chunk() const { return kc; }
     __device__ __forceinline__ void advance(const SearchParams& sp, int k) {
         kc += k;
         if (kc < (p ? nch1 : nch0)) return;
@@ -249,7 +266,7 @@ struct StepIt {
 #define EPI4_PROF 0
 #endif
 #if EPI4_PROF
-constexpr int TR_STEPS = 96, TR_EV = 14;
+constexpr int TR_STEPS = 96, TR_EV = 16;
 __device__ long long g_trace[2][TR_EV][TR_STEPS];
 #define TRACE(ev, step)                                                                                    \
     do {                                                                                                   \
@@ -284,7 +301,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
     if (tid == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&sfull_bar[s], 1);
-            mbar_init(&full_bar[s], tc::CLUSTER);         // (leader) one producer arrival per CTA
+            mbar_init(&full_bar[s], tc::CLUSTER + 1);     // (leader) both CTAs' producers + the follower's A relay
             mbar_init(&empty_bar[s], 1);                  // the leader's MMA commit
         }
         for (int b = 0; b < 2; ++b) {
@@ -306,7 +323,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
     if (warp >= tc::EPI_WARP0) {
         const int ew = warp - tc::EPI_WARP0, q = warp & 3, h = ew >> 2;
         const uint32_t tq = s_tmem + ((uint32_t)(q * 32) << 16);
-        for (int col = 16 * h; col < tc::TMEM_COLS; col += 32) tmem_zero16(tq + (uint32_t)col);
+        for (int col = 16 * h; col < tc::ACC_COLS; col += 32) tmem_zero16(tq + (uint32_t)col);
+        if (h == 0)                      // E8M0 scale factors 2^0 for every MMA (any layout reads 0x7F)
+            for (int col = tc::SF_COL; col < tc::TMEM_COLS; col += 16) tmem_fill16(tq + (uint32_t)col, 0x7F7F7F7Fu);
         tmem_wait_st();
     }
     tc_fence_before();
@@ -318,8 +337,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
     const long long t_base = clock64();
 #endif
     const int64_t first_tile = cluster_id_x(), tile_stride = nclusters_x();
-    const int64_t chunk_stride = (int64_t)d.npad * 2 * tc::KCH;   // bytes of one chunk of expl
-    const int nch0_r = d.nchunks[0], nch1_r = d.nchunks[1];
+    const int64_t chunk_stride = (int64_t)d.npad * 2 * tc::ROWB;  // bytes of one fp4 chunk of expl
+    const int nch0_r = d.nchunks4[0], nch1_r = d.nchunks4[1];
     const uint8_t* const expl0 = d.expl[0];
     const uint8_t* const expl1 = d.expl[1];
 
@@ -333,6 +352,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
             const int m = warp;
             const uint32_t ring_s = smem_u32(ring);
             const uint64_t adesc0 = sw128_desc(ring_s), bdesc0 = sw128_desc(ring_s + tc::A_BYTES);
+            const uint32_t sf_addr = tmem + tc::SF_COL;
             int stage = m;
             uint32_t phase = 0, soff = (uint32_t)m * (tc::STAGE_BYTES >> 4);
             int it = 0, gstep = 0;
@@ -345,22 +365,24 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
                 tc_fence_after();
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
-                    const uint32_t dcol = tmem + (uint32_t)(buf * 256 + p * 128);
+                    const uint32_t dcol = tmem + (uint32_t)(buf * 2 * tc::N + p * tc::N);
                     const int nch = p ? nch1_r : nch0_r;
 #pragma unroll 1
                     for (int kc = 0; kc < nch; ++kc, ++gstep) {
                         if ((gstep & (tc::MMA_WARPS - 1)) != m) continue;
                         const long long t0 = PCLK();
                         if (lane == 0) TRACE(12, gstep);
-                        mbar_wait(&full_bar[stage], phase);         // both B halves built, both A halves landed
+                        mbar_wait(&full_bar[stage], phase);         // both B halves built, follower's A landed
+                        if (lane == 0) TRACE(15, gstep);
+                        mbar_wait(&sfull_bar[stage], phase);        // own A landed
                         t_wait += PCLK() - t0;
                         if (lane == 0) TRACE(10, gstep);
                         tc_fence_after();
                         if (elect_one()) {
                             if (do_mma) {
 #pragma unroll
-                                for (int k = 0; k < tc::KCH / 32; ++k)
-                                    mma2_i8(dcol, adesc0 + soff + 2 * k, bdesc0 + soff + 2 * k, 1u);
+                                for (int k = 0; k < tc::ROWB / 32; ++k)
+                                    mma2_mxf4(dcol, adesc0 + soff + 2 * k, bdesc0 + soff + 2 * k, sf_addr);
                             }
                             mma2_commit_mc(&empty_bar[stage]);      // frees the stage in both CTAs
                         }
@@ -375,46 +397,64 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
                 __syncwarp();
             }
             if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
-        }
-        __syncwarp();
-    } else if (warp == tc::TMA_WARP) {
-        // ===================== TMA issuer: this CTA's A (16 KiB per step) =====================
-        // whole warp runs the loop (uniform operands), one elected lane issues
-        {
+        } else if (warp == 0) {
+            // follower: relay "my A landed" (sfull) to the leader's full barrier, off the producers' path
             int stage = 0;
             uint32_t phase = 0;
             StepIt st;
             st.init(sp);
+            for (int gstep = 0; st.valid(sp); st.advance(sp, 1), ++gstep) {
+                mbar_wait(&sfull_bar[stage], phase);
+                if (lane == 0) TRACE(14, gstep);
+                if (lane == 0) mbar_arrive_cluster(&full_bar[stage], 0);
+                __syncwarp();
+                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+            }
+        }
+        __syncwarp();
+    } else if (warp < tc::PROD_WARP0) {
+        // ===================== TMA issuers: this CTA's A (16 KiB per step) =====================
+        // warp t takes the steps s with s % TMA_WARPS == t; the whole warp runs the loop (uniform operands),
+        // one elected lane issues
+        {
+            const int tw = warp - tc::TMA_WARP0;
+            int stage = tw;
+            uint32_t phase = 0;
+            StepIt st;
+            st.init(sp);
+            st.advance(sp, tw);
             long long t_wait = 0;
             const uint32_t ring_s = smem_u32(ring);
-            for (int gstep = 0; st.valid(sp); st.advance(sp, 1), ++gstep) {
+            for (int gstep = tw; st.valid(sp); st.advance(sp, tc::TMA_WARPS), gstep += tc::TMA_WARPS) {
                 const long long t0 = PCLK();
                 mbar_wait(&empty_bar[stage], phase ^ 1u);
                 t_wait += PCLK() - t0;
                 if (lane == 0) TRACE(0, gstep);
-                const uint8_t* E = (st.p ? expl1 : expl0) + (int64_t)st.kc * chunk_stride;
+                const uint8_t* E = (st.p ? expl1 : expl0) + (int64_t)st.chunk() * chunk_stride;
                 const int64_t wrow = (int64_t)(st.ti.wp * 2 + (int)rank) * EPI4_WR * 2;   // first A row
                 if (elect_one()) {
                     mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                                 ::"r"(ring_s + (uint32_t)(stage * tc::STAGE_BYTES)), "l"(E + wrow * tc::KCH),
+                                 ::"r"(ring_s + (uint32_t)(stage * tc::STAGE_BYTES)), "l"(E + wrow * tc::ROWB),
                                  "r"((uint32_t)tc::A_BYTES), "r"(smem_u32(&sfull_bar[stage]))
                                  : "memory");
                 }
                 __syncwarp();
                 if (lane == 0) TRACE(1, gstep);
-                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+                stage += tc::TMA_WARPS;
+                if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; }
             }
             if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
         }
     } else if (warp < tc::EPI_WARP0) {
         // ===================== producers =====================
         // Producer warp j builds this CTA's B half of every step s with s % PROD_WARPS == j.  Its singles
-        // (x, z and the CTA's 8 y SNPs: 20 rows of 128 B, pre-swizzled in HBM) are prefetched PF own steps
-        // ahead with cp.async into the warp's private ring.  Lane: 16-byte piece cc = lane & 7 of the
-        // 128-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k (k = 0..3);
-        // B[n = 8 y_local + 4b + 2c + d] = x_b & y_c & z_d.  The warp waits for its CTA's A (sfull) before
-        // arriving on the leader's `full` barrier, so `full` also certifies the follower's A.
+        // (x, z and 8 y SNPs of which the CTA's 7 are used: 20 rows of 128 B, pre-swizzled in HBM) are
+        // prefetched PF own steps ahead with cp.async into the warp's private ring.  Lane: 16-byte piece
+        // cc = lane & 7 of the 256-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k
+        // (k = 0..3, y_local < 7); B[n = 8 y_local + 4b + 2c + d] = x_b & y_c & z_d (a nibble-wise AND of
+        // E2M1 {0, 1.0} values is their product).  The follower's A is certified to the leader by the relay
+        // warp, so producers never wait for the TMA.
         const int pw = warp - tc::PROD_WARP0;
         const int cc = lane & 7, cpl = (lane >> 3) & 1, yq = lane >> 4;
         const bool build = !(sp.debug & 1);
@@ -435,11 +475,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
         pre = st;
         auto prefetch = [&](int slot, const StepIt& it) {
             if (it.valid(sp)) {
-                const uint8_t* E = (it.p ? expl1 : expl0) + (int64_t)it.kc * chunk_stride;
+                const uint8_t* E = (it.p ? expl1 : expl0) + (int64_t)it.chunk() * chunk_stride;
                 unsigned char* dst = my_sgl + slot * tc::SGL_BYTES;
-                const uint8_t* srcxz = E + (int64_t)(lane < 16 ? it.ti.x : it.ti.z) * 2 * tc::KCH + pxz;
+                const uint8_t* srcxz = E + (int64_t)(lane < 16 ? it.ti.x : it.ti.z) * 2 * tc::ROWB + pxz;
                 cp_async16(dst + lane * 16, srcxz);
-                const uint8_t* srcy = E + (int64_t)(it.ti.y0 + tc::YH * (int)rank) * 2 * tc::KCH + lane * 16;
+                const uint8_t* srcy = E + (int64_t)(it.ti.y0 + tc::YH * (int)rank) * 2 * tc::ROWB + lane * 16;
 #pragma unroll
                 for (int k = 0; k < 4; ++k) cp_async16(dst + tc::SY_OFF + k * 512 + lane * 16, srcy + k * 512);
             }
@@ -484,9 +524,10 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
                 const uint4 xz[4] = {and4(x0, z0), and4(x0, z1), and4(x1, z0), and4(x1, z1)};   // [b*2 + d]
 #pragma unroll
                 for (int k = 0; k < 4; ++k)
+                    if (k < 3 || yq == 0)                 // y_local = 7 is the other CTA's
 #pragma unroll
-                    for (int bd = 0; bd < 4; ++bd)
-                        *reinterpret_cast<uint4*>(sb + boff[bd] + k * 2048) = and4(yv[k], xz[bd]);
+                        for (int bd = 0; bd < 4; ++bd)
+                            *reinterpret_cast<uint4*>(sb + boff[bd] + k * 2048) = and4(yv[k], xz[bd]);
                 if (lane == 0) TRACE(6, step);
                 fence_proxy_async();                      // generic-proxy stores -> visible to the tensor core
             }
@@ -494,8 +535,6 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
             const long long t2 = PCLK();
             if (lane == 0) {
                 TRACE(7, step);
-                mbar_wait(&sfull_bar[stage], phase);      // this CTA's A landed
-                TRACE(8, step);
                 if (leader) mbar_arrive_local(&full_bar[stage]);
                 else mbar_arrive_cluster(&full_bar[stage], 0);           // the leader's barrier
                 TRACE(9, step);
@@ -541,16 +580,21 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
             t_wait += t1 - t0;
             tc_fence_after();
             const int w = (ti.wp * 2 + (int)rank) * EPI4_WR + wl;
-            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * 256);
+            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * 2 * tc::N);
 #pragma unroll 1
-            for (int g = h; g < 8; g += 2) {
+            for (int g = h; g < tc::NG; g += 2) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(tbase + 16 * g, v0);
-                tmem_ld16(tbase + 128 + 16 * g, v1);
+                tmem_ld16(tbase + tc::N + 16 * g, v1);
                 tmem_wait_ld();
                 tmem_zero16(tbase + 16 * g);              // ready for the next tile's accumulation
-                tmem_zero16(tbase + 128 + 16 * g);
-                if (g + 2 >= 8) {
+                tmem_zero16(tbase + tc::N + 16 * g);
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {            // fp32 accumulators hold exact integers
+                    v0[k] = (uint32_t)__uint_as_float(v0[k]);
+                    v1[k] = (uint32_t)__uint_as_float(v1[k]);
+                }
+                if (g + 2 >= tc::NG) {
                     tmem_wait_st();
                     tc_fence_before();
                     __syncwarp();
@@ -627,11 +671,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
 #if EPI4_PROF
     if (tracing && tid == 0) {
         for (int k = 0; k < TR_STEPS; ++k)
-            printf("TR %u %d %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld\n", rank, k,
+            printf("TR %u %d %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld %lld\n", rank, k,
                    g_trace[rank][0][k], g_trace[rank][1][k], g_trace[rank][2][k], g_trace[rank][3][k],
                    g_trace[rank][4][k], g_trace[rank][5][k], g_trace[rank][6][k], g_trace[rank][7][k],
                    g_trace[rank][8][k], g_trace[rank][9][k], g_trace[rank][10][k], g_trace[rank][11][k],
-                   g_trace[rank][12][k], g_trace[rank][13][k]);
+                   g_trace[rank][12][k], g_trace[rank][13][k], g_trace[rank][14][k], g_trace[rank][15][k]);
     }
 #endif
 }
@@ -657,7 +701,8 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
 // cluster (1 tile); the CUDA-core kernel processes them as 2 tiles
-int32_t quad_split(int32_t pipe) { return pipe == EPI4_PIPE_I8TC ? 1 : 2; }
+int32_t quad_split(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? 2 : 1; }
+int32_t quad_yr(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? EPI4_YR : EPI4_YR_TC; }
 
 cudaError_t launch_quad_i8tc(const SearchParams& sp_in, int32_t grid, cudaStream_t s, int64_t* launches) {
     SearchParams sp = sp_in;
