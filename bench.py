@@ -2,7 +2,7 @@
 """Benchmark of the exhaustive fourth-order K2 search (BASELINE.json metric: tera quads/s scaled to
 sample size, C(N,4)*M / t).
 
-  python bench.py --gpus N --steps K --warmup W [--config C2] [--pipe i8tc] [--impl ours|reference]
+  python bench.py --gpus N --steps K --warmup W [--config C2] [--pipe tc] [--impl ours|reference]
 
 A step = one pass of the whole hot path over the config's synthetic dataset:
 pack the byte genotypes into bit planes (a1), T1/T2/T3 (a2, a4), the 4-way contraction with the fused
@@ -195,11 +195,13 @@ def run_ours(args):
     st = eng.stats()
     pk, pk_src = peaks()
     useful_macs = 16.0 * comb4(n) * m / world
-    if args.pipe == "i8tc":
-        peak = 2.0 * pk["bf16_tflops_sustained"]          # i8 dense = 2 x bf16 (guide nominal ratio)
+    if args.pipe == "tc":
+        # kind::mxf4 (E2M1 operands): dense fp4 = 4 x bf16 (guide nominal 9 / 2.25 PFLOP/s), sustained
+        # figure because the kernel runs for ~1 s or more inside a long step
+        peak = 4.0 * pk["bf16_tflops_sustained"]
         bound, unit = "tensor", "TFLOP/s"
-        achieved = 2.0 * useful_macs / (t_quad / 1e3) / 1e12  # int8 ops (2 per MAC) per second
-        peak_note = f"{pk_src} bf16_tflops_sustained x 2 (i8/bf16 nominal ratio)"
+        achieved = 2.0 * useful_macs / (t_quad / 1e3) / 1e12  # fp4 ops (2 per {0,1}-MAC) per second
+        peak_note = f"{pk_src} bf16_tflops_sustained x 4 (fp4/bf16 nominal ratio, kind::mxf4)"
     else:
         # ALU-bound popcount pipe: 16 POPC/clk/SM x 32 bit-MACs x 148 SMs x sm_max clock, 2 ops per MAC
         peak = 2.0 * 16 * 32 * 148 * pk.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
@@ -216,7 +218,7 @@ def run_ours(args):
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": t_step, "higher_is_better": True, "scaling": "strong",
-        "vs_baseline": None, "dtype": "u8" if args.pipe == "i8tc" else "u32",
+        "vs_baseline": None, "dtype": "e2m1 (mxf4, f32 accum)" if args.pipe == "tc" else "u32",
         "data": "synthetic (seeded HWE genotypes + planted 4-way interaction, SURVEY.md §8(d))",
         "config": {"workload": f"{args.config}: N={n} SNPs, M={m} samples ({d.n_controls} controls / "
                                f"{d.n_cases} cases), exhaustive C(N,4)={comb4(n)} quads, top_k={top_k}",
@@ -284,7 +286,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2", choices=list(datagen.CONFIGS))
-    ap.add_argument("--pipe", default="i8tc", choices=["i8tc", "lop3"])
+    ap.add_argument("--pipe", default="tc", choices=["tc", "lop3"])
     ap.add_argument("--top-k", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

@@ -34,7 +34,7 @@ extern "C" {
 #define EPI4_ENODEV  (-5)  /* no sm_100 device / the requested device is unusable */
 
 /* ---- options ---------------------------------------------------------------------------- */
-#define EPI4_PIPE_I8TC  0  /* tcgen05.mma kind::i8 on {0,1}-expanded tiles, TMEM accumulators */
+#define EPI4_PIPE_TC    0  /* tcgen05.mma.cta_group::2.kind::mxf4 on E2M1 {0,1} nibble tiles, fp32 TMEM accumulators */
 #define EPI4_PIPE_LOP3  1  /* CUDA-core LOP3 (AND) + POPC contraction (cross-check path) */
 
 #define EPI4_PTR_HOST   0
@@ -53,7 +53,7 @@ typedef struct {
     int32_t reserved[3];
 } epi4_opts;
 
-/* Fill *opts with defaults (block 32, pipe I8TC, rank 0, world 1, grid 0). */
+/* Fill *opts with defaults (block 32, pipe TC, rank 0, world 1, grid 0). */
 void epi4_default_opts(epi4_opts* opts);
 
 /* Create a context on CUDA device `cuda_device` (selects it on the calling thread).

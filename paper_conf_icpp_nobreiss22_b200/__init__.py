@@ -28,7 +28,7 @@ def unpack_index(idx) -> tuple:
 class Epi4:
     """One search context on one GPU (one per rank)."""
 
-    def __init__(self, device: int = 0, pipe: str = "i8tc", rank: int = 0, world: int = 1, grid: int = 0,
+    def __init__(self, device: int = 0, pipe: str = "tc", rank: int = 0, world: int = 1, grid: int = 0,
                  debug: int = 0):
         o = binding.epi4_default_opts()
         o.pipe = binding.PIPES[pipe]

@@ -18,10 +18,10 @@ LIB_PATH = os.path.join(HERE, "libepi4.so")
 HEADER = os.path.join(os.path.dirname(HERE), "include", "epi4.h")
 
 EPI4_OK, EPI4_EINVAL, EPI4_ENOMEM, EPI4_ECUDA, EPI4_ESTATE, EPI4_ENODEV = 0, -1, -2, -3, -4, -5
-EPI4_PIPE_I8TC, EPI4_PIPE_LOP3 = 0, 1
+EPI4_PIPE_TC, EPI4_PIPE_LOP3 = 0, 1
 EPI4_PTR_HOST, EPI4_PTR_DEVICE = 0, 1
 EPI4_MAX_TOPK = 1024
-PIPES = {"i8tc": EPI4_PIPE_I8TC, "lop3": EPI4_PIPE_LOP3}
+PIPES = {"tc": EPI4_PIPE_TC, "lop3": EPI4_PIPE_LOP3}
 
 
 class Epi4Error(RuntimeError):

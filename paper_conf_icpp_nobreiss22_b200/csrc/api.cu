@@ -288,7 +288,7 @@ void epi4_default_opts(epi4_opts* o) {
     if (!o) return;
     std::memset(o, 0, sizeof *o);
     o->block = EPI4_B;
-    o->pipe = EPI4_PIPE_I8TC;
+    o->pipe = EPI4_PIPE_TC;
     o->rank = 0;
     o->world = 1;
     o->grid = 0;
@@ -297,7 +297,7 @@ void epi4_default_opts(epi4_opts* o) {
 const char* epi4_last_error(void) { return g_err.c_str(); }
 
 const char* epi4_version(void) {
-    return "libepi4 sm_100a (pipes: i8tc=tcgen05.mma.kind::i8, lop3=CUDA-core AND+POPC)";
+    return "libepi4 sm_100a (pipes: tc=tcgen05.mma.cta_group::2.kind::mxf4, lop3=CUDA-core AND+POPC)";
 }
 
 int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
@@ -307,7 +307,7 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
     epi4_default_opts(&o);
     if (opts) o = *opts;
     if (o.block != EPI4_B) return fail(EPI4_EINVAL, "block=%d: only B=32 is supported", o.block);
-    if (o.pipe != EPI4_PIPE_I8TC && o.pipe != EPI4_PIPE_LOP3) return fail(EPI4_EINVAL, "unknown pipe %d", o.pipe);
+    if (o.pipe != EPI4_PIPE_TC && o.pipe != EPI4_PIPE_LOP3) return fail(EPI4_EINVAL, "unknown pipe %d", o.pipe);
     if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return fail(EPI4_EINVAL, "bad rank/world %d/%d", o.rank, o.world);
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(EPI4_ENODEV, "no CUDA device");
@@ -560,7 +560,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaEventRecord(c->ev[2], c->stream));
     if (acc > 0) {
         cudaError_t e = c->opts.pipe == EPI4_PIPE_LOP3 ? launch_quad_lop3(sp, grid, c->stream, &c->stats.launches)
-                                                       : launch_quad_i8tc(sp, grid, c->stream, &c->stats.launches);
+                                                       : launch_quad_tc(sp, grid, c->stream, &c->stats.launches);
         CU(e);
     }
     CU(cudaEventRecord(c->ev[3], c->stream));

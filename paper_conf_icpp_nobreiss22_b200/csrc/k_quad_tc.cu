@@ -279,7 +279,7 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 #endif
 
 template <int STAGES>
-__global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
+__global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     static_assert(STAGES % tc::STAGE_Q == 0, "a producer's / issuer's successive uses of a stage must be one phase apart");
     extern __shared__ unsigned char smem_raw[];
     __shared__ __align__(8) uint64_t sfull_bar[STAGES], full_bar[STAGES], empty_bar[STAGES];
@@ -682,7 +682,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_i8tc(SearchParams sp) {
 
 template <int STAGES>
 static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
-    cudaError_t e = cudaFuncSetAttribute(k_quad_i8tc<STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
@@ -696,7 +696,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_quad_i8tc<STAGES>, sp);
+    return cudaLaunchKernelEx(&cfg, k_quad_tc<STAGES>, sp);
 }
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
@@ -704,7 +704,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
 int32_t quad_split(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? 2 : 1; }
 int32_t quad_yr(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? EPI4_YR : EPI4_YR_TC; }
 
-cudaError_t launch_quad_i8tc(const SearchParams& sp_in, int32_t grid, cudaStream_t s, int64_t* launches) {
+cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t s, int64_t* launches) {
     SearchParams sp = sp_in;
     grid = grid / tc::CLUSTER * tc::CLUSTER;
     int dev = 0, optin = 0;
@@ -726,7 +726,7 @@ cudaError_t launch_quad_i8tc(const SearchParams& sp_in, int32_t grid, cudaStream
     const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES +
                         (sp.use_lfx ? lfx_bytes : 0) + topk_smem_bytes(sp.topk);
     if (getenv("EPI4_VERBOSE"))
-        fprintf(stderr, "k_quad_i8tc: %d producer warps, %d stages, lfx %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
+        fprintf(stderr, "k_quad_tc: %d producer warps, %d stages, lfx %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
                 sp.use_lfx, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
     auto go = [&](auto S) {

@@ -15,7 +15,7 @@ import oracle
 
 pytestmark = pytest.mark.gpu
 
-PIPES = ["lop3", "i8tc"]
+PIPES = ["lop3", "tc"]
 
 
 def _epi():

@@ -10,7 +10,7 @@ import paper_conf_icpp_nobreiss22_b200 as epi  # noqa: E402
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
-ap.add_argument("--pipe", default="i8tc")
+ap.add_argument("--pipe", default="tc")
 ap.add_argument("--units", type=int, default=-1, help="first U units of the plan (-1 = all)")
 ap.add_argument("--top-k", type=int, default=16)
 ap.add_argument("--repeat", type=int, default=1)
