@@ -72,10 +72,8 @@ struct epi4_ctx {
     uint32_t* planes[2] = {nullptr, nullptr};
     uint32_t *T1 = nullptr, *T2 = nullptr, *T3 = nullptr;
     double* lgam = nullptr;
-    int32_t* lfx = nullptr;
-    int32_t lfx_shift = 0;
     uint8_t* expl[2] = {nullptr, nullptr};
-    size_t cap_planes[2] = {0, 0}, cap_T1 = 0, cap_T2 = 0, cap_T3 = 0, cap_lgam = 0, cap_lfx = 0, cap_expl[2] = {0, 0};
+    size_t cap_planes[2] = {0, 0}, cap_T1 = 0, cap_T2 = 0, cap_T3 = 0, cap_lgam = 0, cap_expl[2] = {0, 0};
     unsigned char* scratch = nullptr;     // H2D staging / pack indices
     std::vector<double> host_L;           // lgamma(n + 1), grown on demand
     size_t cap_scratch = 0;
@@ -100,6 +98,24 @@ struct epi4_ctx {
 
 namespace {
 
+// Offset of the fp32 K2 filter (epilogue.cuh, reading #16): a quad is scored exactly iff
+// ln2 A + off <= threshold, off = -81 - 81 C0 - 13.5 - E(M): K2 - (ln2 A_exact - 81 - 81 C0) > -13.5 (Stirling
+// remainder) and E(M) bounds ln2 |A - A_exact| from fp32 arithmetic (A in log2 units).  Over a quad's 243
+// terms, sum (k + 1/2) <= 2M + 203 and every argument is <= M + 2:
+//   lg2.approx: absolute error <= 2^-21 max(1, log2(M + 2)), times the coefficient (k + 1/2);
+//   per cell: FMUL + 2 FFMA, 3 roundings of relative 2^-24 of at most (n + 3/2) log2(M + 2);
+//   81-term sum (two interleaved partial sums + 1 add): 81 roundings of at most M + 81 (log2(M + 2) + 2).
+// E is doubled for safety; at M = 16384 E ~ 0.6, at M = 100003 ~ 4.
+double filter_offset(int64_t m) {
+    const double M = (double)m, u = std::ldexp(1.0, -24), l2M = std::log2(M + 2.0), ln2 = std::log(2.0);
+    const double e_log = std::ldexp(1.0, -21) * std::max(1.0, l2M) * (2.0 * M + 203.0);
+    const double e_cell = 3.0 * u * (M + 122.0) * l2M;
+    const double e_acc = 81.0 * u * (M + 81.0 * (l2M + 2.0));
+    const double E = 2.0 * ln2 * (e_log + e_cell + e_acc);
+    const double C0 = 0.5 * std::log(2.0 * M_PI) - 1.0;
+    return -81.0 - 81.0 * C0 - 13.5 - E;
+}
+
 DevData devdata(const epi4_ctx* c) {
     DevData d;
     d.planes[0] = c->planes[0];
@@ -118,11 +134,7 @@ DevData devdata(const epi4_ctx* c) {
     d.lgam = c->lgam;
     d.expl[0] = c->expl[0];
     d.expl[1] = c->expl[1];
-    d.lfx = c->lfx;
-    d.lfx_n = (int32_t)(c->np[0] + c->np[1] + 2);
-    d.lfx_inv_scale = std::ldexp(1.0, -c->lfx_shift);
-    // 243 table roundings of <= 1/2 unit each, plus slack for the double rounding of the exact K2
-    d.lfx_err = 122.0 * d.lfx_inv_scale + 1e-6;
+    d.flt_off = filter_offset(c->np[0] + c->np[1]);
     return d;
 }
 
@@ -134,7 +146,6 @@ void release_data(epi4_ctx* c) {
     dfree(c->T2);
     dfree(c->T3);
     dfree(c->lgam);
-    dfree(c->lfx);
     dfree(c->expl[0]);
     dfree(c->expl[1]);
     c->loaded = false;
@@ -225,21 +236,7 @@ int finish_load(epi4_ctx* c) {
     }
     CU(grow(c->lgam, c->cap_lgam, ((size_t)m + 2) * sizeof(double)));
     CU(cudaMemcpyAsync(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
-    // fixed-point copy for the K2 filter: every entry and every K2 (<= L[M + 81], superadditivity of
-    // log n!) must fit in int32 -> shift s = floor(log2((2^31 - 1) / L[M + 81]))
-    {
-        const double kmax = std::lgamma((double)(m + 81) + 1.0);
-        int s = 0;
-        while (s < 30 && std::ldexp(kmax, s + 1) < 2147483647.0) ++s;
-        c->lfx_shift = s;
-        std::vector<int32_t> F((size_t)m + 2);
-        for (size_t k = 0; k < F.size(); ++k) F[k] = (int32_t)std::llrint(std::ldexp(L[k], s));
-        // the double table must be resident before the async copies complete: both copies are
-        // stream-ordered and we synchronize below, so the host vectors outlive them
-        CU(grow(c->lfx, c->cap_lfx, F.size() * sizeof(int32_t)));
-        CU(cudaMemcpyAsync(c->lfx, F.data(), F.size() * sizeof(int32_t), cudaMemcpyHostToDevice, c->stream));
-        CU(cudaStreamSynchronize(c->stream));
-    }
+    CU(cudaStreamSynchronize(c->stream));   // the host table must outlive the async copy
     CU(cudaEventRecord(c->ev[2], c->stream));
     for (int p = 0; p < 2; ++p) {
         CU(grow(c->expl[p], c->cap_expl[p], (size_t)((c->nchunks[p] + 1) / 2) * c->npad * 2 * 128));   // fp4 rows
@@ -553,8 +550,8 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.status = c->d_status;
     sp.quads_done = c->d_counters + 1;
     sp.prof = c->d_counters + 16;
-    sp.use_lfx = 0;
     sp.debug = c->opts.reserved[0];
+    sp.use_filter = !(sp.debug & 16);   // debug 16: exact K2 for every quad (no filter)
 
     c->stats.launches = 0;
     CU(cudaEventRecord(c->ev[2], c->stream));

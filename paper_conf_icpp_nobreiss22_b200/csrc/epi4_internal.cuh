@@ -62,10 +62,7 @@ struct DevData {
     const uint32_t* T3;
     const double* lgam;          // M + 2 entries
     const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
-    const int32_t* lfx;          // fixed-point lgamma table round(L[n] * 2^lfx_shift), M + 2 entries
-    int32_t lfx_n;
-    double lfx_inv_scale;        // 2^-lfx_shift
-    double lfx_err;              // bound on |acc * 2^-s - K2| (filter slack)
+    double flt_off;              // fp32 K2 filter: exact-score a quad iff ln2 A + flt_off <= threshold (epilogue.cuh)
 };
 
 // offset (in uint32 words) of (chunk kc, snp, g, word w) in a chunked plane array
@@ -128,7 +125,7 @@ struct SearchParams {
     unsigned int* status;
     unsigned long long* quads_done;   // useful quads evaluated (atomicAdd once per CTA)
     unsigned long long* prof;  // [16] diagnostics: [0] exact K2 evaluations, [1..] per-role cycle counters
-    int32_t use_lfx;           // fixed-point K2 filter table resident in shared memory
+    int32_t use_filter;        // fp32 Stirling K2 filter before the exact double K2 (epilogue.cuh)
 
     int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA
 };

@@ -146,31 +146,55 @@ __device__ __forceinline__ void mobius3(int (&g)[27]) {
     }
 }
 
+// ---- the fp32 K2 filter (reading #16) -----------------------------------------------------
+// Stirling (ln k! = ln Gamma(k+1), z = k+1): ln k! = (k + 1/2) ln(k+1) - k + C0 + mu(k+1), C0 = ln(2 pi)/2 - 1,
+// 0 < mu(z) < 1/(12 z).  In a cell the "-k" parts cancel to -1 ((n+1) - r0 - r1), so with
+//     T_c = (n + 3/2) lg2(n + 2) - (r0 + 1/2) lg2(r0 + 1) - (r1 + 1/2) lg2(r1 + 1)      (fp32, MUFU lg2)
+// the cell term is t_c = ln2 T_c - 1 - C0 + [mu(n+2) - mu(r0+1) - mu(r1+1)], and over the 81 cells
+// K2 - (ln2 sum T_c - 81 - 81 C0) lies in (-13.5, 3.375).  With the fp32 rounding bound E(M) computed on the
+// host (api.cu: filter_offset), K2 > ln2 A - 81 - 81 C0 - 13.5 - E for the computed A = sum T_c, so a quad is
+// scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
+// is exactly the oracle's.  Per cell: 2 LOP3 + 7 FADD/FMUL + 2 FFMA + 3 MUFU, no table, no conversions
+// (a count r < 2^22 becomes the float 2^23 + r by an OR of the exponent bits; r + 1 and r + 1/2 then follow
+// by one exact FADD each).
+__device__ __forceinline__ float lg2_approx(float x) {
+    float y;
+    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float cell_T(int r0, int r1) {
+    const float m0 = __int_as_float(r0 | 0x4B000000), m1 = __int_as_float(r1 | 0x4B000000);   // 2^23 + r
+    const float f0 = m0 + (1.0f - 8388608.0f), f1 = m1 + (1.0f - 8388608.0f);              // r + 1
+    const float h0 = m0 + (0.5f - 8388608.0f), h1 = m1 + (0.5f - 8388608.0f);              // r + 1/2
+    const float fn = f0 + f1, hn = fn - 0.5f;                                               // n + 2, n + 3/2
+    float t = hn * lg2_approx(fn);
+    t = fmaf(-h0, lg2_approx(f0), t);
+    return fmaf(-h1, lg2_approx(f1), t);
+}
+
 // Per-quad evaluation in canonical cell order, one slab (27 cells x 2 phenotypes) at a time:
-// α = AA (cells 0..26), Aa (27..53), aa (54..80).  FIX: fixed-point K2 filter sum with the smem table lfx
-// (DESIGN.md §5); DBL: exact K2 in double, t_c = (L[r+1] - L[r0]) - L[r1], K2 += t_c, c = 0..80
-// (reading #4); DUMP: write the 2 x 81 cells (controls first).
-template <bool FIX, bool DBL, bool DUMP>
+// alpha = AA (cells 0..26), Aa (27..53), aa (54..80).  MODE 0: the fp32 filter value A = sum T_c (above);
+// MODE 1: exact K2 in double, t_c = (L[r+1] - L[r0]) - L[r1], K2 += t_c, c = 0..80 (
+// reading #4); MODE 2: exact K2 and the 2 x 81 cells written to dump (controls first).
+template <int MODE>
 __device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y, int z, const uint32_t (&c0)[16],
-                                          const uint32_t (&c1)[16], const int32_t* lfx, uint32_t& acc, double& k2,
-                                          uint32_t* dump) {
-    uint32_t a0 = 0, a1 = 0;
+                                          const uint32_t (&c1)[16], float& flt, double& k2, uint32_t* dump) {
+    float fa = 0.0f, fb = 0.0f;
     double kk = 0.0;
     auto consume = [&](const int (&T0)[27], const int (&T1)[27], int base) {
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
             const int r0 = T0[c], r1 = T1[c];
-            if (FIX) {
-                const uint32_t t = (uint32_t)lfx[r0 + r1 + 1] - (uint32_t)lfx[r0] - (uint32_t)lfx[r1];
-                if (c & 1) a1 += t; else a0 += t;
-            }
-            if (DBL) {
+            if (MODE == 0) {
+                const float t = cell_T(r0, r1);
+                if (c & 1) fb += t; else fa += t;
+            } else {
                 const double t = __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1));
                 kk = __dadd_rn(kk, t);
-            }
-            if (DUMP) {
-                dump[base + c] = (uint32_t)r0;
-                dump[81 + base + c] = (uint32_t)r1;
+                if (MODE == 2) {
+                    dump[base + c] = (uint32_t)r0;
+                    dump[81 + base + c] = (uint32_t)r1;
+                }
             }
         }
     };
@@ -184,7 +208,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y,
         mobius3(T1);
         consume(T0, T1, 27 * a);
     }
-    acc = a0 + a1;
+    flt = fa + fb;
     k2 = kk;
 }
 
@@ -193,10 +217,10 @@ __device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y,
 static __device__ __noinline__ double score_quad(const DevData& d, int w, int x, int y, int z,
                                           const uint32_t (&c0)[16], const uint32_t (&c1)[16],
                                           uint32_t* dump_row) {
-    uint32_t acc;
+    float flt;
     double k2;
-    if (dump_row) quad_eval<false, true, true>(d, w, x, y, z, c0, c1, nullptr, acc, k2, dump_row);
-    else quad_eval<false, true, false>(d, w, x, y, z, c0, c1, nullptr, acc, k2, nullptr);
+    if (dump_row) quad_eval<2>(d, w, x, y, z, c0, c1, flt, k2, dump_row);
+    else quad_eval<1>(d, w, x, y, z, c0, c1, flt, k2, nullptr);
     return k2;
 }
 

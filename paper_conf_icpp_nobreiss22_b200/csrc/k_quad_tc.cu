@@ -111,13 +111,33 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
     return ok != 0;
 }
-// Bounded wait: a pipeline bug traps (kernel error) after ~20 s instead of hanging the GPU.
+__device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity), "r"(1000000u)
+        : "memory");
+    return ok != 0;
+}
+// Bounded waits: a pipeline bug traps (kernel error) instead of hanging the GPU.  The poll loop counts
+// iterations instead of reading the clock (the clock reads made every poll ~8 instructions, and the spinning
+// warps took issue slots from the epilogue).  mbar_wait polls (latency-critical waiters); mbar_wait_sleep
+// passes a suspend-time hint so a long waiter (the epilogue waiting for a whole tile) sleeps in the barrier
+// unit until the phase completes instead of polling.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    if (mbar_try_wait(bar, parity)) return;
-    const long long t0 = clock64();
-    while (!mbar_try_wait(bar, parity)) {
-        if (clock64() - t0 > 40000000000LL) __trap();
-    }
+    uint32_t n = 0;
+    while (!mbar_try_wait(bar, parity))
+        if (++n == (1u << 30)) __trap();
+}
+#ifndef EPI4_SLEEP
+#define EPI4_SLEEP 1
+#endif
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+    if (!EPI4_SLEEP) return mbar_wait(bar, parity);
+    uint32_t n = 0;
+    while (!mbar_try_wait_sleep(bar, parity))
+        if (++n == (1u << 24)) __trap();
 }
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t tx) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(tx) : "memory");
@@ -285,14 +305,12 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     __shared__ __align__(8) uint64_t sfull_bar[STAGES], full_bar[STAGES], empty_bar[STAGES];
     __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2];
     __shared__ uint32_t s_tmem;
-    // 1024-aligned stage ring, the producers' singles rings, the fixed-point lgamma table, the top-k state
+    // 1024-aligned stage ring, the producers' singles rings, the top-k state
     // (same offsets in both CTAs of the pair: the MMA addresses the peer's operands at the same offsets)
     const uint32_t raw = smem_u32(smem_raw);
     unsigned char* ring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
     unsigned char* sgl_ring = ring + STAGES * tc::STAGE_BYTES;   // [PROD_WARPS][SGL_SLOTS][SGL_BYTES]
-    int32_t* s_lfx = reinterpret_cast<int32_t*>(sgl_ring + tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES);
-    const int lfx_words = sp.use_lfx ? ((sp.d.lfx_n + 3) & ~3) : 0;
-    TopKSmem tk = topk_carve(reinterpret_cast<unsigned char*>(s_lfx + lfx_words), sp.topk);
+    TopKSmem tk = topk_carve(sgl_ring + tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES, sp.topk);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const DevData& d = sp.d;
@@ -316,7 +334,6 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
     }
     topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);
-    for (int e = tid; e < lfx_words; e += tc::THREADS) s_lfx[e] = e < d.lfx_n ? __ldg(d.lfx + e) : 0;
     // Accumulators are zeroed by the epilogue after it reads them (and once here), so every MMA accumulates:
     // the two issuers' MMAs into one tile may then complete in any order.
     __syncthreads();                     // TMEM address visible
@@ -575,7 +592,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             const int buf = it & 1;
             const uint32_t tphase = (uint32_t)((it >> 1) & 1);
             const long long t0 = PCLK();
-            mbar_wait(&tfull_bar[buf], tphase);
+            mbar_wait_sleep(&tfull_bar[buf], tphase);
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             tc_fence_after();
@@ -590,9 +607,10 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 tmem_zero16(tbase + 16 * g);              // ready for the next tile's accumulation
                 tmem_zero16(tbase + tc::N + 16 * g);
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {            // fp32 accumulators hold exact integers
-                    v0[k] = (uint32_t)__uint_as_float(v0[k]);
-                    v1[k] = (uint32_t)__uint_as_float(v1[k]);
+                for (int k = 0; k < 16; ++k) {            // fp32 accumulators hold exact integers < 2^23:
+                    // adding 2^23 puts the integer in the mantissa bits (FADD + LOP instead of F2I)
+                    v0[k] = __float_as_uint(__uint_as_float(v0[k]) + 8388608.0f) & 0x7FFFFFu;
+                    v1[k] = __float_as_uint(__uint_as_float(v1[k]) + 8388608.0f) & 0x7FFFFFu;
                 }
                 if (g + 2 >= tc::NG) {
                     tmem_wait_st();
@@ -625,20 +643,30 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     uint32_t* dump = sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
                     offer = true;
                     if (dump) {
-                        key = score_quad(d, w, ti.x, y, ti.z, c0, c1, dump);
-                    } else if (sp.use_lfx) {
-                        // exact-bounded fixed-point filter; only possible top-k members get the exact K2
-                        uint32_t acc;
-                        double dummy;
-                        quad_eval<true, false, false>(d, w, ti.x, y, ti.z, c0, c1, s_lfx, acc, dummy, nullptr);
+                        uint32_t e0[16], e1[16];
+#pragma unroll
+                        for (int k = 0; k < 16; ++k) { e0[k] = c0[k]; e1[k] = c1[k]; }
+                        key = score_quad(d, w, ti.x, y, ti.z, e0, e1, dump);
+                    } else if (sp.use_filter) {
+                        // fp32 Stirling filter (epilogue.cuh); only possible top-k members get the exact K2
+                        float flt;
+                        double unused;
+                        quad_eval<0>(d, w, ti.x, y, ti.z, c0, c1, flt, unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
-                        offer = (double)(int32_t)acc * d.lfx_inv_scale - d.lfx_err <= thr;
+                        offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
-                            key = score_quad(d, w, ti.x, y, ti.z, c0, c1, nullptr);
+                            // rare path: the noinline exact scorer takes the counts through local memory
+                            uint32_t e0[16], e1[16];
+#pragma unroll
+                            for (int k = 0; k < 16; ++k) { e0[k] = c0[k]; e1[k] = c1[k]; }
+                            key = score_quad(d, w, ti.x, y, ti.z, e0, e1, nullptr);
                             ++n_exact;
                         }
                     } else {
-                        key = score_quad(d, w, ti.x, y, ti.z, c0, c1, nullptr);
+                        uint32_t e0[16], e1[16];
+#pragma unroll
+                        for (int k = 0; k < 16; ++k) { e0[k] = c0[k]; e1[k] = c1[k]; }
+                        key = score_quad(d, w, ti.x, y, ti.z, e0, e1, nullptr);
                     }
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;
@@ -712,22 +740,17 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024 +   // alignment + static smem slack
                          (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES;
-    const size_t lfx_bytes = (size_t)((sp.d.lfx_n + 3) & ~3) * sizeof(int32_t);
-    // most pipeline stages that fit (a multiple of the producer warp count: each warp takes every
-    // PROD_WARPS-th step); the fixed-point K2 filter table in smem is preferred, falling back to exact-only
-    // scoring when it cannot fit with the minimum ring
+    // most pipeline stages that fit (a multiple of STAGE_Q: each producer / issuer / TMA warp takes every
+    // PROD_WARPS-th / MMA_WARPS-th / TMA_WARPS-th step and must meet its stages one phase apart)
     int st = 0;
-    for (int pass = 0; pass < 2 && !st; ++pass) {
-        sp.use_lfx = pass == 0 && sp.d.lfx != nullptr && !(sp.debug & 16);   // debug 16: no table
-        for (int cand = tc::MAX_STAGES / tc::STAGE_Q * tc::STAGE_Q; cand >= tc::STAGE_Q && !st; cand -= tc::STAGE_Q)
-            if (fixed + (size_t)cand * tc::STAGE_BYTES + (sp.use_lfx ? lfx_bytes : 0) <= (size_t)optin) st = cand;
-    }
+    for (int cand = tc::MAX_STAGES / tc::STAGE_Q * tc::STAGE_Q; cand >= tc::STAGE_Q && !st; cand -= tc::STAGE_Q)
+        if (fixed + (size_t)cand * tc::STAGE_BYTES <= (size_t)optin) st = cand;
     if (!st) return cudaErrorInvalidConfiguration;
     const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES +
-                        (sp.use_lfx ? lfx_bytes : 0) + topk_smem_bytes(sp.topk);
+                        topk_smem_bytes(sp.topk);
     if (getenv("EPI4_VERBOSE"))
-        fprintf(stderr, "k_quad_tc: %d producer warps, %d stages, lfx %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
-                sp.use_lfx, smem, grid);
+        fprintf(stderr, "k_quad_tc: %d producer warps, %d stages, filter %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
+                sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
     auto go = [&](auto S) {
         constexpr int v = decltype(S)::value;
@@ -740,6 +763,7 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     go(std::integral_constant<int, 6>{});
     go(std::integral_constant<int, 8>{});
     go(std::integral_constant<int, 9>{});
+    go(std::integral_constant<int, 10>{});
     go(std::integral_constant<int, 12>{});
     if (launches) ++*launches;
     return e;
