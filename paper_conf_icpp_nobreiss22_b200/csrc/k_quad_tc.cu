@@ -59,15 +59,28 @@ constexpr int SGL_BYTES = (4 + 16) * ROWB;                 // 20 rows x 128 B
 constexpr int PF = EPI4_PF;                                // prefetch distance (own steps)
 constexpr int SGL_SLOTS = PF + 1;
 #ifndef EPI4_PROD_WARPS
-#define EPI4_PROD_WARPS 3
+#define EPI4_PROD_WARPS 4
 #endif
 constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
 constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate steps (one thread cannot hide
                                          // its own wait/bookkeeping latency behind the blocking MMA issue)
 constexpr int TMA_WARPS = 2;             // a bulk-copy issue blocks its thread ~150-200 cycles: two warps alternate
 constexpr int TMA_WARP0 = MMA_WARPS, PROD_WARP0 = TMA_WARP0 + TMA_WARPS, EPI_WARP0 = PROD_WARP0 + PROD_WARPS;
-constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 480 with 3 producer warps: 128 registers
+constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 512 with 4 producer warps (128 registers each before setmaxnreg)
 constexpr int MAX_STAGES = 12;
+// register split across the 4 warpgroups (needs the 16-warp layout: MMA+TMA | producers | 2 x epilogue)
+#ifndef EPI4_REGSPLIT
+#define EPI4_REGSPLIT 1
+#endif
+constexpr bool REGSPLIT = EPI4_REGSPLIT && PROD_WARPS == 4 && MMA_WARPS + TMA_WARPS == 4 && EPI_WARPS == 8;
+#ifndef EPI4_REGS_CTL
+#define EPI4_REGS_CTL 56
+#endif
+#ifndef EPI4_REGS_PROD
+#define EPI4_REGS_PROD 96
+#endif
+constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
+constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 56 / 96
 constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
 constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
 constexpr int STAGE_Q = lcm_c(lcm_c(PROD_WARPS, MMA_WARPS), TMA_WARPS);   // stage counts: multiples
@@ -359,6 +372,14 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     const uint8_t* const expl0 = d.expl[0];
     const uint8_t* const expl1 = d.expl[1];
 
+    // Warp-specialised register budgets (setmaxnreg, per warpgroup): the MMA/TMA issuers and the producers
+    // need few registers; the epilogue warpgroups take the rest (EPI4_REGS_EPI) so the per-quad evaluation
+    // runs without spills and with more loads in flight.
+    if (tc::REGSPLIT) {
+        if (warp < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_CTL));
+        else if (warp < 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_PROD));
+        else asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(tc::REGS_EPI));
+    }
     if (warp < tc::MMA_WARPS) {
         // ===================== MMA issuers (leader CTA) =====================
         // Issuer m takes the steps s with s % MMA_WARPS == m.  The whole warp runs the loop (warp-uniform
