@@ -124,6 +124,9 @@ DevData devdata(const epi4_ctx* c) {
     d.nchunks[1] = c->nchunks[1];
     d.nchunks4[0] = (c->nchunks[0] + 1) / 2;
     d.nchunks4[1] = (c->nchunks[1] + 1) / 2;
+    d.nsteps[0] = (d.nchunks4[0] + 1) / 2;
+    d.nsteps[1] = (d.nchunks4[1] + 1) / 2;
+    d.nrb = c->npad / 64;
     d.n = c->n;
     d.npad = c->npad;
     d.np[0] = (uint32_t)c->np[0];
@@ -239,7 +242,7 @@ int finish_load(epi4_ctx* c) {
     CU(cudaStreamSynchronize(c->stream));   // the host table must outlive the async copy
     CU(cudaEventRecord(c->ev[2], c->stream));
     for (int p = 0; p < 2; ++p) {
-        CU(grow(c->expl[p], c->cap_expl[p], (size_t)((c->nchunks[p] + 1) / 2) * c->npad * 2 * 128));   // fp4 rows
+        CU(grow(c->expl[p], c->cap_expl[p], (size_t)(((c->nchunks[p] + 1) / 2 + 1) / 2 * 2) * c->npad * 2 * 128));   // fp4 rows
         CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
     }
     CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, c->stream, &c->stats.launches_load));
@@ -578,12 +581,13 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     c->stats.quads = (int64_t)ctr[1];
     for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)ctr[16 + i];
     c->stats.tiles = acc / G;
-    // MACs the contraction executes: 128 (w, a) rows x 8 YR columns per tile and sample (the tensor-core
-    // operands run over whole 256-sample fp4 chunks, the CUDA-core kernel over 128-sample chunks)
+    // MACs the contraction executes: 256 (w, a) rows (a 128-SNP w-range) x 8 YR columns per unit tile and
+    // sample; the tensor-core operands run over whole 512-sample steps (two fp4 chunks, zero-padded), the
+    // CUDA-core kernel over 128-sample chunks
     const double ksamples = c->opts.pipe == EPI4_PIPE_LOP3
                                 ? (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES
-                                : (double)((c->nchunks[0] + 1) / 2 + (c->nchunks[1] + 1) / 2) * 256.0;
-    c->stats.executed_macs = (double)(acc / G) * 128.0 * 8.0 * YR * ksamples;
+                                : (double)(sp.d.nsteps[0] + sp.d.nsteps[1]) * 512.0;
+    c->stats.executed_macs = (double)(acc / G) * 256.0 * 8.0 * YR * ksamples;
     *n_out = nout;
     return 0;
 }

@@ -4,10 +4,11 @@
 //   planes[p]  : uint32, chunked K-major: [chunk kc][snp (padded, see npad)][g = 0 AA, 1 Aa][4 words]
 //                one chunk = 128 samples of phenotype p; pad bits are 0 (PAPER.md:L66-68 encoding,
 //                re-tiled so that consecutive SNPs are contiguous per chunk).
-//   expl[p]    : uint8 {0,1}, the same planes expanded to one byte per sample, [chunk][row r = 2 snp + g]
-//                [128 bytes] with the UMMA 128-byte swizzle applied in HBM (16-byte piece c of row r stored
-//                at piece c ^ (r & 7)), so a linear bulk copy of 8-row-aligned rows lands in the canonical
-//                K-major SW128 shared-memory layout.
+//   expl[p]    : the same planes as E2M1 {0, 1.0} nibbles (256 samples = 128 bytes per row and fp4 chunk),
+//                blocked [chunk pair][128-row block][chunk & 1][row r = 2 snp + g][128 bytes] (expl_off) with the
+//                UMMA 128-byte swizzle applied in HBM (16-byte piece c of row r stored at piece c ^ (r & 7)), so
+//                one linear 32 KiB bulk copy lands two chunks of a 128-row A tile in the canonical K-major SW128
+//                shared-memory layout; the chunk count is padded to even with zero chunks.
 //   T1[snp][p][2]          popc(P_a(snp))                              (PAPER.md:L85 indivPop)
 //   T2[rank2][p][4]        popc(P_a(i) & P_b(j)), i<j, cell 2a+b       (PAPER.md:L86 pairwPop)
 //   T3[rank3][p][8]        popc(P_a(i) & P_b(j) & P_c(k)), i<j<k, cell 4a+2b+c
@@ -54,6 +55,8 @@ struct DevData {
     const uint32_t* planes[2];   // chunked planes per phenotype
     int32_t nchunks[2];          // 128-sample chunks per phenotype
     int32_t nchunks4[2];         // 256-sample fp4 chunks per phenotype (rows of expl)
+    int32_t nsteps[2];           // tensor-core pipeline steps per phenotype: pairs of fp4 chunks (512 samples)
+    int32_t nrb;                 // 128-row blocks of expl per chunk (= npad / 64)
     int32_t n;                   // SNPs
     int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
     uint32_t np[2];              // n0, n1
@@ -64,6 +67,13 @@ struct DevData {
     const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
     double flt_off;              // fp32 K2 filter: exact-score a quad iff ln2 A + flt_off <= threshold (epilogue.cuh)
 };
+
+// byte offset of (fp4 chunk C, row r = 2 snp + g) in expl: blocked [chunk pair][128-row block][C & 1][row][128 B]
+// so that the 2 chunks x 128 rows of one A tile are one contiguous 32 KiB bulk copy (a 16 KiB copy is processed
+// at ~42 B/clk/SM, a 32 KiB copy at ~75: tools/probe_tma3.cu)
+__host__ __device__ __forceinline__ int64_t expl_off(int64_t C, int64_t r, int32_t nrb) {
+    return ((((C >> 1) * nrb + (r >> 7)) * 2 + (C & 1)) * 128 + (r & 127)) * 128;
+}
 
 // offset (in uint32 words) of (chunk kc, snp, g, word w) in a chunked plane array
 __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, int32_t snp, int g, int w) {

@@ -191,12 +191,12 @@ __global__ void __launch_bounds__(256) k_expand(const uint32_t* __restrict__ pla
         o[k] = v;
     }
     const int sw = cc ^ (int)(r & 7);
-    reinterpret_cast<uint4*>(expl)[rowid * 8 + sw] = make_uint4(o[0], o[1], o[2], o[3]);
+    reinterpret_cast<uint4*>(expl + expl_off(C, r, npad / 64))[sw] = make_uint4(o[0], o[1], o[2], o[3]);
 }
 
 cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,
                           int64_t* launches) {
-    const int64_t nc4 = (nchunks + 1) / 2;
+    const int64_t nc4 = ((nchunks + 1) / 2 + 1) / 2 * 2;   // fp4 chunks, padded to even (zero chunk)
     const int64_t total16 = nc4 * npad * 2 * 8;
     if (total16 > 0) {
         k_expand<<<(unsigned)((total16 + 255) / 256), 256, 0, s>>>(planes, npad, nchunks, total16, expl);

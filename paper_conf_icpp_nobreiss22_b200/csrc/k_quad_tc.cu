@@ -22,18 +22,20 @@
 // CTA pair (cluster of 2): CTA r holds the A rows of w-range 2wp + r (64 SNPs x {AA, Aa}) and builds the
 // B columns of y = y0 + 7r .. y0 + 7r + 6; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
 // receives its 128 rows x all 112 columns and its epilogue scores its 64 x 14 quads.
-// Warp roles (each CTA: 15 warps, 1 CTA per SM, persistent, static tile stride over clusters):
+// Warp roles (each CTA: 16 warps = 4 warpgroups with setmaxnreg budgets, 1 CTA per SM, persistent, static
+// tile stride over clusters):
 //   warps 0..1  : leader — MMA issuers (alternating steps, one elected lane each); follower — warp 0 relays
 //                 "A landed" to the leader's `full` barrier; warp 0 also allocates TMEM (cta_group::2)
-//   warps 2..3  : TMA issuers (alternating steps): the CTA's A, 16 KiB per step, pre-swizzled in HBM
-//   warps 4..6  : producers (every 3rd step each) — the CTA's half of B, x_b & y_c & z_d per 16-byte piece,
-//                 K-major SW128, from singles prefetched with cp.async; then an arrival on the leader's `full`
-//   warps 7..14 : epilogue — tcgen05.ld of the control and case accumulators, lane-pair exchange so one
+//   warps 2..3  : TMA issuers (alternating steps): the CTA's A, one 32 KiB bulk copy per step, pre-swizzled in HBM
+//   warps 4..7  : producers (one chunk of every 2nd step each) — the CTA's half of B, x_b & y_c & z_d per
+//                 16-byte piece, K-major SW128, from singles prefetched with cp.async; then an arrival on the
+//                 leader's `full`
+//   warps 8..15 : epilogue — tcgen05.ld of the control and case accumulators, lane-pair exchange so one
 //                 thread holds one quad's 2 x 16 counts, re-zeroing of the accumulators, the shared epilogue
 //                 (epilogue.cuh); an arrival on the leader's `tempty` barrier
 // Pipelines: STAGES x {A, B half} per CTA (sfull: own TMA landed; full @leader: both B halves built and the
 // follower's A landed; empty: the issuer's MMA commit, multicast to both CTAs); TMEM double buffer
-// 2 x [112 ctrl | 112 case].  One step = one 256-sample fp4 chunk of one phenotype = 4 MMAs.
+// 2 x [112 ctrl | 112 case].  One step = two 256-sample fp4 chunks of one phenotype = 8 MMAs.
 #include <cstdio>
 #include <cstdlib>
 #include <type_traits>
@@ -43,12 +45,15 @@ namespace epi4 {
 
 namespace tc {
 constexpr int M = 256, N = 8 * EPI4_YR_TC;   // UMMA shape (cta_group::2), K = 64 fp4 = 32 bytes per instruction
-constexpr int ROWB = 128;                // bytes of one K-major operand row per stage (256 fp4 samples)
-constexpr int A_BYTES = 128 * ROWB;      // this CTA's 128 A rows
+constexpr int ROWB = 128;                // bytes of one K-major operand row per fp4 chunk (256 samples)
+constexpr int CHUNKS = 2;                // fp4 chunks per pipeline stage (512 samples): one 32 KiB A copy
+constexpr int A_SUB = 128 * ROWB;        // this CTA's 128 A rows of one chunk (16 KiB)
+constexpr int A_BYTES = CHUNKS * A_SUB;
 constexpr int B_ROWS = N / 2;            // this CTA's 56 B columns
-constexpr int B_BYTES = (B_ROWS + 7) / 8 * 1024;
+constexpr int B_SUB = (B_ROWS + 7) / 8 * 1024;
+constexpr int B_BYTES = CHUNKS * B_SUB;
 constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (7)
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 23 KiB, 1024-aligned
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 46 KiB, 1024-aligned
 constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per stage
 // singles (x, z and 8 y rows-pairs of one step) prefetched by each producer warp with cp.async into its ring
 constexpr int SX_OFF = 0, SZ_OFF = 2 * ROWB, SY_OFF = 4 * ROWB;
@@ -62,6 +67,8 @@ constexpr int SGL_SLOTS = PF + 1;
 #define EPI4_PROD_WARPS 4
 #endif
 constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
+static_assert(PROD_WARPS % CHUNKS == 0, "producer warps come in groups of CHUNKS (one chunk of a step each)");
+constexpr int PROD_STRIDE = PROD_WARPS / CHUNKS;          // steps between two steps of one producer warp
 constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate steps (one thread cannot hide
                                          // its own wait/bookkeeping latency behind the blocking MMA issue)
 constexpr int TMA_WARPS = 2;             // a bulk-copy issue blocks its thread ~150-200 cycles: two warps alternate
@@ -83,7 +90,7 @@ constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
 constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 56 / 96
 constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
 constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
-constexpr int STAGE_Q = lcm_c(lcm_c(PROD_WARPS, MMA_WARPS), TMA_WARPS);   // stage counts: multiples
+constexpr int STAGE_Q = lcm_c(lcm_c(PROD_STRIDE, MMA_WARPS), TMA_WARPS);   // stage counts: multiples
 constexpr int TMEM_COLS = 512;
 constexpr int ACC_COLS = 4 * N;          // [buf][p] accumulators: columns buf * 2N + p * N
 constexpr int SF_COL = 480;              // scale factors (all E8M0 0x7F = 1.0): columns 480..511, every lane
@@ -271,8 +278,8 @@ struct StepIt {
         tile = cluster_id_x();
         p = 0;
         kc = 0;
-        nch0 = sp.d.nchunks4[0];
-        nch1 = sp.d.nchunks4[1];
+        nch0 = sp.d.nsteps[0];
+        nch1 = sp.d.nsteps[1];
         if (tile < sp.ntiles) ti = decode_tile(sp, tile);
     }
     __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
@@ -332,7 +339,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     if (tid == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&sfull_bar[s], 1);
-            mbar_init(&full_bar[s], tc::CLUSTER + 1);     // (leader) both CTAs' producers + the follower's A relay
+            mbar_init(&full_bar[s], tc::CLUSTER * tc::CHUNKS + 1);   // (leader) both CTAs' producers + the A relay
             mbar_init(&empty_bar[s], 1);                  // the leader's MMA commit
         }
         for (int b = 0; b < 2; ++b) {
@@ -367,8 +374,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     const long long t_base = clock64();
 #endif
     const int64_t first_tile = cluster_id_x(), tile_stride = nclusters_x();
-    const int64_t chunk_stride = (int64_t)d.npad * 2 * tc::ROWB;  // bytes of one fp4 chunk of expl
-    const int nch0_r = d.nchunks4[0], nch1_r = d.nchunks4[1];
+    const int nch0_r = d.nsteps[0], nch1_r = d.nsteps[1];
+    const int32_t nrb = d.nrb;
     const uint8_t* const expl0 = d.expl[0];
     const uint8_t* const expl1 = d.expl[1];
 
@@ -394,12 +401,14 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             int stage = m;
             uint32_t phase = 0, soff = (uint32_t)m * (tc::STAGE_BYTES >> 4);
             int it = 0, gstep = 0;
-            long long t_wait = 0;
+            long long t_wait = 0, t_tempty = 0;
             const bool do_mma = !(sp.debug & 4);
             for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
                 const int buf = it & 1;
                 const uint32_t tphase = (uint32_t)((it >> 1) & 1);
+                const long long te0 = PCLK();
                 mbar_wait(&tempty_bar[buf], tphase ^ 1u);   // both CTAs' epilogues drained this buffer
+                t_tempty += PCLK() - te0;
                 tc_fence_after();
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
@@ -419,8 +428,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         if (elect_one()) {
                             if (do_mma) {
 #pragma unroll
-                                for (int k = 0; k < tc::ROWB / 32; ++k)
-                                    mma2_mxf4(dcol, adesc0 + soff + 2 * k, bdesc0 + soff + 2 * k, sf_addr);
+                                for (int j = 0; j < tc::CHUNKS; ++j)
+#pragma unroll
+                                    for (int k = 0; k < tc::ROWB / 32; ++k)
+                                        mma2_mxf4(dcol, adesc0 + soff + j * (tc::A_SUB >> 4) + 2 * k,
+                                                  bdesc0 + soff + j * (tc::B_SUB >> 4) + 2 * k, sf_addr);
                             }
                             mma2_commit_mc(&empty_bar[stage]);      // frees the stage in both CTAs
                         }
@@ -434,7 +446,10 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 if (elect_one()) mma2_commit_mc(&tfull_bar[buf]);   // this issuer's MMAs of the tile are done
                 __syncwarp();
             }
-            if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
+            if (EPI4_PROF && lane == 0) {
+                atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
+                atomicAdd(sp.prof + 7, (unsigned long long)t_tempty);
+            }
         } else if (warp == 0) {
             // follower: relay "my A landed" (sfull) to the leader's full barrier, off the producers' path
             int stage = 0;
@@ -468,12 +483,13 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 mbar_wait(&empty_bar[stage], phase ^ 1u);
                 t_wait += PCLK() - t0;
                 if (lane == 0) TRACE(0, gstep);
-                const uint8_t* E = (st.p ? expl1 : expl0) + (int64_t)st.chunk() * chunk_stride;
-                const int64_t wrow = (int64_t)(st.ti.wp * 2 + (int)rank) * EPI4_WR * 2;   // first A row
+                // this CTA's 128 A rows (row block 2 wp + rank) of the step's two chunks: one 32 KiB bulk copy
+                const uint8_t* src = (st.p ? expl1 : expl0) +
+                                     expl_off(2 * (int64_t)st.chunk(), (int64_t)(st.ti.wp * 2 + (int)rank) * 128, nrb);
                 if (elect_one()) {
                     mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                                 ::"r"(ring_s + (uint32_t)(stage * tc::STAGE_BYTES)), "l"(E + wrow * tc::ROWB),
+                                 ::"r"(ring_s + (uint32_t)(stage * tc::STAGE_BYTES)), "l"(src),
                                  "r"((uint32_t)tc::A_BYTES), "r"(smem_u32(&sfull_bar[stage]))
                                  : "memory");
                 }
@@ -486,7 +502,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         }
     } else if (warp < tc::EPI_WARP0) {
         // ===================== producers =====================
-        // Producer warp j builds this CTA's B half of every step s with s % PROD_WARPS == j.  Its singles
+        // Producer warp j builds chunk j % CHUNKS of this CTA's B half of every step s with
+        // s % PROD_STRIDE == j / CHUNKS.  Its singles
         // (x, z and 8 y SNPs of which the CTA's 7 are used: 20 rows of 128 B, pre-swizzled in HBM) are
         // prefetched PF own steps ahead with cp.async into the warp's private ring.  Lane: 16-byte piece
         // cc = lane & 7 of the 256-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k
@@ -494,6 +511,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         // E2M1 {0, 1.0} values is their product).  The follower's A is certified to the leader by the relay
         // warp, so producers never wait for the TMA.
         const int pw = warp - tc::PROD_WARP0;
+        const int jc = pw % tc::CHUNKS, pstep0 = pw / tc::CHUNKS;   // chunk of the step, first step
         const int cc = lane & 7, cpl = (lane >> 3) & 1, yq = lane >> 4;
         const bool build = !(sp.debug & 1);
         unsigned char* my_sgl = sgl_ring + pw * tc::SGL_SLOTS * tc::SGL_BYTES;
@@ -504,36 +522,36 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             const int n7 = (bd >> 1) * 4 + cpl * 2 + (bd & 1);
             boff[bd] = (uint32_t)(yq * 1024 + n7 * 128 + ((cc ^ n7) << 4));
         }
-        // this lane's 5 pieces of a singles slot: piece 0 = x|z row piece, pieces 1..4 = y rows
-        const int pxz = lane < 16 ? lane * 16 : (lane - 16) * 16;     // byte offset inside the x or z rows
         long long t_wait = 0, t_busy = 0, t_arr = 0;
         StepIt st, pre;
         st.init(sp);
-        st.advance(sp, pw);
+        st.advance(sp, pstep0);
         pre = st;
         auto prefetch = [&](int slot, const StepIt& it) {
             if (it.valid(sp)) {
-                const uint8_t* E = (it.p ? expl1 : expl0) + (int64_t)it.chunk() * chunk_stride;
+                const uint8_t* E = it.p ? expl1 : expl0;
+                const int64_t C = 2 * (int64_t)it.chunk() + jc;
                 unsigned char* dst = my_sgl + slot * tc::SGL_BYTES;
-                const uint8_t* srcxz = E + (int64_t)(lane < 16 ? it.ti.x : it.ti.z) * 2 * tc::ROWB + pxz;
-                cp_async16(dst + lane * 16, srcxz);
-                const uint8_t* srcy = E + (int64_t)(it.ti.y0 + tc::YH * (int)rank) * 2 * tc::ROWB + lane * 16;
+                const int64_t rxz = 2 * (int64_t)(lane < 16 ? it.ti.x : it.ti.z) + ((lane >> 3) & 1);
+                cp_async16(dst + lane * 16, E + expl_off(C, rxz, nrb) + (lane & 7) * 16);
+                const int64_t ry = 2 * (int64_t)(it.ti.y0 + tc::YH * (int)rank) + (lane >> 3);
 #pragma unroll
-                for (int k = 0; k < 4; ++k) cp_async16(dst + tc::SY_OFF + k * 512 + lane * 16, srcy + k * 512);
+                for (int k = 0; k < 4; ++k)
+                    cp_async16(dst + tc::SY_OFF + k * 512 + lane * 16, E + expl_off(C, ry + 4 * k, nrb) + (lane & 7) * 16);
             }
             cp_async_commit();                                    // (an empty group past the end)
         };
 #pragma unroll 1
         for (int k = 0; k < tc::PF; ++k) {
             prefetch(k, pre);
-            pre.advance(sp, tc::PROD_WARPS);
+            pre.advance(sp, tc::PROD_STRIDE);
         }
-        int slot = 0, stage = pw;
+        int slot = 0, stage = pstep0;
         uint32_t phase = 0;
-        for (int step = pw; st.valid(sp); step += tc::PROD_WARPS) {
+        for (int step = pstep0; st.valid(sp); step += tc::PROD_STRIDE) {
             if (lane == 0) TRACE(2, step);
             prefetch(slot == 0 ? tc::PF : slot - 1, pre);         // slot (slot + PF) % (PF + 1)
-            pre.advance(sp, tc::PROD_WARPS);
+            pre.advance(sp, tc::PROD_STRIDE);
             cp_async_wait<tc::PF>();                              // this step's singles landed (own lane)
             __syncwarp();                                         // ... and every lane's
             if (lane == 0) TRACE(3, step);
@@ -544,7 +562,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             if (lane == 0) TRACE(4, step);
             if (build) {
                 const unsigned char* sg = my_sgl + slot * tc::SGL_BYTES;
-                unsigned char* sb = ring + stage * tc::STAGE_BYTES + tc::A_BYTES;
+                unsigned char* sb = ring + stage * tc::STAGE_BYTES + tc::A_BYTES + jc * tc::B_SUB;
                 const int x = st.ti.x, zc = st.ti.z, y0h = st.ti.y0 + tc::YH * (int)rank;
                 // singles keep the HBM swizzle: piece cc of absolute row r sits at piece cc ^ (r & 7)
                 const uint4 x0 = *reinterpret_cast<const uint4*>(sg + tc::SX_OFF + ((cc ^ ((2 * x) & 7)) << 4));
@@ -583,16 +601,16 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 t_busy += t3 - t1;
                 t_arr += t3 - t2;
             }
-            st.advance(sp, tc::PROD_WARPS);
+            st.advance(sp, tc::PROD_STRIDE);
             if (++slot == tc::SGL_SLOTS) slot = 0;
-            stage += tc::PROD_WARPS;
+            stage += tc::PROD_STRIDE;
             if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; }
         }
         cp_async_wait<0>();
         if (EPI4_PROF && lane == 0) {
             atomicAdd(sp.prof + 3, (unsigned long long)t_busy);
             atomicAdd(sp.prof + 4, (unsigned long long)t_wait);
-            atomicAdd(sp.prof + 7, (unsigned long long)t_arr);
+            (void)t_arr;
         }
     } else {
         // ===================== epilogue =====================
