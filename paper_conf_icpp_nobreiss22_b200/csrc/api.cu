@@ -127,6 +127,8 @@ DevData devdata(const epi4_ctx* c) {
     d.nsteps[0] = (d.nchunks4[0] + 1) / 2;
     d.nsteps[1] = (d.nchunks4[1] + 1) / 2;
     d.nrb = c->npad / 64;
+    d.pk_shift = 1;
+    while (d.pk_shift < 31 && ((int64_t)1 << d.pk_shift) <= c->np[0]) ++d.pk_shift;   // c0 <= n0 < 2^pk_shift
     d.n = c->n;
     d.npad = c->npad;
     d.np[0] = (uint32_t)c->np[0];
@@ -501,6 +503,15 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!quads_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
+    if (c->opts.pipe == EPI4_PIPE_TC) {
+        // the tensor-core epilogue packs (c0, c1) into 32 bits and the fp32 filter needs counts < 2^22
+        const DevData dd = devdata(c);
+        if (c->np[0] >= ((int64_t)1 << 22) || c->np[1] >= ((int64_t)1 << 22) ||
+            c->np[1] >= ((int64_t)1 << (32 - dd.pk_shift)))
+            return fail(EPI4_EINVAL, "n0=%lld / n1=%lld: the tensor-core pipe needs both counts to fit one 32-bit word "
+                        "(bits(n0) + bits(n1) <= 32) and each < 2^22; use pipe lop3", (long long)c->np[0],
+                        (long long)c->np[1]);
+    }
     CU(cudaSetDevice(c->device));
     std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
     const int64_t nall = (int64_t)plan.size();

@@ -24,7 +24,7 @@
 #define EPI4_WR 64            // w-range of one CTA / rows of its A operand: 64 SNPs x {AA, Aa}
 #define EPI4_WP 128           // w-range of a work unit (a CTA pair: two 64-SNP halves)
 #define EPI4_YR 16            // y-range of a CUDA-core (LOP3) tile: 16 consecutive SNPs after x
-#define EPI4_YR_TC 14         // y-range of a tensor-core tile (N = 112 = 14 x 8 columns; TMEM budget, k_quad_tc.cu)
+#define EPI4_YR_TC 20         // y-range of a tensor-core tile (N = 160 = 20 x 8 columns; TMEM budget, k_quad_tc.cu)
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
 
@@ -57,6 +57,7 @@ struct DevData {
     int32_t nchunks4[2];         // 256-sample fp4 chunks per phenotype (rows of expl)
     int32_t nsteps[2];           // tensor-core pipeline steps per phenotype: pairs of fp4 chunks (512 samples)
     int32_t nrb;                 // 128-row blocks of expl per chunk (= npad / 64)
+    int32_t pk_shift;            // tensor-core epilogue: (control, case) counts packed as c0 | c1 << pk_shift
     int32_t n;                   // SNPs
     int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
     uint32_t np[2];              // n0, n1

@@ -3,10 +3,10 @@
 // epilogue.
 //
 // What it computes: for a tile (w-range pair wp, x, y-range y0, z) and each
-// phenotype p the 256 x 112 matrix
+// phenotype p the 256 x 160 matrix
 //     C_p[(w, a)][(y, b, c, d)] = sum over samples s of phenotype p of P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]
-// for the 128 SNPs w of the range pair and the 14 SNPs y = y0..y0+13: the 16 non-aa genotype counts of the
-// 128 x 14 quads (w, x, y, z) ("a matrix with 16 values per each quad").
+// for the 128 SNPs w of the range pair and the 20 SNPs y = y0..y0+19: the 16 non-aa genotype counts of the
+// 128 x 20 quads (w, x, y, z) ("a matrix with 16 values per each quad").
 // Factorisation: the paper ANDs SNP pairs into both operands (combine);
 // here the A operand is the raw single-SNP planes (w, a), copied from HBM by the TMA engine, and x is folded
 // into the B operand, whose columns are triple products P_b(x) & P_c(y) & P_d(z) built on chip.
@@ -14,28 +14,36 @@
 // legacy IMMA).  A set bit is the E2M1 value 1.0 (nibble 0x2), so AND of packed nibbles
 // is the product, and with all E8M0 block scales = 1 the MMA sums exact small integers: the fp32 accumulator
 // is exact up to 2^24 per phenotype (host check; tools/probe_mxf4.cu: 0 mismatches, counts to 76800).
-// kind::mxf4 runs M=256 N=128 K=64 in 64 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the
+// kind::mxf4 runs M=256 N=160 K=64 in 80 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the
 // operand bytes (2 samples per byte).
 // Why 2-CTA: a 1-CTA M=128 MMA issues every ~97 cycles whatever N; cta_group::2 reaches the full rate.
-// Why N = 112: TMEM holds 2 buffers x 2 phenotypes x 112 fp32 columns (448) plus the scale factors.
+// Why N = 160: the A operand is streamed from L2 once per (tile, sample chunk), i.e. 128 B per row and 256
+// samples for every N columns; at N = 112 a full-rate MMA needs 73 B/clk/SM of A, the whole TMA ingest an SM
+// gets from L2 (tools/probe_tma3.cu: ~75 B/clk/SM with 32 KiB copies); N = 160 needs 51.  TMEM holds three
+// regions of 160 fp32 columns plus the scale factors; tile t accumulates its controls in region (-t) mod 3 and
+// its cases in the next one.  When the tile is done the epilogue first packs every (control, case) pair into
+// one 32-bit word in the case region and zeroes the control region (pass 1, a few hundred cycles), which the
+// case accumulation of tile t+1 reuses; it then scores the quads from the packed region (pass 2), which the
+// control accumulation of tile t+2 reuses.  Two buffers of 2 x 160 columns would not fit in 512.
 //
 // CTA pair (cluster of 2): CTA r holds the A rows of w-range 2wp + r (64 SNPs x {AA, Aa}) and builds the
-// B columns of y = y0 + 7r .. y0 + 7r + 6; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
-// receives its 128 rows x all 112 columns and its epilogue scores its 64 x 14 quads.
+// B columns of y = y0 + 10r .. y0 + 10r + 9; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
+// receives its 128 rows x all 160 columns and its epilogue scores its 64 x 20 quads.
 // Warp roles (each CTA: 16 warps = 4 warpgroups with setmaxnreg budgets, 1 CTA per SM, persistent, static
 // tile stride over clusters):
 //   warps 0..1  : leader — MMA issuers (alternating steps, one elected lane each); follower — warp 0 relays
 //                 "A landed" to the leader's `full` barrier; warp 0 also allocates TMEM (cta_group::2)
 //   warps 2..3  : TMA issuers (alternating steps): the CTA's A, one 32 KiB bulk copy per step, pre-swizzled in HBM
 //   warps 4..7  : producers (one chunk of every 2nd step each) — the CTA's half of B, x_b & y_c & z_d per
-//                 16-byte piece, K-major SW128, from singles prefetched with cp.async; then an arrival on the
-//                 leader's `full`
-//   warps 8..15 : epilogue — tcgen05.ld of the control and case accumulators, lane-pair exchange so one
-//                 thread holds one quad's 2 x 16 counts, re-zeroing of the accumulators, the shared epilogue
-//                 (epilogue.cuh); an arrival on the leader's `tempty` barrier
+//                 16-byte piece, K-major SW128, from singles loaded into registers one step ahead; then an
+//                 arrival on the leader's `full`
+//   warps 8..15 : epilogue — pass 1 (pack, arrive `pk`), pass 2: tcgen05.ld of the packed counts, lane-pair
+//                 exchange so one thread holds one quad's 2 x 16 counts, re-zeroing, the shared per-quad
+//                 evaluation (epilogue.cuh); an arrival on the leader's `ep` barrier
 // Pipelines: STAGES x {A, B half} per CTA (sfull: own TMA landed; full @leader: both B halves built and the
-// follower's A landed; empty: the issuer's MMA commit, multicast to both CTAs); TMEM double buffer
-// 2 x [112 ctrl | 112 case].  One step = two 256-sample fp4 chunks of one phenotype = 8 MMAs.
+// follower's A landed; empty: the issuer's MMA commit, multicast to both CTAs); TMEM: the region rotation
+// above (tfull -> epilogue; pk, ep -> MMA issuers).  One step = two 256-sample fp4 chunks of one phenotype =
+// 8 MMAs.
 #include <cstdio>
 #include <cstdlib>
 #include <type_traits>
@@ -49,20 +57,12 @@ constexpr int ROWB = 128;                // bytes of one K-major operand row per
 constexpr int CHUNKS = 2;                // fp4 chunks per pipeline stage (512 samples): one 32 KiB A copy
 constexpr int A_SUB = 128 * ROWB;        // this CTA's 128 A rows of one chunk (16 KiB)
 constexpr int A_BYTES = CHUNKS * A_SUB;
-constexpr int B_ROWS = N / 2;            // this CTA's 56 B columns
+constexpr int B_ROWS = N / 2;            // this CTA's 80 B columns
 constexpr int B_SUB = (B_ROWS + 7) / 8 * 1024;
 constexpr int B_BYTES = CHUNKS * B_SUB;
-constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (7)
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 46 KiB, 1024-aligned
+constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (10)
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 52 KiB, 1024-aligned
 constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per stage
-// singles (x, z and 8 y rows-pairs of one step) prefetched by each producer warp with cp.async into its ring
-constexpr int SX_OFF = 0, SZ_OFF = 2 * ROWB, SY_OFF = 4 * ROWB;
-constexpr int SGL_BYTES = (4 + 16) * ROWB;                 // 20 rows x 128 B
-#ifndef EPI4_PF
-#define EPI4_PF 1
-#endif
-constexpr int PF = EPI4_PF;                                // prefetch distance (own steps)
-constexpr int SGL_SLOTS = PF + 1;
 #ifndef EPI4_PROD_WARPS
 #define EPI4_PROD_WARPS 4
 #endif
@@ -84,7 +84,7 @@ constexpr bool REGSPLIT = EPI4_REGSPLIT && PROD_WARPS == 4 && MMA_WARPS + TMA_WA
 #define EPI4_REGS_CTL 56
 #endif
 #ifndef EPI4_REGS_PROD
-#define EPI4_REGS_PROD 96
+#define EPI4_REGS_PROD 104
 #endif
 constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
 constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 56 / 96
@@ -92,7 +92,8 @@ constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
 constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
 constexpr int STAGE_Q = lcm_c(lcm_c(PROD_STRIDE, MMA_WARPS), TMA_WARPS);   // stage counts: multiples
 constexpr int TMEM_COLS = 512;
-constexpr int ACC_COLS = 4 * N;          // [buf][p] accumulators: columns buf * 2N + p * N
+constexpr int REGIONS = 3;               // accumulator regions of N columns, rotated per tile (header comment)
+constexpr int ACC_COLS = REGIONS * N;
 constexpr int SF_COL = 480;              // scale factors (all E8M0 0x7F = 1.0): columns 480..511, every lane
 static_assert(ACC_COLS <= SF_COL, "TMEM: accumulators overlap the scale factors");
 constexpr int NG = N / 16;               // 16-column groups of an accumulator (7)
@@ -218,6 +219,13 @@ __device__ __forceinline__ void tmem_fill16(uint32_t taddr, uint32_t v) {
         : "memory");
 }
 __device__ __forceinline__ void tmem_zero16(uint32_t taddr) { tmem_fill16(taddr, 0u); }
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+        "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+        : "memory");
+}
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // byte offset of (row r, 16-byte chunk c) inside a K-major SW128 tile of 128-byte rows
@@ -323,14 +331,13 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     static_assert(STAGES % tc::STAGE_Q == 0, "a producer's / issuer's successive uses of a stage must be one phase apart");
     extern __shared__ unsigned char smem_raw[];
     __shared__ __align__(8) uint64_t sfull_bar[STAGES], full_bar[STAGES], empty_bar[STAGES];
-    __shared__ __align__(8) uint64_t tfull_bar[2], tempty_bar[2];
+    __shared__ __align__(8) uint64_t tfull_bar[2], pk_bar, ep_bar[2];
     __shared__ uint32_t s_tmem;
-    // 1024-aligned stage ring, the producers' singles rings, the top-k state
+    // 1024-aligned stage ring, then the top-k state
     // (same offsets in both CTAs of the pair: the MMA addresses the peer's operands at the same offsets)
     const uint32_t raw = smem_u32(smem_raw);
     unsigned char* ring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-    unsigned char* sgl_ring = ring + STAGES * tc::STAGE_BYTES;   // [PROD_WARPS][SGL_SLOTS][SGL_BYTES]
-    TopKSmem tk = topk_carve(sgl_ring + tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES, sp.topk);
+    TopKSmem tk = topk_carve(ring + STAGES * tc::STAGE_BYTES, sp.topk);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const DevData& d = sp.d;
@@ -344,8 +351,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&tfull_bar[b], tc::MMA_WARPS);      // each issuer's commit after its last step
-            mbar_init(&tempty_bar[b], tc::CLUSTER * tc::EPI_WARPS);   // (leader) every epilogue warp of the pair
+            mbar_init(&ep_bar[b], tc::CLUSTER * tc::EPI_WARPS);   // (leader) every epilogue warp of the pair
         }
+        mbar_init(&pk_bar, tc::CLUSTER * tc::EPI_WARPS);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 0) {
@@ -403,16 +411,23 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             int it = 0, gstep = 0;
             long long t_wait = 0, t_tempty = 0;
             const bool do_mma = !(sp.debug & 4);
+            int r0 = 0;                                   // p0 region of this tile: (-it) mod 3; p1: r0 + 1 mod 3
             for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
                 const int buf = it & 1;
-                const uint32_t tphase = (uint32_t)((it >> 1) & 1);
                 const long long te0 = PCLK();
-                mbar_wait(&tempty_bar[buf], tphase ^ 1u);   // both CTAs' epilogues drained this buffer
+                // the p0 region held the packed counts of tile it - 2: both CTAs' epilogues are done with them
+                if (it >= 2) mbar_wait(&ep_bar[buf], (uint32_t)(((it >> 1) & 1) ^ 1));
                 t_tempty += PCLK() - te0;
                 tc_fence_after();
+                const int r1 = r0 == 2 ? 0 : r0 + 1;
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
-                    const uint32_t dcol = tmem + (uint32_t)(buf * 2 * tc::N + p * tc::N);
+                    if (p == 1 && it >= 1) {
+                        // the p1 region held the controls of tile it - 1: its pack pass moved them out
+                        mbar_wait(&pk_bar, (uint32_t)((it - 1) & 1));
+                        tc_fence_after();
+                    }
+                    const uint32_t dcol = tmem + (uint32_t)((p ? r1 : r0) * tc::N);
                     const int nch = p ? nch1_r : nch0_r;
 #pragma unroll 1
                     for (int kc = 0; kc < nch; ++kc, ++gstep) {
@@ -445,6 +460,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 }
                 if (elect_one()) mma2_commit_mc(&tfull_bar[buf]);   // this issuer's MMAs of the tile are done
                 __syncwarp();
+                r0 = r0 == 0 ? 2 : r0 - 1;
             }
             if (EPI4_PROF && lane == 0) {
                 atomicAdd(sp.prof + 5, (unsigned long long)t_wait);
@@ -502,20 +518,20 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         }
     } else if (warp < tc::EPI_WARP0) {
         // ===================== producers =====================
-        // Producer warp j builds chunk j % CHUNKS of this CTA's B half of every step s with
-        // s % PROD_STRIDE == j / CHUNKS.  Its singles
-        // (x, z and 8 y SNPs of which the CTA's 7 are used: 20 rows of 128 B, pre-swizzled in HBM) are
-        // prefetched PF own steps ahead with cp.async into the warp's private ring.  Lane: 16-byte piece
-        // cc = lane & 7 of the 256-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k
-        // (k = 0..3, y_local < 7); B[n = 8 y_local + 4b + 2c + d] = x_b & y_c & z_d (a nibble-wise AND of
-        // E2M1 {0, 1.0} values is their product).  The follower's A is certified to the leader by the relay
-        // warp, so producers never wait for the TMA.
+        // Producer warp j builds chunk jc = j % CHUNKS of this CTA's B half of every step s with
+        // s % PROD_STRIDE == j / CHUNKS.  Its singles (x, z and the CTA's YH y SNPs, two planes each, pre-swizzled
+        // in HBM) are loaded straight into registers one own step ahead (no shared-memory staging).  Lane:
+        // 16-byte piece cc = lane & 7 of the 256-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k
+        // (k = 0..YH/2-1); B[n = 8 y_local + 4b + 2c + d] = x_b & y_c & z_d (a nibble-wise AND of E2M1 {0, 1.0}
+        // values is their product).  The follower's A is certified to the leader by the relay warp, so producers
+        // never wait for the TMA.
+        static_assert(tc::YH % 2 == 0, "two y per lane pair");
+        constexpr int YK = tc::YH / 2;
         const int pw = warp - tc::PROD_WARP0;
         const int jc = pw % tc::CHUNKS, pstep0 = pw / tc::CHUNKS;   // chunk of the step, first step
         const int cc = lane & 7, cpl = (lane >> 3) & 1, yq = lane >> 4;
         const bool build = !(sp.debug & 1);
-        unsigned char* my_sgl = sgl_ring + pw * tc::SGL_SLOTS * tc::SGL_BYTES;
-        // store offsets inside the B half for bd = 2b + d (y_local = yq; + 2048 per k)
+        // store offsets inside the B sub-tile for bd = 2b + d (y_local = yq; + 2048 per k)
         uint32_t boff[4];
 #pragma unroll
         for (int bd = 0; bd < 4; ++bd) {
@@ -527,63 +543,50 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         st.init(sp);
         st.advance(sp, pstep0);
         pre = st;
-        auto prefetch = [&](int slot, const StepIt& it) {
-            if (it.valid(sp)) {
+        // logical piece cc of absolute row r sits at piece cc ^ (r & 7) of the row in HBM
+        auto ld_piece = [&](const uint8_t* E, int64_t C, int64_t r) -> uint4 {
+            return __ldg(reinterpret_cast<const uint4*>(E + expl_off(C, r, nrb) + ((cc ^ (int)(r & 7)) << 4)));
+        };
+        uint4 nx[4], ny[YK];
+        auto load = [&](const StepIt& it) {
+            if (it.valid(sp) && build) {
                 const uint8_t* E = it.p ? expl1 : expl0;
                 const int64_t C = 2 * (int64_t)it.chunk() + jc;
-                unsigned char* dst = my_sgl + slot * tc::SGL_BYTES;
-                const int64_t rxz = 2 * (int64_t)(lane < 16 ? it.ti.x : it.ti.z) + ((lane >> 3) & 1);
-                cp_async16(dst + lane * 16, E + expl_off(C, rxz, nrb) + (lane & 7) * 16);
-                const int64_t ry = 2 * (int64_t)(it.ti.y0 + tc::YH * (int)rank) + (lane >> 3);
+                nx[0] = ld_piece(E, C, 2 * (int64_t)it.ti.x);
+                nx[1] = ld_piece(E, C, 2 * (int64_t)it.ti.x + 1);
+                nx[2] = ld_piece(E, C, 2 * (int64_t)it.ti.z);
+                nx[3] = ld_piece(E, C, 2 * (int64_t)it.ti.z + 1);
+                const int64_t ry = 2 * (int64_t)(it.ti.y0 + tc::YH * (int)rank + yq) + cpl;
 #pragma unroll
-                for (int k = 0; k < 4; ++k)
-                    cp_async16(dst + tc::SY_OFF + k * 512 + lane * 16, E + expl_off(C, ry + 4 * k, nrb) + (lane & 7) * 16);
+                for (int k = 0; k < YK; ++k) ny[k] = ld_piece(E, C, ry + 4 * k);
             }
-            cp_async_commit();                                    // (an empty group past the end)
         };
-#pragma unroll 1
-        for (int k = 0; k < tc::PF; ++k) {
-            prefetch(k, pre);
-            pre.advance(sp, tc::PROD_STRIDE);
-        }
-        int slot = 0, stage = pstep0;
+        load(pre);
+        pre.advance(sp, tc::PROD_STRIDE);
+        int stage = pstep0;
         uint32_t phase = 0;
         for (int step = pstep0; st.valid(sp); step += tc::PROD_STRIDE) {
             if (lane == 0) TRACE(2, step);
-            prefetch(slot == 0 ? tc::PF : slot - 1, pre);         // slot (slot + PF) % (PF + 1)
+            uint4 cx[4], cy[YK];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) cx[k] = nx[k];
+#pragma unroll
+            for (int k = 0; k < YK; ++k) cy[k] = ny[k];
+            load(pre);                                            // next own step's singles (in flight)
             pre.advance(sp, tc::PROD_STRIDE);
-            cp_async_wait<tc::PF>();                              // this step's singles landed (own lane)
-            __syncwarp();                                         // ... and every lane's
-            if (lane == 0) TRACE(3, step);
             const long long t0 = PCLK();
             mbar_wait(&empty_bar[stage], phase ^ 1u);             // B slot free (MMA of step - STAGES done)
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             if (lane == 0) TRACE(4, step);
             if (build) {
-                const unsigned char* sg = my_sgl + slot * tc::SGL_BYTES;
                 unsigned char* sb = ring + stage * tc::STAGE_BYTES + tc::A_BYTES + jc * tc::B_SUB;
-                const int x = st.ti.x, zc = st.ti.z, y0h = st.ti.y0 + tc::YH * (int)rank;
-                // singles keep the HBM swizzle: piece cc of absolute row r sits at piece cc ^ (r & 7)
-                const uint4 x0 = *reinterpret_cast<const uint4*>(sg + tc::SX_OFF + ((cc ^ ((2 * x) & 7)) << 4));
-                const uint4 x1 = *reinterpret_cast<const uint4*>(sg + tc::SX_OFF + 128 + ((cc ^ ((2 * x + 1) & 7)) << 4));
-                const uint4 z0 = *reinterpret_cast<const uint4*>(sg + tc::SZ_OFF + ((cc ^ ((2 * zc) & 7)) << 4));
-                const uint4 z1 = *reinterpret_cast<const uint4*>(sg + tc::SZ_OFF + 128 + ((cc ^ ((2 * zc + 1) & 7)) << 4));
-                const unsigned char* ybase = sg + tc::SY_OFF + (2 * yq + cpl) * 128;
-                const int ra0 = 2 * y0h + 2 * yq + cpl;                        // absolute row of k = 0
-                const uint32_t yo0 = (uint32_t)((cc ^ (ra0 & 7)) << 4), yo1 = (uint32_t)((cc ^ ((ra0 + 4) & 7)) << 4);
-                uint4 yv[4];
+                const uint4 xz[4] = {and4(cx[0], cx[2]), and4(cx[0], cx[3]), and4(cx[1], cx[2]), and4(cx[1], cx[3])};
 #pragma unroll
-                for (int k = 0; k < 4; ++k)
-                    yv[k] = *reinterpret_cast<const uint4*>(ybase + k * 512 + ((k & 1) ? yo1 : yo0));
-                if (lane == 0) TRACE(5, step);
-                const uint4 xz[4] = {and4(x0, z0), and4(x0, z1), and4(x1, z0), and4(x1, z1)};   // [b*2 + d]
+                for (int k = 0; k < YK; ++k)
 #pragma unroll
-                for (int k = 0; k < 4; ++k)
-                    if (k < 3 || yq == 0)                 // y_local = 7 is the other CTA's
-#pragma unroll
-                        for (int bd = 0; bd < 4; ++bd)
-                            *reinterpret_cast<uint4*>(sb + boff[bd] + k * 2048) = and4(yv[k], xz[bd]);
+                    for (int bd = 0; bd < 4; ++bd)
+                        *reinterpret_cast<uint4*>(sb + boff[bd] + k * 2048) = and4(cy[k], xz[bd]);
                 if (lane == 0) TRACE(6, step);
                 fence_proxy_async();                      // generic-proxy stores -> visible to the tensor core
             }
@@ -602,11 +605,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 t_arr += t3 - t2;
             }
             st.advance(sp, tc::PROD_STRIDE);
-            if (++slot == tc::SGL_SLOTS) slot = 0;
             stage += tc::PROD_STRIDE;
             if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; }
         }
-        cp_async_wait<0>();
         if (EPI4_PROF && lane == 0) {
             atomicAdd(sp.prof + 3, (unsigned long long)t_busy);
             atomicAdd(sp.prof + 4, (unsigned long long)t_wait);
@@ -626,52 +627,71 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         long long t_wait = 0, t_busy = 0;
         const bool score = !(sp.debug & 2);
         int it = 0;
+        const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
+        int r0 = 0;                                     // the MMA issuers' region rotation
         for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
             const TileInfo ti = decode_tile(sp, tile);
             const int buf = it & 1;
             const uint32_t tphase = (uint32_t)((it >> 1) & 1);
+            const int r1 = r0 == 2 ? 0 : r0 + 1;
             const long long t0 = PCLK();
             mbar_wait_sleep(&tfull_bar[buf], tphase);
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             tc_fence_after();
             const int w = (ti.wp * 2 + (int)rank) * EPI4_WR + wl;
-            const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * 2 * tc::N);
+            const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
+            const uint32_t R0 = tq + (uint32_t)(r0 * tc::N), R1 = tq + (uint32_t)(r1 * tc::N);
+            // pass 1: pack each (control, case) count pair into one 32-bit word, in place in the case region,
+            // and zero the control region, which the next tile's case accumulation reuses
 #pragma unroll 1
             for (int g = h; g < tc::NG; g += 2) {
                 uint32_t v0[16], v1[16];
-                tmem_ld16(tbase + 16 * g, v0);
-                tmem_ld16(tbase + tc::N + 16 * g, v1);
+                tmem_ld16(R0 + 16 * g, v0);
+                tmem_ld16(R1 + 16 * g, v1);
                 tmem_wait_ld();
-                tmem_zero16(tbase + 16 * g);              // ready for the next tile's accumulation
-                tmem_zero16(tbase + tc::N + 16 * g);
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {            // fp32 accumulators hold exact integers < 2^23:
-                    // adding 2^23 puts the integer in the mantissa bits (FADD + LOP instead of F2I)
-                    v0[k] = __float_as_uint(__uint_as_float(v0[k]) + 8388608.0f) & 0x7FFFFFu;
-                    v1[k] = __float_as_uint(__uint_as_float(v1[k]) + 8388608.0f) & 0x7FFFFFu;
-                }
+                for (int k = 0; k < 16; ++k)              // fp32 accumulators hold exact integers < 2^23: adding
+                    v1[k] = (__float_as_uint(__uint_as_float(v0[k]) + 8388608.0f) & 0x7FFFFFu) |   // 2^23 puts
+                            ((__float_as_uint(__uint_as_float(v1[k]) + 8388608.0f) & 0x7FFFFFu) << pks);  // them in
+                tmem_st16(R1 + 16 * g, v1);                                              // the mantissa
+                tmem_zero16(R0 + 16 * g);
+            }
+            tmem_wait_st();
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+                if (leader) mbar_arrive_local(&pk_bar);
+                else mbar_arrive_cluster(&pk_bar, 0);   // the leader's barrier
+            }
+            // pass 2: score the quads from the packed counts
+#pragma unroll 1
+            for (int g = h; g < tc::NG; g += 2) {
+                uint32_t v[16];
+                tmem_ld16(R1 + 16 * g, v);
+                tmem_wait_ld();
+                tmem_zero16(R1 + 16 * g);                 // ready for a later tile's accumulation
                 if (g + 2 >= tc::NG) {
                     tmem_wait_st();
                     tc_fence_before();
                     __syncwarp();
                     if (lane == 0) {
-                        if (leader) mbar_arrive_local(&tempty_bar[buf]);
-                        else mbar_arrive_cluster(&tempty_bar[buf], 0);   // the leader's barrier
+                        if (leader) mbar_arrive_local(&ep_bar[buf]);
+                        else mbar_arrive_cluster(&ep_bar[buf], 0);   // the leader's barrier
                     }
                 }
                 uint32_t c0[16], c1[16];
 #pragma unroll
                 for (int k = 0; k < 8; ++k) {
                     // send my values for the other lane's quad, keep mine
-                    const uint32_t s0 = a ? v0[k] : v0[8 + k], s1 = a ? v1[k] : v1[8 + k];
-                    const uint32_t r0 = __shfl_xor_sync(0xffffffffu, s0, 1);
-                    const uint32_t r1 = __shfl_xor_sync(0xffffffffu, s1, 1);
+                    const uint32_t sv = a ? v[k] : v[8 + k];
+                    const uint32_t rv = __shfl_xor_sync(0xffffffffu, sv, 1);
                     // lane a keeps c16[8a + k] = its own v[8a + k] and takes c16[8(1-a) + k] from the partner
-                    c0[k] = a ? r0 : v0[k];
-                    c0[8 + k] = a ? v0[8 + k] : r0;
-                    c1[k] = a ? r1 : v1[k];
-                    c1[8 + k] = a ? v1[8 + k] : r1;
+                    const uint32_t lo = a ? rv : v[k], hi = a ? v[8 + k] : rv;
+                    c0[k] = lo & pkm;
+                    c1[k] = lo >> pks;
+                    c0[8 + k] = hi & pkm;
+                    c1[8 + k] = hi >> pks;
                 }
                 const int y = ti.y0 + 2 * g + a;
                 const bool valid = (w < ti.x) && (y < ti.z) && score;
@@ -713,6 +733,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 warp_offer(tk, offer, key, idx);
             }
             t_busy += PCLK() - t1;
+            r0 = r0 == 0 ? 2 : r0 - 1;
         }
         unsigned long long v = my_quads, ne = n_exact;
 #pragma unroll
@@ -777,16 +798,14 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     int dev = 0, optin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024 +   // alignment + static smem slack
-                         (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES;
+    const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024;   // alignment + static smem slack
     // most pipeline stages that fit (a multiple of STAGE_Q: each producer / issuer / TMA warp takes every
-    // PROD_WARPS-th / MMA_WARPS-th / TMA_WARPS-th step and must meet its stages one phase apart)
+    // PROD_STRIDE-th / MMA_WARPS-th / TMA_WARPS-th step and must meet its stages one phase apart)
     int st = 0;
     for (int cand = tc::MAX_STAGES / tc::STAGE_Q * tc::STAGE_Q; cand >= tc::STAGE_Q && !st; cand -= tc::STAGE_Q)
         if (fixed + (size_t)cand * tc::STAGE_BYTES <= (size_t)optin) st = cand;
     if (!st) return cudaErrorInvalidConfiguration;
-    const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + (size_t)tc::PROD_WARPS * tc::SGL_SLOTS * tc::SGL_BYTES +
-                        topk_smem_bytes(sp.topk);
+    const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + topk_smem_bytes(sp.topk);
     if (getenv("EPI4_VERBOSE"))
         fprintf(stderr, "k_quad_tc: %d producer warps, %d stages, filter %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
                 sp.use_filter, smem, grid);
