@@ -280,3 +280,26 @@ def test_full_C2_units_sample_and_planted(pipe):
     assert epi.unpack_index(idx[0]) == datagen.planted_quad_for(n)
     qs = np.array([epi.unpack_index(v) for v in idx], dtype=np.int32)
     np.testing.assert_array_equal(k2, oracle.score(d.geno, d.phen, qs))
+
+
+@pytest.mark.parametrize("cfg", ["C5", "C2"])
+def test_fp32_filter_keeps_exact_topk(cfg):
+    """The tensor-core epilogue scores a quad exactly only when its fp32 Stirling lower bound can beat the
+    CTA's k-th best K2 (epilogue.cuh, reading #16).  With a large k (a loose threshold for most
+    of the run) and the largest M (C5, the widest rounding bound), the top-1024 must equal both the
+    oracle's and the unfiltered run's (debug flag 16: exact K2 for every quad)."""
+    w = WINDOWS[cfg]
+    d = datagen.make_config(cfg, n_snps=w, planted=False)
+    ref_idx, ref_k2 = oracle.search(d.geno, d.phen, top_k=1024)
+    with _engine("tc") as e:
+        e.load_genotypes(d.geno, d.phen)
+        idx, k2 = e.search(1024)
+        n_exact = e.stats()["prof"][0]
+    with _engine("tc", debug=16) as e:
+        e.load_genotypes(d.geno, d.phen)
+        idx_u, k2_u = e.search(1024)
+    np.testing.assert_array_equal(idx, ref_idx)
+    np.testing.assert_array_equal(k2, ref_k2)
+    np.testing.assert_array_equal(idx_u, ref_idx)
+    np.testing.assert_array_equal(k2_u, ref_k2)
+    assert 1024 <= n_exact < len(all_quads(w))          # the filter did filter
