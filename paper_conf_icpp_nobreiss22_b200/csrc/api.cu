@@ -133,6 +133,7 @@ DevData devdata(const epi4_ctx* c) {
     d.npad = c->npad;
     d.np[0] = (uint32_t)c->np[0];
     d.np[1] = (uint32_t)c->np[1];
+    d.npk = (uint32_t)c->np[0] | ((uint32_t)c->np[1] << d.pk_shift);
     d.T1 = c->T1;
     d.T2 = c->T2;
     d.T3 = c->T3;
@@ -220,11 +221,18 @@ int finish_load(epi4_ctx* c) {
     if (st & EPI4_ST_BAD_PHEN) return fail(EPI4_EINVAL, "phenotype value > 1");
     if (st & EPI4_ST_PAD_BITS) return fail(EPI4_EINVAL, "pad bits beyond the sample count are set");
     if (st & EPI4_ST_AA_AND_Aa) return fail(EPI4_EINVAL, "a sample has both AA and Aa bits set");
-    // lower-order tables
+    // lower-order tables: packed (control | case << pk_shift) words, epilogue.cuh
+    {
+        const DevData dd = devdata(c);
+        if (c->np[0] >= ((int64_t)1 << 22) || c->np[1] >= ((int64_t)1 << 22) ||
+            c->np[1] >= ((int64_t)1 << (32 - dd.pk_shift)))
+            return fail(EPI4_EINVAL, "n0=%lld / n1=%lld: counts are packed (control | case) into one 32-bit word, which "
+                        "needs bits(n0) + bits(n1) <= 32 and each < 2^22", (long long)c->np[0], (long long)c->np[1]);
+    }
     const int64_t n = c->n;
-    CU(grow(c->T1, c->cap_T1, (size_t)n * 4 * sizeof(uint32_t)));
-    CU(grow(c->T2, c->cap_T2, (size_t)c2(n) * 8 * sizeof(uint32_t)));
-    const size_t t3b = (size_t)c3(n) * 16 * sizeof(uint32_t);
+    CU(grow(c->T1, c->cap_T1, (size_t)n * 2 * sizeof(uint32_t)));
+    CU(grow(c->T2, c->cap_T2, (size_t)c2(n) * 4 * sizeof(uint32_t)));
+    const size_t t3b = (size_t)c3(n) * 8 * sizeof(uint32_t);
     size_t freeb = 0, totb = 0;
     CU(cudaMemGetInfo(&freeb, &totb));
     if (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
@@ -503,15 +511,6 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!quads_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
-    if (c->opts.pipe == EPI4_PIPE_TC) {
-        // the tensor-core epilogue packs (c0, c1) into 32 bits and the fp32 filter needs counts < 2^22
-        const DevData dd = devdata(c);
-        if (c->np[0] >= ((int64_t)1 << 22) || c->np[1] >= ((int64_t)1 << 22) ||
-            c->np[1] >= ((int64_t)1 << (32 - dd.pk_shift)))
-            return fail(EPI4_EINVAL, "n0=%lld / n1=%lld: the tensor-core pipe needs both counts to fit one 32-bit word "
-                        "(bits(n0) + bits(n1) <= 32) and each < 2^22; use pipe lop3", (long long)c->np[0],
-                        (long long)c->np[1]);
-    }
     CU(cudaSetDevice(c->device));
     std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
     const int64_t nall = (int64_t)plan.size();

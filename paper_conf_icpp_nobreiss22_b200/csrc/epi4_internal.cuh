@@ -9,9 +9,10 @@
 //                UMMA 128-byte swizzle applied in HBM (16-byte piece c of row r stored at piece c ^ (r & 7)), so
 //                one linear 32 KiB bulk copy lands two chunks of a 128-row A tile in the canonical K-major SW128
 //                shared-memory layout; the chunk count is padded to even with zero chunks.
-//   T1[snp][p][2]          popc(P_a(snp))                              (PAPER.md:L85 indivPop)
-//   T2[rank2][p][4]        popc(P_a(i) & P_b(j)), i<j, cell 2a+b       (PAPER.md:L86 pairwPop)
-//   T3[rank3][p][8]        popc(P_a(i) & P_b(j) & P_c(k)), i<j<k, cell 4a+2b+c
+//   lower-order tables, every entry a PACKED pair c0 | c1 << pk_shift (controls low, cases high; epilogue.cuh):
+//   T1[snp][2]          popc(P_a(snp))                              (PAPER.md:L85 indivPop)
+//   T2[rank2][4]        popc(P_a(i) & P_b(j)), i<j, cell 2a+b       (PAPER.md:L86 pairwPop)
+//   T3[rank3][8]        popc(P_a(i) & P_b(j) & P_c(k)), i<j<k, cell 4a+2b+c
 //   lgam[n] = lgamma(n+1) for n in [0, M+1], double, built on the host
 // colex ranks: rank2(i,j) = C(j,2)+i, rank3(i,j,k) = C(k,3)+C(j,2)+i, rank4 = C(l,4)+C(k,3)+C(j,2)+i.
 #pragma once
@@ -57,10 +58,11 @@ struct DevData {
     int32_t nchunks4[2];         // 256-sample fp4 chunks per phenotype (rows of expl)
     int32_t nsteps[2];           // tensor-core pipeline steps per phenotype: pairs of fp4 chunks (512 samples)
     int32_t nrb;                 // 128-row blocks of expl per chunk (= npad / 64)
-    int32_t pk_shift;            // tensor-core epilogue: (control, case) counts packed as c0 | c1 << pk_shift
+    int32_t pk_shift;            // (control, case) counts packed as c0 | c1 << pk_shift everywhere (bits(n0))
     int32_t n;                   // SNPs
     int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
     uint32_t np[2];              // n0, n1
+    uint32_t npk;                // n0 | n1 << pk_shift
     const uint32_t* T1;
     const uint32_t* T2;
     const uint32_t* T3;

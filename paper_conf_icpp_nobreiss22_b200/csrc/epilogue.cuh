@@ -11,7 +11,8 @@
 //   (2) recover every cell with an aa genotype axis by axis, v_aa = v_* - v_AA - v_Aa
 //       ("subtracting the counts for genotypes {..Y0..} and {..Y1..} from the counts
 //       for the third-order genotype", applied recursively, L130-131) — after axis t the digit 2 on
-//       axis t means aa; 4 axes x 27 slices x 2 subtractions = 216 per phenotype;
+//       axis t means aa; 108 three-input subtractions on packed (control | case) words cover both
+//       phenotypes at once (section "packed counts" below);
 //   (3) K2 in double in canonical cell order (reading #4):
 //       t_c = (L[r_c0 + r_c1 + 1] - L[r_c0]) - L[r_c1], K2 += t_c, c = 0..80, L[n] = lgamma(n+1);
 //   (4) keep the best quads: (K2, packed index) keys offered to a per-CTA sorted top-k list in shared
@@ -21,37 +22,83 @@
 
 namespace epi4 {
 
-// ---- lower-order table access (both phenotypes of an entry are adjacent) ----------------------------
-// T3 entry of (i<j<k): 16 uint32 = [p][4a+2b+c];  T2 entry of (i<j): 8 uint32 = [p][2a+b];  T1[snp]: [p][a].
-__device__ __forceinline__ uint4 t3_half(const DevData& d, int i, int j, int k, int p, int a) {
-    // the 4 cells with first genotype a of phenotype p
-    return __ldg(reinterpret_cast<const uint4*>(d.T3 + rank3(i, j, k) * 16 + p * 8 + a * 4));
+// ---- packed counts -----------------------------------------------------------------------------------
+// Every count the epilogue handles is a PACKED pair v = c0 | c1 << pks (controls in the low pks bits, cases
+// above; pks = bits(n0), api.cu checks bits(n0) + bits(n1) <= 32).  The aa recovery of PAPER.md:L126 is a
+// chain of subtractions v_aa = v_* - v_AA - v_Aa in which every operand and every result is the number of
+// samples of one phenotype in a genotype subset, i.e. a non-negative count per field: no borrow ever crosses
+// the field boundary, so one 32-bit subtraction recovers both phenotypes exactly (half the instructions of
+// two separate recoveries, and half the table bytes).
+//
+// Lower-order tables (api.cu / k_prep.cu, colex ranks):  T3[rank3(i,j,k)][4a+2b+c], T2[rank2(i,j)][2a+b],
+// T1[snp][a], all packed; d.npk = n0 | n1 << pks.
+__device__ __forceinline__ uint4 t3_half(const DevData& d, int64_t r3, int a) {   // cells (a, b, c), 2b + c
+    return __ldg(reinterpret_cast<const uint4*>(d.T3 + r3 * 8 + a * 4));
 }
-__device__ __forceinline__ uint2 t2_row(const DevData& d, int i, int j, int p, int a) {
-    return __ldg(reinterpret_cast<const uint2*>(d.T2 + rank2(i, j) * 8 + p * 4 + a * 2));
+__device__ __forceinline__ uint4 t2_all(const DevData& d, int64_t r2) {            // cells 2a + b
+    return __ldg(reinterpret_cast<const uint4*>(d.T2 + r2 * 4));
 }
-__device__ __forceinline__ uint4 t2_all(const DevData& d, int i, int j, int p) {
-    return __ldg(reinterpret_cast<const uint4*>(d.T2 + rank2(i, j) * 8 + p * 4));
-}
-__device__ __forceinline__ uint2 t1_all(const DevData& d, int i, int p) {
-    return __ldg(reinterpret_cast<const uint2*>(d.T1 + (int64_t)i * 4 + p * 2));
+__device__ __forceinline__ uint2 t1_all(const DevData& d, int i) {                 // cells a
+    return __ldg(reinterpret_cast<const uint2*>(d.T1 + (int64_t)i * 2));
 }
 __device__ __forceinline__ uint32_t u4(const uint4& v, int k) { return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w; }
 __device__ __forceinline__ uint32_t u2(const uint2& v, int k) { return k == 0 ? v.x : v.y; }
 
-// Slab decomposition along the first SNP (w) of the quad.  For α in {0, 1, '*'} the slab
-// S_α[β][γ][δ] = G[α][β][γ][δ] holds 27 generalized counts (digits in {0, 1, 2 = '*'}):
-//   slab '*' (w marginalised): T3(x,y,z), T2 of (x,y),(x,z),(y,z), T1 of x,y,z and n_p;
-//   slab α in {0,1}:           the 4-way counts c16[α...], T3 of (w,x,y),(w,x,z),(w,y,z), T2 of (w,.),
-//                              T1(w) — all restricted to genotype α of w.
-// Möbius on the remaining three axes gives the cells r[α][...] for α = 0, 1; and, because the
-// recovery is linear, r[2][...] = M3(S_*) - M3(S_0) - M3(S_1)  (PAPER.md:L126 applied on axis w).
-// Cells therefore come out a-major, i.e. in canonical order c = 27a + 9b + 3c + d.
-template <int P>
-__device__ __forceinline__ void fill_slab_star(int (&g)[27], const DevData& d, int x, int y, int z) {
-    const uint4 txyz0 = t3_half(d, x, y, z, P, 0), txyz1 = t3_half(d, x, y, z, P, 1);
-    const uint4 pxy = t2_all(d, x, y, P), pxz = t2_all(d, x, z, P), pyz = t2_all(d, y, z, P);
-    const uint2 sx = t1_all(d, x, P), sy = t1_all(d, y, P), sz = t1_all(d, z, P);
+// colex ranks of the lower-order tables a quad w < x < y < z reads
+struct QuadRanks {
+    int64_t wxy, wxz, wyz, xyz;   // T3
+    int64_t wx, wy, wz, xy, xz, yz;   // T2
+};
+__device__ __forceinline__ QuadRanks quad_ranks(int w, int x, int y, int z) {
+    QuadRanks q;
+    const int64_t c2x = c2(x), c2y = c2(y), c2z = c2(z), c3y = c3(y), c3z = c3(z);
+    q.wxy = c3y + c2x + w;
+    q.wxz = c3z + c2x + w;
+    q.wyz = c3z + c2y + w;
+    q.xyz = c3z + c2y + x;
+    q.wx = c2x + w;
+    q.wy = c2y + w;
+    q.wz = c2z + w;
+    q.xy = c2y + x;
+    q.xz = c2z + x;
+    q.yz = c2z + y;
+    return q;
+}
+
+// Generalized counts of one slab along the first SNP w: for w-genotype A in {AA, Aa}
+// or '*' (any), S[9b + 3e + f] with digits b (x), e (y), f (z) in {0 = AA, 1 = Aa, 2 = '*'}:
+//   no '*'    -> the 4-way contraction counts c16[8A + 4b + 2e + f]
+//   one '*'   -> 3-way tables of the other three SNPs
+//   two '*'   -> 2-way tables
+//   three '*' -> 1-way table / n_p
+template <int A>
+__device__ __forceinline__ void fill_slab_w(uint32_t (&S)[27], const uint32_t (&c16)[16], const uint4& twxy,
+                                            const uint4& twxz, const uint4& twyz, const uint4& pwx, const uint4& pwy,
+                                            const uint4& pwz, const uint2& sw) {
+#pragma unroll
+    for (int c = 0; c < 27; ++c) {
+        const int b = c / 9, e = (c / 3) % 3, f = c % 3;
+        const int ns = (b == 2) + (e == 2) + (f == 2);
+        uint32_t v;
+        if (ns == 0) v = c16[A * 8 + b * 4 + e * 2 + f];
+        else if (ns == 1) {
+            if (f == 2) v = u4(twxy, b * 2 + e);
+            else if (e == 2) v = u4(twxz, b * 2 + f);
+            else v = u4(twyz, e * 2 + f);
+        } else if (ns == 2) {
+            if (b != 2) v = u4(pwx, A * 2 + b);
+            else if (e != 2) v = u4(pwy, A * 2 + e);
+            else v = u4(pwz, A * 2 + f);
+        } else {
+            v = u2(sw, A);
+        }
+        S[c] = v;
+    }
+}
+// slab w = '*': the (x, y, z) marginal tables
+__device__ __forceinline__ void fill_slab_star(uint32_t (&S)[27], const uint4& txyz0, const uint4& txyz1,
+                                               const uint4& pxy, const uint4& pxz, const uint4& pyz, const uint2& sx,
+                                               const uint2& sy, const uint2& sz, uint32_t npk) {
 #pragma unroll
     for (int c = 0; c < 27; ++c) {
         const int b = c / 9, e = (c / 3) % 3, f = c % 3;
@@ -67,76 +114,14 @@ __device__ __forceinline__ void fill_slab_star(int (&g)[27], const DevData& d, i
             else if (e != 2) v = u2(sy, e);
             else v = u2(sz, f);
         } else {
-            v = d.np[P];
+            v = npk;
         }
-        g[c] = (int)v;
-    }
-}
-template <int P, int A>
-__device__ __forceinline__ void fill_slab_w(int (&g)[27], const uint32_t (&c16)[16], const DevData& d, int w, int x,
-                                            int y, int z) {
-    const uint4 twxy = t3_half(d, w, x, y, P, A), twxz = t3_half(d, w, x, z, P, A), twyz = t3_half(d, w, y, z, P, A);
-    const uint2 pwx = t2_row(d, w, x, P, A), pwy = t2_row(d, w, y, P, A), pwz = t2_row(d, w, z, P, A);
-    const uint2 sw = t1_all(d, w, P);
-#pragma unroll
-    for (int c = 0; c < 27; ++c) {
-        const int b = c / 9, e = (c / 3) % 3, f = c % 3;
-        const int ns = (b == 2) + (e == 2) + (f == 2);
-        uint32_t v;
-        if (ns == 0) v = c16[A * 8 + b * 4 + e * 2 + f];
-        else if (ns == 1) {
-            if (f == 2) v = u4(twxy, b * 2 + e);
-            else if (e == 2) v = u4(twxz, b * 2 + f);
-            else v = u4(twyz, e * 2 + f);
-        } else if (ns == 2) {
-            if (b != 2) v = u2(pwx, b);
-            else if (e != 2) v = u2(pwy, e);
-            else v = u2(pwz, f);
-        } else {
-            v = u2(sw, A);
-        }
-        g[c] = (int)v;
+        S[c] = v;
     }
 }
 
-// Slab α = aa of w, before recovery: S_*[c] - S_0[c] - S_1[c] (the generalized counts restricted to w = aa).
-// Because the recovery is linear, M3 of it is r[2][...] (PAPER.md:L126 applied on axis w); computing it from
-// the raw tables (instead of keeping M3(S_*), M3(S_0), M3(S_1) alive) holds one slab per phenotype at a time.
-template <int P>
-__device__ __forceinline__ void fill_slab_aa(int (&g)[27], const uint32_t (&c16)[16], const DevData& d, int w, int x,
-                                             int y, int z) {
-    const uint4 txyz0 = t3_half(d, x, y, z, P, 0), txyz1 = t3_half(d, x, y, z, P, 1);
-    const uint4 pxy = t2_all(d, x, y, P), pxz = t2_all(d, x, z, P), pyz = t2_all(d, y, z, P);
-    const uint2 sx = t1_all(d, x, P), sy = t1_all(d, y, P), sz = t1_all(d, z, P);
-    const uint4 twxy0 = t3_half(d, w, x, y, P, 0), twxy1 = t3_half(d, w, x, y, P, 1);
-    const uint4 twxz0 = t3_half(d, w, x, z, P, 0), twxz1 = t3_half(d, w, x, z, P, 1);
-    const uint4 twyz0 = t3_half(d, w, y, z, P, 0), twyz1 = t3_half(d, w, y, z, P, 1);
-    const uint4 pwx = t2_all(d, w, x, P), pwy = t2_all(d, w, y, P), pwz = t2_all(d, w, z, P);
-    const uint2 sw = t1_all(d, w, P);
-#pragma unroll
-    for (int c = 0; c < 27; ++c) {
-        const int b = c / 9, e = (c / 3) % 3, f = c % 3;
-        const int ns = (b == 2) + (e == 2) + (f == 2);
-        uint32_t v;
-        if (ns == 0) {
-            v = (b ? u4(txyz1, e * 2 + f) : u4(txyz0, e * 2 + f)) - c16[b * 4 + e * 2 + f] - c16[8 + b * 4 + e * 2 + f];
-        } else if (ns == 1) {
-            if (f == 2) v = u4(pxy, b * 2 + e) - u4(twxy0, b * 2 + e) - u4(twxy1, b * 2 + e);
-            else if (e == 2) v = u4(pxz, b * 2 + f) - u4(twxz0, b * 2 + f) - u4(twxz1, b * 2 + f);
-            else v = u4(pyz, e * 2 + f) - u4(twyz0, e * 2 + f) - u4(twyz1, e * 2 + f);
-        } else if (ns == 2) {
-            if (b != 2) v = u2(sx, b) - u4(pwx, b) - u4(pwx, 2 + b);
-            else if (e != 2) v = u2(sy, e) - u4(pwy, e) - u4(pwy, 2 + e);
-            else v = u2(sz, f) - u4(pwz, f) - u4(pwz, 2 + f);
-        } else {
-            v = d.np[P] - sw.x - sw.y;
-        }
-        g[c] = (int)v;
-    }
-}
-
-// aa recovery on the three axes of a slab (strides 9, 3, 1): 3 x 9 x 2 = 54 subtractions
-__device__ __forceinline__ void mobius3(int (&g)[27]) {
+// aa recovery on the three axes of a slab (strides 9, 3, 1): 27 three-input subtractions on packed words
+__device__ __forceinline__ void mobius3(uint32_t (&g)[27]) {
 #pragma unroll
     for (int ax = 0; ax < 3; ++ax) {
         const int s = ax == 0 ? 9 : ax == 1 ? 3 : 1;
@@ -154,74 +139,102 @@ __device__ __forceinline__ void mobius3(int (&g)[27]) {
 // K2 - (ln2 sum T_c - 81 - 81 C0) lies in (-13.5, 3.375).  With the fp32 rounding bound E(M) computed on the
 // host (api.cu: filter_offset), K2 > ln2 A - 81 - 81 C0 - 13.5 - E for the computed A = sum T_c, so a quad is
 // scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
-// is exactly the oracle's.  Per cell: 2 LOP3 + 7 FADD/FMUL + 2 FFMA + 3 MUFU, no table, no conversions
-// (a count r < 2^22 becomes the float 2^23 + r by an OR of the exponent bits; r + 1 and r + 1/2 then follow
-// by one exact FADD each).
+// is exactly the oracle's.  Per cell: 3 ALU (unpack), 6 FADD + FMUL + 2 FFMA + 1 FADD, 3 MUFU; no table and
+// no conversion instruction (a count r < 2^22 becomes the float 2^23 + r by an OR of the exponent bits).
 __device__ __forceinline__ float lg2_approx(float x) {
     float y;
     asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
 }
-__device__ __forceinline__ float cell_T(int r0, int r1) {
-    const float m0 = __int_as_float(r0 | 0x4B000000), m1 = __int_as_float(r1 | 0x4B000000);   // 2^23 + r
-    const float f0 = m0 + (1.0f - 8388608.0f), f1 = m1 + (1.0f - 8388608.0f);              // r + 1
-    const float h0 = m0 + (0.5f - 8388608.0f), h1 = m1 + (0.5f - 8388608.0f);              // r + 1/2
-    const float fn = f0 + f1, hn = fn - 0.5f;                                               // n + 2, n + 3/2
+__device__ __forceinline__ float cell_T(uint32_t v, uint32_t pks, uint32_t pkm) {
+    const float m0 = __uint_as_float((v & pkm) | 0x4B000000u), m1 = __uint_as_float((v >> pks) | 0x4B000000u);
+    const float f0 = m0 - 8388607.0f, f1 = m1 - 8388607.0f;     // r + 1
+    const float h0 = m0 - 8388607.5f, h1 = m1 - 8388607.5f;     // r + 1/2
+    const float fn = f0 + f1, hn = h0 + f1;                     // n + 2, n + 3/2
     float t = hn * lg2_approx(fn);
     t = fmaf(-h0, lg2_approx(f0), t);
     return fmaf(-h1, lg2_approx(f1), t);
 }
 
-// Per-quad evaluation in canonical cell order, one slab (27 cells x 2 phenotypes) at a time:
-// alpha = AA (cells 0..26), Aa (27..53), aa (54..80).  MODE 0: the fp32 filter value A = sum T_c (above);
-// MODE 1: exact K2 in double, t_c = (L[r+1] - L[r0]) - L[r1], K2 += t_c, c = 0..80 (
-// reading #4); MODE 2: exact K2 and the 2 x 81 cells written to dump (controls first).
+// Per-quad evaluation from the 16 packed contraction counts c16[8a + 4b + 2c + d] of quad (w, x, y, z).
+// Slabs along w: R2 := M3(S_*) (the recovered (x, y, z) table); for A = AA, Aa: r_A = M3(S_A) is consumed
+// and subtracted from R2, which ends as r_aa = M3(S_*) - M3(S_AA) - M3(S_Aa) (linearity of the recovery,
+// PAPER.md:L126 applied on axis w).  Cells are consumed slab by slab in canonical order c = 27a + 9b + 3c + d.
+// MODE 0: the fp32 filter value A = sum T_c (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
+// L[r_c0]) - L[r_c1], K2 += t_c, c = 0..80 (reading #4); MODE 2: exact K2 and the
+// 2 x 81 cells written to dump (controls first).
 template <int MODE>
-__device__ __forceinline__ void quad_eval(const DevData& d, int w, int x, int y, int z, const uint32_t (&c0)[16],
-                                          const uint32_t (&c1)[16], float& flt, double& k2, uint32_t* dump) {
+__device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, int w, int x, int y, int z,
+                                          const uint32_t (&c16)[16], float& flt, double& k2, uint32_t* dump) {
+    const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
+    // all table reads up front (one round of load latency per quad)
+    const uint4 txyz0 = t3_half(d, q.xyz, 0), txyz1 = t3_half(d, q.xyz, 1);
+    const uint4 pxy = t2_all(d, q.xy), pxz = t2_all(d, q.xz), pyz = t2_all(d, q.yz);
+    const uint2 sx = t1_all(d, x), sy = t1_all(d, y), sz = t1_all(d, z);
+    const uint4 twxy0 = t3_half(d, q.wxy, 0), twxz0 = t3_half(d, q.wxz, 0), twyz0 = t3_half(d, q.wyz, 0);
+    const uint4 twxy1 = t3_half(d, q.wxy, 1), twxz1 = t3_half(d, q.wxz, 1), twyz1 = t3_half(d, q.wyz, 1);
+    const uint4 pwx = t2_all(d, q.wx), pwy = t2_all(d, q.wy), pwz = t2_all(d, q.wz);
+    const uint2 sw = t1_all(d, w);
     float fa = 0.0f, fb = 0.0f;
     double kk = 0.0;
-    auto consume = [&](const int (&T0)[27], const int (&T1)[27], int base) {
+    auto consume = [&](const uint32_t (&S)[27], int base) {
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
-            const int r0 = T0[c], r1 = T1[c];
             if (MODE == 0) {
-                const float t = cell_T(r0, r1);
+                const float t = cell_T(S[c], pks, pkm);
                 if (c & 1) fb += t; else fa += t;
             } else {
+                const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
                 const double t = __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1));
                 kk = __dadd_rn(kk, t);
                 if (MODE == 2) {
-                    dump[base + c] = (uint32_t)r0;
-                    dump[81 + base + c] = (uint32_t)r1;
+                    dump[base + c] = r0;
+                    dump[81 + base + c] = r1;
                 }
             }
         }
     };
+    uint32_t R2[27];
+    fill_slab_star(R2, txyz0, txyz1, pxy, pxz, pyz, sx, sy, sz, d.npk);
+    mobius3(R2);
+    {
+        uint32_t S[27];
+        fill_slab_w<0>(S, c16, twxy0, twxz0, twyz0, pwx, pwy, pwz, sw);
+        mobius3(S);
+        consume(S, 0);
 #pragma unroll
-    for (int a = 0; a < 3; ++a) {
-        int T0[27], T1[27];
-        if (a == 0) { fill_slab_w<0, 0>(T0, c0, d, w, x, y, z); fill_slab_w<1, 0>(T1, c1, d, w, x, y, z); }
-        else if (a == 1) { fill_slab_w<0, 1>(T0, c0, d, w, x, y, z); fill_slab_w<1, 1>(T1, c1, d, w, x, y, z); }
-        else { fill_slab_aa<0>(T0, c0, d, w, x, y, z); fill_slab_aa<1>(T1, c1, d, w, x, y, z); }
-        mobius3(T0);
-        mobius3(T1);
-        consume(T0, T1, 27 * a);
+        for (int c = 0; c < 27; ++c) R2[c] -= S[c];
     }
+    {
+        uint32_t S[27];
+        fill_slab_w<1>(S, c16, twxy1, twxz1, twyz1, pwx, pwy, pwz, sw);
+        mobius3(S);
+        consume(S, 27);
+#pragma unroll
+        for (int c = 0; c < 27; ++c) R2[c] -= S[c];
+    }
+    consume(R2, 54);
     flt = fa + fb;
     k2 = kk;
 }
 
-// exact K2 of one quad (double, canonical order); optionally dumps its 162 cells.  Not inlined: in the
-// tensor-core epilogue it runs only for filter candidates, so its registers must not add to the hot loop's.
+// exact K2 of one quad (double, canonical order) from its packed contraction counts; optionally dumps its 162
+// cells.  Not inlined: in the tensor-core epilogue it runs only for filter candidates, so its registers must
+// not add to the hot loop's.
 static __device__ __noinline__ double score_quad(const DevData& d, int w, int x, int y, int z,
-                                          const uint32_t (&c0)[16], const uint32_t (&c1)[16],
-                                          uint32_t* dump_row) {
+                                                 const uint32_t (&c16)[16], uint32_t* dump_row) {
     float flt;
     double k2;
-    if (dump_row) quad_eval<2>(d, w, x, y, z, c0, c1, flt, k2, dump_row);
-    else quad_eval<1>(d, w, x, y, z, c0, c1, flt, k2, nullptr);
+    const QuadRanks q = quad_ranks(w, x, y, z);
+    if (dump_row) quad_eval<2>(d, q, w, x, y, z, c16, flt, k2, dump_row);
+    else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;
+}
+// pack separate control / case counts (CUDA-core kernels)
+__device__ __forceinline__ void pack16(const DevData& d, const uint32_t (&c0)[16], const uint32_t (&c1)[16],
+                                       uint32_t (&c16)[16]) {
+#pragma unroll
+    for (int k = 0; k < 16; ++k) c16[k] = c0[k] | (c1[k] << d.pk_shift);
 }
 
 // ---------------------------------------------------------------------------------------------

@@ -217,8 +217,7 @@ __global__ void __launch_bounds__(256) k_pop1(DevData d, uint32_t* __restrict__ 
                 const uint4 v = __ldg(reinterpret_cast<const uint4*>(d.planes[p] + plane_off(kc, d.npad, snp, g, 0)));
                 c[p][g] += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
             }
-    uint4 o = make_uint4(c[0][0], c[0][1], c[1][0], c[1][1]);
-    reinterpret_cast<uint4*>(T1)[snp] = o;
+    reinterpret_cast<uint2*>(T1)[snp] = make_uint2(c[0][0] | (c[1][0] << d.pk_shift), c[0][1] | (c[1][1] << d.pk_shift));
 }
 
 __device__ __forceinline__ void decode2(int64_t r, int& i, int& j) {
@@ -265,9 +264,9 @@ __global__ void __launch_bounds__(256) k_pop2(DevData d, uint32_t* __restrict__ 
 #pragma unroll
         for (int q = 0; q < 4; ++q) out[p][q] = c[q];
     }
-    uint4* o = reinterpret_cast<uint4*>(T2 + r * 8);
-    o[0] = make_uint4(out[0][0], out[0][1], out[0][2], out[0][3]);
-    o[1] = make_uint4(out[1][0], out[1][1], out[1][2], out[1][3]);
+    const uint32_t s = (uint32_t)d.pk_shift;
+    reinterpret_cast<uint4*>(T2)[r] = make_uint4(out[0][0] | (out[1][0] << s), out[0][1] | (out[1][1] << s),
+                                                 out[0][2] | (out[1][2] << s), out[0][3] | (out[1][3] << s));
 }
 
 __global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ T3, int64_t ntri) {
@@ -297,11 +296,12 @@ __global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ 
 #pragma unroll
         for (int q = 0; q < 8; ++q) out[p][q] = c[q];
     }
-    uint4* o = reinterpret_cast<uint4*>(T3 + r * 16);
-    o[0] = make_uint4(out[0][0], out[0][1], out[0][2], out[0][3]);
-    o[1] = make_uint4(out[0][4], out[0][5], out[0][6], out[0][7]);
-    o[2] = make_uint4(out[1][0], out[1][1], out[1][2], out[1][3]);
-    o[3] = make_uint4(out[1][4], out[1][5], out[1][6], out[1][7]);
+    const uint32_t s = (uint32_t)d.pk_shift;
+    uint4* o = reinterpret_cast<uint4*>(T3 + r * 8);
+    o[0] = make_uint4(out[0][0] | (out[1][0] << s), out[0][1] | (out[1][1] << s), out[0][2] | (out[1][2] << s),
+                      out[0][3] | (out[1][3] << s));
+    o[1] = make_uint4(out[0][4] | (out[1][4] << s), out[0][5] | (out[1][5] << s), out[0][6] | (out[1][6] << s),
+                      out[0][7] | (out[1][7] << s));
 }
 
 cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, cudaStream_t s,

@@ -110,7 +110,9 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
                     c1[c] = s_cnt[((1 * LOP3_Q + m) * 16 + c) * LOP3_THREADS + tid];
                 }
                 uint32_t* dump = sp.dump ? sp.dump + rank4(w, x, y, z) * 162 : nullptr;
-                key = score_quad(d, w, x, y, z, c0, c1, dump);
+                uint32_t c16[16];
+                pack16(d, c0, c1, c16);
+                key = score_quad(d, w, x, y, z, c16, dump);
                 idx = pack_quad(w, x, y, z);
                 ++my_quads;
             }

@@ -61,8 +61,12 @@ constexpr int B_ROWS = N / 2;            // this CTA's 80 B columns
 constexpr int B_SUB = (B_ROWS + 7) / 8 * 1024;
 constexpr int B_BYTES = CHUNKS * B_SUB;
 constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (10)
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;             // 52 KiB, 1024-aligned
-constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per stage
+constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per A stage
+#ifndef EPI4_A_SPLIT
+#define EPI4_A_SPLIT 4
+#endif
+constexpr int A_SPLIT = EPI4_A_SPLIT;    // lanes issuing one A stage's bulk copy in pieces (tools/probe_tma.cu: several
+                                         // concurrently issued copies ingest faster than one)
 #ifndef EPI4_PROD_WARPS
 #define EPI4_PROD_WARPS 4
 #endif
@@ -74,7 +78,6 @@ constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate st
 constexpr int TMA_WARPS = 2;             // a bulk-copy issue blocks its thread ~150-200 cycles: two warps alternate
 constexpr int TMA_WARP0 = MMA_WARPS, PROD_WARP0 = TMA_WARP0 + TMA_WARPS, EPI_WARP0 = PROD_WARP0 + PROD_WARPS;
 constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 512 with 4 producer warps (128 registers each before setmaxnreg)
-constexpr int MAX_STAGES = 12;
 // register split across the 4 warpgroups (needs the 16-warp layout: MMA+TMA | producers | 2 x epilogue)
 #ifndef EPI4_REGSPLIT
 #define EPI4_REGSPLIT 1
@@ -90,7 +93,6 @@ constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
 constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 56 / 96
 constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
 constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
-constexpr int STAGE_Q = lcm_c(lcm_c(PROD_STRIDE, MMA_WARPS), TMA_WARPS);   // stage counts: multiples
 constexpr int TMEM_COLS = 512;
 constexpr int REGIONS = 3;               // accumulator regions of N columns, rotated per tile (header comment)
 constexpr int ACC_COLS = REGIONS * N;
@@ -326,28 +328,40 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 #define PCLK() 0LL
 #endif
 
-template <int STAGES>
+// Global step s of a cluster uses A stage s % SA (phase (s / SA) & 1) and B stage s % SB.  The two MMA
+// issuers may issue (and complete) the steps of the other parity out of order, so a waiter is only protected
+// from phase aliasing if its previous wait on a ring was on the same issuer's steps: both ring sizes must be
+// multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
+template <int SA, int SB>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
-    static_assert(STAGES % tc::STAGE_Q == 0, "a producer's / issuer's successive uses of a stage must be one phase apart");
+    static_assert(SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2,
+                  "ring sizes must be multiples of the alternating warps' stride (phase aliasing)");
     extern __shared__ unsigned char smem_raw[];
-    __shared__ __align__(8) uint64_t sfull_bar[STAGES], full_bar[STAGES], empty_bar[STAGES];
+    // A ring: afull (own TMA landed), apeer (@leader: the follower's A landed, relayed), aempty (MMA commit);
+    // B ring: bfull (@leader: both CTAs' producers), bempty (MMA commit)
+    __shared__ __align__(8) uint64_t afull_bar[SA], apeer_bar[SA], aempty_bar[SA], bfull_bar[SB], bempty_bar[SB];
     __shared__ __align__(8) uint64_t tfull_bar[2], pk_bar, ep_bar[2];
     __shared__ uint32_t s_tmem;
-    // 1024-aligned stage ring, then the top-k state
+    // 1024-aligned A ring, then the B ring, then the top-k state
     // (same offsets in both CTAs of the pair: the MMA addresses the peer's operands at the same offsets)
     const uint32_t raw = smem_u32(smem_raw);
     unsigned char* ring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-    TopKSmem tk = topk_carve(ring + STAGES * tc::STAGE_BYTES, sp.topk);
+    unsigned char* bring = ring + SA * tc::A_BYTES;
+    TopKSmem tk = topk_carve(bring + SB * tc::B_BYTES, sp.topk);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const DevData& d = sp.d;
     const uint32_t rank = cluster_rank();
     const bool leader = rank == 0;
     if (tid == 0) {
-        for (int s = 0; s < STAGES; ++s) {
-            mbar_init(&sfull_bar[s], 1);
-            mbar_init(&full_bar[s], tc::CLUSTER * tc::CHUNKS + 1);   // (leader) both CTAs' producers + the A relay
-            mbar_init(&empty_bar[s], 1);                  // the leader's MMA commit
+        for (int s = 0; s < SA; ++s) {
+            mbar_init(&afull_bar[s], 1);
+            mbar_init(&apeer_bar[s], 1);                  // (leader) the follower's relay
+            mbar_init(&aempty_bar[s], 1);                 // the leader's MMA commit
+        }
+        for (int s = 0; s < SB; ++s) {
+            mbar_init(&bfull_bar[s], tc::CLUSTER * tc::CHUNKS);   // (leader) both CTAs' producers
+            mbar_init(&bempty_bar[s], 1);                 // the leader's MMA commit
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&tfull_bar[b], tc::MMA_WARPS);      // each issuer's commit after its last step
@@ -403,11 +417,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         // epilogue re-zeroes the accumulators), so the two issuers' MMAs commute.
         if (leader) {
             const int m = warp;
-            const uint32_t ring_s = smem_u32(ring);
-            const uint64_t adesc0 = sw128_desc(ring_s), bdesc0 = sw128_desc(ring_s + tc::A_BYTES);
+            const uint32_t ring_s = smem_u32(ring), bring_s = smem_u32(bring);
+            const uint64_t adesc0 = sw128_desc(ring_s), bdesc0 = sw128_desc(bring_s);
             const uint32_t sf_addr = tmem + tc::SF_COL;
-            int stage = m;
-            uint32_t phase = 0, soff = (uint32_t)m * (tc::STAGE_BYTES >> 4);
             int it = 0, gstep = 0;
             long long t_wait = 0, t_tempty = 0;
             const bool do_mma = !(sp.debug & 4);
@@ -432,30 +444,32 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 #pragma unroll 1
                     for (int kc = 0; kc < nch; ++kc, ++gstep) {
                         if ((gstep & (tc::MMA_WARPS - 1)) != m) continue;
+                        const int sa = gstep % SA, sb = gstep % SB;
+                        const uint32_t pa = (uint32_t)((gstep / SA) & 1), pb = (uint32_t)((gstep / SB) & 1);
                         const long long t0 = PCLK();
                         if (lane == 0) TRACE(12, gstep);
-                        mbar_wait(&full_bar[stage], phase);         // both B halves built, follower's A landed
+                        mbar_wait(&bfull_bar[sb], pb);              // both B halves built
                         if (lane == 0) TRACE(15, gstep);
-                        mbar_wait(&sfull_bar[stage], phase);        // own A landed
+                        mbar_wait(&apeer_bar[sa], pa);              // follower's A landed
+                        mbar_wait(&afull_bar[sa], pa);              // own A landed
                         t_wait += PCLK() - t0;
                         if (lane == 0) TRACE(10, gstep);
                         tc_fence_after();
                         if (elect_one()) {
                             if (do_mma) {
+                                const uint32_t aoff = (uint32_t)sa * (tc::A_BYTES >> 4), boff = (uint32_t)sb * (tc::B_BYTES >> 4);
 #pragma unroll
                                 for (int j = 0; j < tc::CHUNKS; ++j)
 #pragma unroll
                                     for (int k = 0; k < tc::ROWB / 32; ++k)
-                                        mma2_mxf4(dcol, adesc0 + soff + j * (tc::A_SUB >> 4) + 2 * k,
-                                                  bdesc0 + soff + j * (tc::B_SUB >> 4) + 2 * k, sf_addr);
+                                        mma2_mxf4(dcol, adesc0 + aoff + j * (tc::A_SUB >> 4) + 2 * k,
+                                                  bdesc0 + boff + j * (tc::B_SUB >> 4) + 2 * k, sf_addr);
                             }
-                            mma2_commit_mc(&empty_bar[stage]);      // frees the stage in both CTAs
+                            mma2_commit_mc(&aempty_bar[sa]);        // frees the A stage in both CTAs
+                            mma2_commit_mc(&bempty_bar[sb]);        // and the B stage
                         }
                         __syncwarp();
                         if (lane == 0) TRACE(11, gstep);
-                        soff += tc::MMA_WARPS * (tc::STAGE_BYTES >> 4);
-                        stage += tc::MMA_WARPS;
-                        if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; soff -= STAGES * (tc::STAGE_BYTES >> 4); }
                     }
                 }
                 if (elect_one()) mma2_commit_mc(&tfull_bar[buf]);   // this issuer's MMAs of the tile are done
@@ -468,16 +482,13 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             }
         } else if (warp == 0) {
             // follower: relay "my A landed" (sfull) to the leader's full barrier, off the producers' path
-            int stage = 0;
-            uint32_t phase = 0;
             StepIt st;
             st.init(sp);
             for (int gstep = 0; st.valid(sp); st.advance(sp, 1), ++gstep) {
-                mbar_wait(&sfull_bar[stage], phase);
+                mbar_wait(&afull_bar[gstep % SA], (uint32_t)((gstep / SA) & 1));
                 if (lane == 0) TRACE(14, gstep);
-                if (lane == 0) mbar_arrive_cluster(&full_bar[stage], 0);
+                if (lane == 0) mbar_arrive_cluster(&apeer_bar[gstep % SA], 0);
                 __syncwarp();
-                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
             }
         }
         __syncwarp();
@@ -487,32 +498,32 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         // one elected lane issues
         {
             const int tw = warp - tc::TMA_WARP0;
-            int stage = tw;
-            uint32_t phase = 0;
             StepIt st;
             st.init(sp);
             st.advance(sp, tw);
             long long t_wait = 0;
             const uint32_t ring_s = smem_u32(ring);
             for (int gstep = tw; st.valid(sp); st.advance(sp, tc::TMA_WARPS), gstep += tc::TMA_WARPS) {
+                const int sa = gstep % SA;
                 const long long t0 = PCLK();
-                mbar_wait(&empty_bar[stage], phase ^ 1u);
+                mbar_wait(&aempty_bar[sa], (uint32_t)((gstep / SA) & 1) ^ 1u);
                 t_wait += PCLK() - t0;
                 if (lane == 0) TRACE(0, gstep);
-                // this CTA's 128 A rows (row block 2 wp + rank) of the step's two chunks: one 32 KiB bulk copy
+                // this CTA's 128 A rows (row block 2 wp + rank) of the step's two chunks: 32 contiguous KiB in HBM,
+                // copied as A_SPLIT pieces issued by as many lanes
                 const uint8_t* src = (st.p ? expl1 : expl0) +
                                      expl_off(2 * (int64_t)st.chunk(), (int64_t)(st.ti.wp * 2 + (int)rank) * 128, nrb);
-                if (elect_one()) {
-                    mbar_expect_tx(&sfull_bar[stage], tc::TX_BYTES);
+                if (lane == 0) mbar_expect_tx(&afull_bar[sa], tc::TX_BYTES);
+                __syncwarp();
+                if (lane < tc::A_SPLIT) {
+                    constexpr uint32_t piece = tc::A_BYTES / tc::A_SPLIT;
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                                 ::"r"(ring_s + (uint32_t)(stage * tc::STAGE_BYTES)), "l"(src),
-                                 "r"((uint32_t)tc::A_BYTES), "r"(smem_u32(&sfull_bar[stage]))
+                                 ::"r"(ring_s + (uint32_t)(sa * tc::A_BYTES) + lane * piece), "l"(src + lane * piece),
+                                 "r"(piece), "r"(smem_u32(&afull_bar[sa]))
                                  : "memory");
                 }
                 __syncwarp();
                 if (lane == 0) TRACE(1, gstep);
-                stage += tc::TMA_WARPS;
-                if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; }
             }
             if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
         }
@@ -563,9 +574,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         };
         load(pre);
         pre.advance(sp, tc::PROD_STRIDE);
-        int stage = pstep0;
-        uint32_t phase = 0;
         for (int step = pstep0; st.valid(sp); step += tc::PROD_STRIDE) {
+            const int sb = step % SB;
             if (lane == 0) TRACE(2, step);
             uint4 cx[4], cy[YK];
 #pragma unroll
@@ -575,18 +585,18 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             load(pre);                                            // next own step's singles (in flight)
             pre.advance(sp, tc::PROD_STRIDE);
             const long long t0 = PCLK();
-            mbar_wait(&empty_bar[stage], phase ^ 1u);             // B slot free (MMA of step - STAGES done)
+            mbar_wait(&bempty_bar[sb], (uint32_t)((step / SB) & 1) ^ 1u);   // B slot free (MMA of step - SB done)
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             if (lane == 0) TRACE(4, step);
             if (build) {
-                unsigned char* sb = ring + stage * tc::STAGE_BYTES + tc::A_BYTES + jc * tc::B_SUB;
+                unsigned char* bdst = bring + sb * tc::B_BYTES + jc * tc::B_SUB;
                 const uint4 xz[4] = {and4(cx[0], cx[2]), and4(cx[0], cx[3]), and4(cx[1], cx[2]), and4(cx[1], cx[3])};
 #pragma unroll
                 for (int k = 0; k < YK; ++k)
 #pragma unroll
                     for (int bd = 0; bd < 4; ++bd)
-                        *reinterpret_cast<uint4*>(sb + boff[bd] + k * 2048) = and4(cy[k], xz[bd]);
+                        *reinterpret_cast<uint4*>(bdst + boff[bd] + k * 2048) = and4(cy[k], xz[bd]);
                 if (lane == 0) TRACE(6, step);
                 fence_proxy_async();                      // generic-proxy stores -> visible to the tensor core
             }
@@ -594,8 +604,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             const long long t2 = PCLK();
             if (lane == 0) {
                 TRACE(7, step);
-                if (leader) mbar_arrive_local(&full_bar[stage]);
-                else mbar_arrive_cluster(&full_bar[stage], 0);           // the leader's barrier
+                if (leader) mbar_arrive_local(&bfull_bar[sb]);
+                else mbar_arrive_cluster(&bfull_bar[sb], 0);             // the leader's barrier
                 TRACE(9, step);
             }
             __syncwarp();
@@ -605,8 +615,6 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 t_arr += t3 - t2;
             }
             st.advance(sp, tc::PROD_STRIDE);
-            stage += tc::PROD_STRIDE;
-            if (stage >= STAGES) { stage -= STAGES; phase ^= 1u; }
         }
         if (EPI4_PROF && lane == 0) {
             atomicAdd(sp.prof + 3, (unsigned long long)t_busy);
@@ -627,7 +635,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         long long t_wait = 0, t_busy = 0;
         const bool score = !(sp.debug & 2);
         int it = 0;
-        const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
+        const uint32_t pks = (uint32_t)d.pk_shift;
         int r0 = 0;                                     // the MMA issuers' region rotation
         for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
             const TileInfo ti = decode_tile(sp, tile);
@@ -680,18 +688,15 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         else mbar_arrive_cluster(&ep_bar[buf], 0);   // the leader's barrier
                     }
                 }
-                uint32_t c0[16], c1[16];
+                uint32_t c16[16];
 #pragma unroll
                 for (int k = 0; k < 8; ++k) {
-                    // send my values for the other lane's quad, keep mine
+                    // send my values for the other lane's quad, keep mine; lane a keeps c16[8a + k] = its own
+                    // v[8a + k] and takes c16[8(1-a) + k] from the partner (packed control | case words)
                     const uint32_t sv = a ? v[k] : v[8 + k];
                     const uint32_t rv = __shfl_xor_sync(0xffffffffu, sv, 1);
-                    // lane a keeps c16[8a + k] = its own v[8a + k] and takes c16[8(1-a) + k] from the partner
-                    const uint32_t lo = a ? rv : v[k], hi = a ? v[8 + k] : rv;
-                    c0[k] = lo & pkm;
-                    c1[k] = lo >> pks;
-                    c0[8 + k] = hi & pkm;
-                    c1[8 + k] = hi >> pks;
+                    c16[k] = a ? rv : v[k];
+                    c16[8 + k] = a ? v[8 + k] : rv;
                 }
                 const int y = ti.y0 + 2 * g + a;
                 const bool valid = (w < ti.x) && (y < ti.z) && score;
@@ -702,30 +707,21 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     uint32_t* dump = sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
                     offer = true;
                     if (dump) {
-                        uint32_t e0[16], e1[16];
-#pragma unroll
-                        for (int k = 0; k < 16; ++k) { e0[k] = c0[k]; e1[k] = c1[k]; }
-                        key = score_quad(d, w, ti.x, y, ti.z, e0, e1, dump);
+                        key = score_quad(d, w, ti.x, y, ti.z, c16, dump);
                     } else if (sp.use_filter) {
                         // fp32 Stirling filter (epilogue.cuh); only possible top-k members get the exact K2
                         float flt;
                         double unused;
-                        quad_eval<0>(d, w, ti.x, y, ti.z, c0, c1, flt, unused, nullptr);
+                        quad_eval<0>(d, quad_ranks(w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt, unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
                         offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
                             // rare path: the noinline exact scorer takes the counts through local memory
-                            uint32_t e0[16], e1[16];
-#pragma unroll
-                            for (int k = 0; k < 16; ++k) { e0[k] = c0[k]; e1[k] = c1[k]; }
-                            key = score_quad(d, w, ti.x, y, ti.z, e0, e1, nullptr);
+                            key = score_quad(d, w, ti.x, y, ti.z, c16, nullptr);
                             ++n_exact;
                         }
                     } else {
-                        uint32_t e0[16], e1[16];
-#pragma unroll
-                        for (int k = 0; k < 16; ++k) { e0[k] = c0[k]; e1[k] = c1[k]; }
-                        key = score_quad(d, w, ti.x, y, ti.z, e0, e1, nullptr);
+                        key = score_quad(d, w, ti.x, y, ti.z, c16, nullptr);
                     }
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;
@@ -768,9 +764,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 #endif
 }
 
-template <int STAGES>
+template <int SA, int SB>
 static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
-    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
@@ -784,7 +780,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_quad_tc<STAGES>, sp);
+    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB>, sp);
 }
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
@@ -799,30 +795,26 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024;   // alignment + static smem slack
-    // most pipeline stages that fit (a multiple of STAGE_Q: each producer / issuer / TMA warp takes every
-    // PROD_STRIDE-th / MMA_WARPS-th / TMA_WARPS-th step and must meet its stages one phase apart)
-    int st = 0;
-    for (int cand = tc::MAX_STAGES / tc::STAGE_Q * tc::STAGE_Q; cand >= tc::STAGE_Q && !st; cand -= tc::STAGE_Q)
-        if (fixed + (size_t)cand * tc::STAGE_BYTES <= (size_t)optin) st = cand;
-    if (!st) return cudaErrorInvalidConfiguration;
-    const size_t smem = 1024 + (size_t)st * tc::STAGE_BYTES + topk_smem_bytes(sp.topk);
+    // deepest rings that fit (the A copies carry the long L2 latency; a B stage is only held from its
+    // production to its MMA)
+    struct Cfg { int sa, sb; };
+    const Cfg cands[] = {{4, 4}, {4, 2}, {2, 2}};
+    Cfg pick{0, 0};
+    for (const Cfg& c : cands)
+        if (!pick.sa && fixed + (size_t)c.sa * tc::A_BYTES + (size_t)c.sb * tc::B_BYTES <= (size_t)optin) pick = c;
+    if (getenv("EPI4_STAGES")) {   // diagnostics: EPI4_STAGES=<sa><sb>, e.g. 43
+        const int v = atoi(getenv("EPI4_STAGES"));
+        pick = Cfg{v / 10, v % 10};
+    }
+    if (!pick.sa) return cudaErrorInvalidConfiguration;
+    const size_t smem = 1024 + (size_t)pick.sa * tc::A_BYTES + (size_t)pick.sb * tc::B_BYTES + topk_smem_bytes(sp.topk);
     if (getenv("EPI4_VERBOSE"))
-        fprintf(stderr, "k_quad_tc: %d producer warps, %d stages, filter %d, smem %zu B, grid %d\n", tc::PROD_WARPS, st,
-                sp.use_filter, smem, grid);
+        fprintf(stderr, "k_quad_tc: %d producer warps, A/B stages %d/%d, A split %d, filter %d, smem %zu B, grid %d\n",
+                tc::PROD_WARPS, pick.sa, pick.sb, tc::A_SPLIT, sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
-    auto go = [&](auto S) {
-        constexpr int v = decltype(S)::value;
-        if constexpr (v % tc::STAGE_Q == 0)
-            if (st == v) e = launch_cfg<v>(sp, smem, grid, s);
-    };
-    go(std::integral_constant<int, 2>{});
-    go(std::integral_constant<int, 3>{});
-    go(std::integral_constant<int, 4>{});
-    go(std::integral_constant<int, 6>{});
-    go(std::integral_constant<int, 8>{});
-    go(std::integral_constant<int, 9>{});
-    go(std::integral_constant<int, 10>{});
-    go(std::integral_constant<int, 12>{});
+    if (pick.sa == 4 && pick.sb == 4) e = launch_cfg<4, 4>(sp, smem, grid, s);
+    else if (pick.sa == 4 && pick.sb == 2) e = launch_cfg<4, 2>(sp, smem, grid, s);
+    else if (pick.sa == 2 && pick.sb == 2) e = launch_cfg<2, 2>(sp, smem, grid, s);
     if (launches) ++*launches;
     return e;
 }
