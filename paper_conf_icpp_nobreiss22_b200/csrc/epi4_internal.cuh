@@ -140,7 +140,8 @@ struct SearchParams {
     unsigned long long* prof;  // [16] diagnostics: [0] exact K2 evaluations, [1..] per-role cycle counters
     int32_t use_filter;        // fp32 Stirling K2 filter before the exact double K2 (epilogue.cuh)
 
-    int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA
+    int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA,
+                               // 128 no A copies (16: exact K2 for every quad, 64: trace)
 };
 
 }  // namespace epi4

@@ -63,7 +63,7 @@ constexpr int B_BYTES = CHUNKS * B_SUB;
 constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (10)
 constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per A stage
 #ifndef EPI4_A_SPLIT
-#define EPI4_A_SPLIT 4
+#define EPI4_A_SPLIT 1
 #endif
 constexpr int A_SPLIT = EPI4_A_SPLIT;    // lanes issuing one A stage's bulk copy in pieces (tools/probe_tma.cu: several
                                          // concurrently issued copies ingest faster than one)
@@ -513,6 +513,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 // copied as A_SPLIT pieces issued by as many lanes
                 const uint8_t* src = (st.p ? expl1 : expl0) +
                                      expl_off(2 * (int64_t)st.chunk(), (int64_t)(st.ti.wp * 2 + (int)rank) * 128, nrb);
+                if (sp.debug & 128) {             // diagnostics: no copy (the MMA reads stale operands)
+                    if (lane == 0) mbar_arrive_local(&afull_bar[sa]);
+                    __syncwarp();
+                    continue;
+                }
                 if (lane == 0) mbar_expect_tx(&afull_bar[sa], tc::TX_BYTES);
                 __syncwarp();
                 if (lane < tc::A_SPLIT) {
@@ -589,6 +594,14 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             if (lane == 0) TRACE(4, step);
+#if EPI4_PROF
+            {   // trace event 3: this step's singles have arrived (a value-dependent branch waits for the loads)
+                uint32_t dep = cx[0].x | cx[1].y | cx[2].z | cx[3].w;
+#pragma unroll
+                for (int k = 0; k < YK; ++k) dep |= cy[k].x;
+                if (lane == 0 && dep != 0x9E3779B9u) TRACE(3, step);
+            }
+#endif
             if (build) {
                 unsigned char* bdst = bring + sb * tc::B_BYTES + jc * tc::B_SUB;
                 const uint4 xz[4] = {and4(cx[0], cx[2]), and4(cx[0], cx[3]), and4(cx[1], cx[2]), and4(cx[1], cx[3])};
