@@ -128,9 +128,10 @@ typedef struct {
     int64_t launches_load; /* kernels launched by the last load                    */
     double executed_macs;  /* MACs issued by the last search's contraction (incl. padding/masking) */
     double prof[8];        /* diagnostics: [0] exact-K2 evaluations (filter candidates); with opts.reserved[0]
-                              & 8 also summed SM cycles: [1] epilogue busy, [2] epilogue waiting for the
-                              accumulators, [3] producer busy, [4] producer waiting for TMA data,
-                              [5] MMA waiting for operands, [6] TMA waiting for a free stage */
+                              & 8 (instrumented build, -DEPI4_PROF) also summed SM cycles: [1] epilogue busy,
+                              [2] MMA waiting for the A operand, [3] producer busy, [4] producer waiting for a
+                              free B stage, [5] MMA waiting for the B operand, [6] TMA waiting for a free A
+                              stage, [7] MMA waiting for a free TMEM region */
 } epi4_stats;
 
 int epi4_get_stats(epi4_ctx* ctx, epi4_stats* out);
