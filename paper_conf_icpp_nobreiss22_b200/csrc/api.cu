@@ -127,8 +127,11 @@ DevData devdata(const epi4_ctx* c) {
     d.nsteps[0] = (d.nchunks4[0] + 1) / 2;
     d.nsteps[1] = (d.nchunks4[1] + 1) / 2;
     d.nrb = c->npad / 64;
+    // c0 <= n0 < 2^pk_shift; 16 whenever both counts fit 16 bits (the epilogue then unpacks each half into a
+    // float with one byte permute, epilogue.cuh cell_T<true>)
     d.pk_shift = 1;
-    while (d.pk_shift < 31 && ((int64_t)1 << d.pk_shift) <= c->np[0]) ++d.pk_shift;   // c0 <= n0 < 2^pk_shift
+    while (d.pk_shift < 31 && ((int64_t)1 << d.pk_shift) <= c->np[0]) ++d.pk_shift;
+    if (c->np[0] < 65536 && c->np[1] < 65536) d.pk_shift = 16;
     d.n = c->n;
     d.npad = c->npad;
     d.np[0] = (uint32_t)c->np[0];

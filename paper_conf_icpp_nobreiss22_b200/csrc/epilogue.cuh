@@ -139,15 +139,19 @@ __device__ __forceinline__ void mobius3(uint32_t (&g)[27]) {
 // K2 - (ln2 sum T_c - 81 - 81 C0) lies in (-13.5, 3.375).  With the fp32 rounding bound E(M) computed on the
 // host (api.cu: filter_offset), K2 > ln2 A - 81 - 81 C0 - 13.5 - E for the computed A = sum T_c, so a quad is
 // scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
-// is exactly the oracle's.  Per cell: 3 ALU (unpack), 6 FADD + FMUL + 2 FFMA + 1 FADD, 3 MUFU; no table and
-// no conversion instruction (a count r < 2^22 becomes the float 2^23 + r by an OR of the exponent bits).
+// is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + FMUL + 2 FFMA + 1 FADD, 3 MUFU;
+// no table and no conversion instruction (a count r < 2^22 becomes the float 2^23 + r by setting the exponent
+// bits).
 __device__ __forceinline__ float lg2_approx(float x) {
     float y;
     asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
 }
+template <bool PK16>
 __device__ __forceinline__ float cell_T(uint32_t v, uint32_t pks, uint32_t pkm) {
-    const float m0 = __uint_as_float((v & pkm) | 0x4B000000u), m1 = __uint_as_float((v >> pks) | 0x4B000000u);
+    // 2^23 + r0, 2^23 + r1 (with pks = 16 one byte permute each: [r.lo, r.hi, 0x00, 0x4B])
+    const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
+    const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
     const float f0 = m0 - 8388607.0f, f1 = m1 - 8388607.0f;     // r + 1
     const float h0 = m0 - 8388607.5f, h1 = m1 - 8388607.5f;     // r + 1/2
     const float fn = f0 + f1, hn = h0 + f1;                     // n + 2, n + 3/2
@@ -163,7 +167,7 @@ __device__ __forceinline__ float cell_T(uint32_t v, uint32_t pks, uint32_t pkm) 
 // MODE 0: the fp32 filter value A = sum T_c (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
 // L[r_c0]) - L[r_c1], K2 += t_c, c = 0..80 (reading #4); MODE 2: exact K2 and the
 // 2 x 81 cells written to dump (controls first).
-template <int MODE>
+template <int MODE, bool PK16 = false>
 __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, int w, int x, int y, int z,
                                           const uint32_t (&c16)[16], float& flt, double& k2, uint32_t* dump) {
     const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
@@ -181,7 +185,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
-                const float t = cell_T(S[c], pks, pkm);
+                const float t = cell_T<PK16>(S[c], pks, pkm);
                 if (c & 1) fb += t; else fa += t;
             } else {
                 const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;

@@ -335,7 +335,7 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 // issuers may issue (and complete) the steps of the other parity out of order, so a waiter is only protected
 // from phase aliasing if its previous wait on a ring was on the same issuer's steps: both ring sizes must be
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
-template <int SA, int SB>
+template <int SA, int SB, bool PK16>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     static_assert(SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2,
                   "ring sizes must be multiples of the alternating warps' stride (phase aliasing)");
@@ -733,7 +733,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         // fp32 Stirling filter (epilogue.cuh); only possible top-k members get the exact K2
                         float flt;
                         double unused;
-                        quad_eval<0>(d, quad_ranks(w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt, unused, nullptr);
+                        quad_eval<0, PK16>(d, quad_ranks(w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt, unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
                         offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
@@ -785,9 +785,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 #endif
 }
 
-template <int SA, int SB>
+template <int SA, int SB, bool PK16>
 static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
-    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
@@ -801,7 +801,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB>, sp);
+    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16>, sp);
 }
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
@@ -833,9 +833,10 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
         fprintf(stderr, "k_quad_tc: %d producer warps, A/B stages %d/%d, A split %d, filter %d, smem %zu B, grid %d\n",
                 tc::PROD_WARPS, pick.sa, pick.sb, tc::A_SPLIT, sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
-    if (pick.sa == 4 && pick.sb == 4) e = launch_cfg<4, 4>(sp, smem, grid, s);
-    else if (pick.sa == 4 && pick.sb == 2) e = launch_cfg<4, 2>(sp, smem, grid, s);
-    else if (pick.sa == 2 && pick.sb == 2) e = launch_cfg<2, 2>(sp, smem, grid, s);
+    const bool pk16 = sp.d.pk_shift == 16;
+    if (pick.sa == 4 && pick.sb == 4) e = pk16 ? launch_cfg<4, 4, true>(sp, smem, grid, s) : launch_cfg<4, 4, false>(sp, smem, grid, s);
+    else if (pick.sa == 4 && pick.sb == 2) e = pk16 ? launch_cfg<4, 2, true>(sp, smem, grid, s) : launch_cfg<4, 2, false>(sp, smem, grid, s);
+    else if (pick.sa == 2 && pick.sb == 2) e = pk16 ? launch_cfg<2, 2, true>(sp, smem, grid, s) : launch_cfg<2, 2, false>(sp, smem, grid, s);
     if (launches) ++*launches;
     return e;
 }
