@@ -81,6 +81,8 @@ struct epi4_ctx {
     Unit* d_units = nullptr;
     int64_t* d_prefix = nullptr;
     size_t units_cap = 0;
+    uint64_t* d_tiles = nullptr;   // tensor-core pipe: decoded tile table (k_tile_table), 8 B per tile
+    size_t cap_tiles = 0;
     unsigned long long* d_counters = nullptr;   // [0] tile counter, [1] quads done
     double* d_list_k2 = nullptr;
     uint64_t* d_list_idx = nullptr;
@@ -358,6 +360,7 @@ void epi4_destroy(epi4_ctx* c) {
     release_data(c);
     dfree(c->d_units);
     dfree(c->d_prefix);
+    dfree(c->d_tiles);
     dfree(c->d_counters);
     dfree(c->d_list_k2);
     dfree(c->d_list_idx);
@@ -555,6 +558,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.d = devdata(c);
     sp.units = c->d_units;
     sp.prefix = c->d_prefix;
+    sp.tile_info = nullptr;
     sp.nunits = nu;
     sp.ntiles = acc;
     sp.tile_counter = c->d_counters;
@@ -570,6 +574,11 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.use_filter = !(sp.debug & 16);   // debug 16: exact K2 for every quad (no filter)
 
     c->stats.launches = 0;
+    if (c->opts.pipe != EPI4_PIPE_LOP3 && acc > 0) {
+        CU(grow(c->d_tiles, c->cap_tiles, (size_t)acc * sizeof(uint64_t)));
+        sp.tile_info = c->d_tiles;
+        CU(launch_tile_table(sp, c->d_tiles, c->stream, &c->stats.launches));
+    }
     CU(cudaEventRecord(c->ev[2], c->stream));
     if (acc > 0) {
         cudaError_t e = c->opts.pipe == EPI4_PIPE_LOP3 ? launch_quad_lop3(sp, grid, c->stream, &c->stats.launches)

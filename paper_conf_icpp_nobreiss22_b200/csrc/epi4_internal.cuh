@@ -127,6 +127,7 @@ struct SearchParams {
     DevData d;
     const Unit* units;
     const int64_t* prefix;     // inclusive prefix of tiles per unit
+    const uint64_t* tile_info; // (tensor-core pipe) decoded tiles: wp | x << 16 | y0 << 32 | z << 48 (k_tile_table)
     int64_t nunits;
     int64_t ntiles;
     unsigned long long* tile_counter;   // dynamic scheduler
@@ -162,6 +163,7 @@ cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T
                        int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
+cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches);
 int32_t quad_split(int32_t pipe);   // tiles per unit tile (CUDA-core kernel: the two 64-SNP halves)
 int32_t quad_yr(int32_t pipe);      // y-range of a tile
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,

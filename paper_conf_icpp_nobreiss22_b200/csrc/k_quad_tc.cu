@@ -280,6 +280,32 @@ __device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t 
     return ti;
 }
 
+// The tile table (one uint64 per tile, filled by k_tile_table before the search): a tile change in the hot
+// kernel costs one load instead of decode_tile's binary search over the unit prefix (~log2(units) dependent
+// global loads) and the y-range loop, which stalled the TMA / producer / epilogue warps at every tile change.
+__global__ void __launch_bounds__(256) k_tile_table(SearchParams sp, uint64_t* __restrict__ out) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= sp.ntiles) return;
+    const TileInfo ti = decode_tile(sp, t);
+    out[t] = (uint64_t)(uint16_t)ti.wp | ((uint64_t)(uint16_t)ti.x << 16) | ((uint64_t)(uint16_t)ti.y0 << 32) |
+             ((uint64_t)(uint16_t)ti.z << 48);
+}
+cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches) {
+    if (sp.ntiles <= 0) return cudaSuccess;
+    k_tile_table<<<(unsigned)((sp.ntiles + 255) / 256), 256, 0, s>>>(sp, out);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+__device__ __forceinline__ TileInfo load_tile(const SearchParams& sp, int64_t tile) {
+    const uint64_t v = __ldg(sp.tile_info + tile);
+    TileInfo ti;
+    ti.wp = (int32_t)(v & 0xFFFF);
+    ti.x = (int32_t)((v >> 16) & 0xFFFF);
+    ti.y0 = (int32_t)((v >> 32) & 0xFFFF);
+    ti.z = (int32_t)(v >> 48);
+    return ti;
+}
+
 // iterator over the (tile, phenotype, chunk) steps of this cluster; advance(k) moves k steps ahead.
 // Chunk counts live in registers (runtime indexing of kernel-parameter arrays spills the parameter block).
 struct StepIt {
@@ -293,7 +319,7 @@ struct StepIt {
         kc = 0;
         nch0 = sp.d.nsteps[0];
         nch1 = sp.d.nsteps[1];
-        if (tile < sp.ntiles) ti = decode_tile(sp, tile);
+        if (tile < sp.ntiles) ti = load_tile(sp, tile);
     }
     __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
     // physical chunk of this step (a tile-dependent rotation of the K loop was measured slower: r01 notes)
@@ -309,7 +335,7 @@ struct StepIt {
                 tile += nclusters_x();
             }
         }
-        if (tile != t0 && tile < sp.ntiles) ti = decode_tile(sp, tile);
+        if (tile != t0 && tile < sp.ntiles) ti = load_tile(sp, tile);
     }
 };
 
@@ -659,7 +685,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         const uint32_t pks = (uint32_t)d.pk_shift;
         int r0 = 0;                                     // the MMA issuers' region rotation
         for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
-            const TileInfo ti = decode_tile(sp, tile);
+            const TileInfo ti = load_tile(sp, tile);
             const int buf = it & 1;
             const uint32_t tphase = (uint32_t)((it >> 1) & 1);
             const int r1 = r0 == 2 ? 0 : r0 + 1;
