@@ -73,6 +73,10 @@ constexpr int A_SPLIT = EPI4_A_SPLIT;    // lanes issuing one A stage's bulk cop
 constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
 static_assert(PROD_WARPS % CHUNKS == 0, "producer warps come in groups of CHUNKS (one chunk of a step each)");
 constexpr int PROD_STRIDE = PROD_WARPS / CHUNKS;          // steps between two steps of one producer warp
+#ifndef EPI4_MMA_ISSUERS
+#define EPI4_MMA_ISSUERS 2
+#endif
+constexpr int MMA_ISSUERS = EPI4_MMA_ISSUERS;   // 1: one issuer, MMAs complete in step order (any ring sizes)
 constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate steps (one thread cannot hide
                                          // its own wait/bookkeeping latency behind the blocking MMA issue)
 constexpr int TMA_WARPS = 2;             // a bulk-copy issue blocks its thread ~150-200 cycles: two warps alternate
@@ -363,7 +367,8 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
 template <int SA, int SB, bool PK16>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
-    static_assert(SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2,
+    static_assert(tc::MMA_ISSUERS == 1 ||
+                  (SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2),
                   "ring sizes must be multiples of the alternating warps' stride (phase aliasing)");
     extern __shared__ unsigned char smem_raw[];
     // A ring: afull (own TMA landed), apeer (@leader: the follower's A landed, relayed), aempty (MMA commit);
@@ -398,7 +403,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             mbar_init(&bempty_bar[s], 1);                 // the leader's MMA commit
         }
         for (int b = 0; b < 2; ++b) {
-            mbar_init(&tfull_bar[b], tc::MMA_WARPS);      // each issuer's commit after its last step
+            mbar_init(&tfull_bar[b], tc::MMA_ISSUERS);    // each issuer's commit after its last step
             mbar_init(&ep_bar[b], tc::CLUSTER * tc::EPI_WARPS);   // (leader) every epilogue warp of the pair
         }
         mbar_init(&pk_bar, tc::CLUSTER * tc::EPI_WARPS);
@@ -449,7 +454,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         // control flow keeps the descriptors in uniform registers); one elected lane issues.  Descriptors are
         // precomputed once: per MMA only a 64-bit add (tools/probe_mma3.cu).  Every MMA accumulates (the
         // epilogue re-zeroes the accumulators), so the two issuers' MMAs commute.
-        if (leader) {
+        if (leader && rw < tc::MMA_ISSUERS) {
             const int m = rw;
             const uint32_t ring_s = smem_u32(ring), bring_s = smem_u32(bring);
             const uint64_t adesc0 = sw128_desc(ring_s), bdesc0 = sw128_desc(bring_s);
@@ -477,7 +482,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     const int nch = p ? nch1_r : nch0_r;
 #pragma unroll 1
                     for (int kc = 0; kc < nch; ++kc, ++gstep) {
-                        if ((gstep & (tc::MMA_WARPS - 1)) != m) continue;
+                        if ((gstep & (tc::MMA_ISSUERS - 1)) != m) continue;
                         const int sa = gstep % SA, sb = gstep % SB;
                         const uint32_t pa = (uint32_t)((gstep / SA) & 1), pb = (uint32_t)((gstep / SB) & 1);
                         const long long t0 = PCLK();
@@ -845,7 +850,7 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     // deepest rings that fit (the A copies carry the long L2 latency; a B stage is only held from its
     // production to its MMA)
     struct Cfg { int sa, sb; };
-    const Cfg cands[] = {{4, 4}, {4, 2}, {2, 2}};
+    const Cfg cands[] = {{tc::MMA_ISSUERS == 1 ? 5 : 4, tc::MMA_ISSUERS == 1 ? 3 : 4}, {4, 4}, {4, 2}, {2, 2}};
     Cfg pick{0, 0};
     for (const Cfg& c : cands)
         if (!pick.sa && fixed + (size_t)c.sa * tc::A_BYTES + (size_t)c.sb * tc::B_BYTES <= (size_t)optin) pick = c;
@@ -860,7 +865,10 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
                 tc::PROD_WARPS, pick.sa, pick.sb, tc::A_SPLIT, sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
     const bool pk16 = sp.d.pk_shift == 16;
-    if (pick.sa == 4 && pick.sb == 4) e = pk16 ? launch_cfg<4, 4, true>(sp, smem, grid, s) : launch_cfg<4, 4, false>(sp, smem, grid, s);
+    if (pick.sa == 5 && pick.sb == 3) {
+        if constexpr (tc::MMA_ISSUERS == 1)
+            e = pk16 ? launch_cfg<5, 3, true>(sp, smem, grid, s) : launch_cfg<5, 3, false>(sp, smem, grid, s);
+    } else if (pick.sa == 4 && pick.sb == 4) e = pk16 ? launch_cfg<4, 4, true>(sp, smem, grid, s) : launch_cfg<4, 4, false>(sp, smem, grid, s);
     else if (pick.sa == 4 && pick.sb == 2) e = pk16 ? launch_cfg<4, 2, true>(sp, smem, grid, s) : launch_cfg<4, 2, false>(sp, smem, grid, s);
     else if (pick.sa == 2 && pick.sb == 2) e = pk16 ? launch_cfg<2, 2, true>(sp, smem, grid, s) : launch_cfg<2, 2, false>(sp, smem, grid, s);
     if (launches) ++*launches;
