@@ -25,7 +25,9 @@
 #define EPI4_WR 64            // w-range of one CTA / rows of its A operand: 64 SNPs x {AA, Aa}
 #define EPI4_WP 128           // w-range of a work unit (a CTA pair: two 64-SNP halves)
 #define EPI4_YR 16            // y-range of a CUDA-core (LOP3) tile: 16 consecutive SNPs after x
-#define EPI4_YR_TC 20         // y-range of a tensor-core tile (N = 160 = 20 x 8 columns; TMEM budget, k_quad_tc.cu)
+#ifndef EPI4_YR_TC
+#define EPI4_YR_TC 16         // y-range of a tensor-core tile (N = 128 = 16 x 8 columns; measured best, k_quad_tc.cu)
+#endif
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
 
@@ -85,7 +87,7 @@ __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, 
 
 // A work unit (wp, x): the quads (w, x, y, z) with w in the 128-SNP range [128 wp, 128 wp + 128), w < x,
 // second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + yr) with y0 = x + 1 + yr k,
-// and z in (y0, n); a tile holds 128 x yr (w, y) combinations (yr = 14 tensor core, 16 CUDA core), split into
+// and z in (y0, n); a tile holds 128 x yr (w, y) combinations (yr = EPI4_YR_TC tensor core, EPI4_YR CUDA core), split into
 // the two 64-SNP halves of the w-range (the two CTAs of a tensor-core cluster, or two tiles of the CUDA-core
 // kernel).
 struct Unit {

@@ -3,10 +3,10 @@
 // epilogue.
 //
 // What it computes: for a tile (w-range pair wp, x, y-range y0, z) and each
-// phenotype p the 256 x 160 matrix
+// phenotype p the 256 x N matrix (N = 8 YR, YR = EPI4_YR_TC = 16 y per tile, N = 128)
 //     C_p[(w, a)][(y, b, c, d)] = sum over samples s of phenotype p of P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]
-// for the 128 SNPs w of the range pair and the 20 SNPs y = y0..y0+19: the 16 non-aa genotype counts of the
-// 128 x 20 quads (w, x, y, z) ("a matrix with 16 values per each quad").
+// for the 128 SNPs w of the range pair and the YR SNPs y = y0..y0+YR-1: the 16 non-aa genotype counts of the
+// 128 x YR quads (w, x, y, z) ("a matrix with 16 values per each quad").
 // Factorisation: the paper ANDs SNP pairs into both operands (combine);
 // here the A operand is the raw single-SNP planes (w, a), copied from HBM by the TMA engine, and x is folded
 // into the B operand, whose columns are triple products P_b(x) & P_c(y) & P_d(z) built on chip.
@@ -14,21 +14,22 @@
 // legacy IMMA).  A set bit is the E2M1 value 1.0 (nibble 0x2), so AND of packed nibbles
 // is the product, and with all E8M0 block scales = 1 the MMA sums exact small integers: the fp32 accumulator
 // is exact up to 2^24 per phenotype (host check; tools/probe_mxf4.cu: 0 mismatches, counts to 76800).
-// kind::mxf4 runs M=256 N=160 K=64 in 80 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the
-// operand bytes (2 samples per byte).
+// kind::mxf4 runs M=256 K=64 in N/2 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the operand
+// bytes (2 samples per byte).
 // Why 2-CTA: a 1-CTA M=128 MMA issues every ~97 cycles whatever N; cta_group::2 reaches the full rate.
-// Why N = 160: the A operand is streamed from L2 once per (tile, sample chunk), i.e. 128 B per row and 256
-// samples for every N columns; at N = 112 a full-rate MMA needs 73 B/clk/SM of A, the whole TMA ingest an SM
-// gets from L2 (tools/probe_tma3.cu: ~75 B/clk/SM with 32 KiB copies); N = 160 needs 51.  TMEM holds three
-// regions of 160 fp32 columns plus the scale factors; tile t accumulates its controls in region (-t) mod 3 and
-// its cases in the next one.  When the tile is done the epilogue first packs every (control, case) pair into
-// one 32-bit word in the case region and zeroes the control region (pass 1, a few hundred cycles), which the
-// case accumulation of tile t+1 reuses; it then scores the quads from the packed region (pass 2), which the
-// control accumulation of tile t+2 reuses.  Two buffers of 2 x 160 columns would not fit in 512.
+// Why N = 128: the A operand is streamed from L2 once per (tile, sample chunk), 128 B per row and 256 samples
+// for every N columns (N = 128 needs 64 B/clk/SM of A at the full MMA rate, below the ~75 B/clk/SM an SM
+// ingests with 32 KiB copies, tools/probe_tma3.cu); N = 160 (20 y) and 96 (12 y) were measured 3 % and 9 %
+// slower at C2 and equal at C5.  TMEM holds three regions of N fp32 columns plus the scale
+// factors; tile t accumulates its controls in region (-t) mod 3 and its cases in the next one.  When the tile
+// is done the epilogue first packs every (control, case) pair into one 32-bit word in the case region and
+// zeroes the control region (pass 1, a few hundred cycles), which the case accumulation of tile t+1 reuses;
+// it then scores the quads from the packed region (pass 2), which the control accumulation of tile t+2
+// reuses (two buffers of 2 x N columns would not fit in 512 at N = 160).
 //
 // CTA pair (cluster of 2): CTA r holds the A rows of w-range 2wp + r (64 SNPs x {AA, Aa}) and builds the
-// B columns of y = y0 + 10r .. y0 + 10r + 9; the leader (r = 0) issues the MMAs for both; each CTA's TMEM
-// receives its 128 rows x all 160 columns and its epilogue scores its 64 x 20 quads.
+// B columns of y = y0 + r YR/2 .. y0 + (r + 1) YR/2 - 1; the leader (r = 0) issues the MMAs for both; each
+// CTA's TMEM receives its 128 rows x all N columns and its epilogue scores its 64 x YR quads.
 // Warp roles (each CTA: 16 warps = 4 warpgroups with setmaxnreg budgets, 1 CTA per SM, persistent, static
 // tile stride over clusters):
 //   warps 0..1  : leader — MMA issuers (alternating steps, one elected lane each); follower — warp 0 relays
@@ -57,10 +58,10 @@ constexpr int ROWB = 128;                // bytes of one K-major operand row per
 constexpr int CHUNKS = 2;                // fp4 chunks per pipeline stage (512 samples): one 32 KiB A copy
 constexpr int A_SUB = 128 * ROWB;        // this CTA's 128 A rows of one chunk (16 KiB)
 constexpr int A_BYTES = CHUNKS * A_SUB;
-constexpr int B_ROWS = N / 2;            // this CTA's 80 B columns
+constexpr int B_ROWS = N / 2;            // this CTA's B columns (64)
 constexpr int B_SUB = (B_ROWS + 7) / 8 * 1024;
 constexpr int B_BYTES = CHUNKS * B_SUB;
-constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (10)
+constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (8)
 constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per A stage
 #ifndef EPI4_A_SPLIT
 #define EPI4_A_SPLIT 1
@@ -105,7 +106,7 @@ constexpr int REGIONS = 3;               // accumulator regions of N columns, ro
 constexpr int ACC_COLS = REGIONS * N;
 constexpr int SF_COL = 480;              // scale factors (all E8M0 0x7F = 1.0): columns 480..511, every lane
 static_assert(ACC_COLS <= SF_COL, "TMEM: accumulators overlap the scale factors");
-constexpr int NG = N / 16;               // 16-column groups of an accumulator (7)
+constexpr int NG = N / 16;               // 16-column groups of an accumulator (8)
 constexpr int CLUSTER = 2;
 // block-scaled instruction descriptor: A/B E2M1 (format 1 at bits 7 and 10), K-major, N>>3 at bit 17,
 // scale format E8M0 (bit 23), M>>4 at bit 24, scale-factor ids 0, K = 64 (bit 31 = 0)
@@ -850,7 +851,7 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     // deepest rings that fit (the A copies carry the long L2 latency; a B stage is only held from its
     // production to its MMA)
     struct Cfg { int sa, sb; };
-    const Cfg cands[] = {{tc::MMA_ISSUERS == 1 ? 5 : 4, tc::MMA_ISSUERS == 1 ? 3 : 4}, {4, 4}, {4, 2}, {2, 2}};
+    const Cfg cands[] = {{tc::MMA_ISSUERS == 1 ? 5 : 4, tc::MMA_ISSUERS == 1 ? 3 : 4}, {6, 2}, {4, 4}, {4, 2}, {2, 2}};
     Cfg pick{0, 0};
     for (const Cfg& c : cands)
         if (!pick.sa && fixed + (size_t)c.sa * tc::A_BYTES + (size_t)c.sb * tc::B_BYTES <= (size_t)optin) pick = c;
@@ -868,6 +869,10 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     if (pick.sa == 5 && pick.sb == 3) {
         if constexpr (tc::MMA_ISSUERS == 1)
             e = pk16 ? launch_cfg<5, 3, true>(sp, smem, grid, s) : launch_cfg<5, 3, false>(sp, smem, grid, s);
+    } else if (pick.sa == 4 && pick.sb == 6) {
+        e = pk16 ? launch_cfg<4, 6, true>(sp, smem, grid, s) : launch_cfg<4, 6, false>(sp, smem, grid, s);
+    } else if (pick.sa == 6 && pick.sb == 2) {
+        e = pk16 ? launch_cfg<6, 2, true>(sp, smem, grid, s) : launch_cfg<6, 2, false>(sp, smem, grid, s);
     } else if (pick.sa == 4 && pick.sb == 4) e = pk16 ? launch_cfg<4, 4, true>(sp, smem, grid, s) : launch_cfg<4, 4, false>(sp, smem, grid, s);
     else if (pick.sa == 4 && pick.sb == 2) e = pk16 ? launch_cfg<4, 2, true>(sp, smem, grid, s) : launch_cfg<4, 2, false>(sp, smem, grid, s);
     else if (pick.sa == 2 && pick.sb == 2) e = pk16 ? launch_cfg<2, 2, true>(sp, smem, grid, s) : launch_cfg<2, 2, false>(sp, smem, grid, s);
