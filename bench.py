@@ -136,7 +136,10 @@ def run_ours(args):
     d = datagen.make_config(args.config)
     n, m = d.n_snps, d.n_samples
     stream = torch.cuda.Stream()
-    eng = epi.Epi4(local, pipe=args.pipe, rank=rank, world=world)
+    # N > 1: each rank builds 1/world of the 3-way table and the shares are all-gathered over NCCL (the
+    # exchange that replaces building T3 on every GPU); --no-shard-t3 builds it everywhere instead
+    shard = world > 1 and not args.no_shard_t3
+    eng = epi.Epi4(local, pipe=args.pipe, rank=rank, world=world, shard_t3=shard)
     eng.set_stream(stream.cuda_stream)
     geno_d = torch.from_numpy(d.geno).to(f"cuda:{local}")
     phen_d = torch.from_numpy(d.phen).to(f"cuda:{local}")
@@ -154,6 +157,8 @@ def run_ours(args):
                                             epi.binding.EPI4_PTR_HOST)
         else:
             eng.load_genotypes(geno_d, phen_d)
+        if shard:
+            eng.gather_t3()
         if world > 1:
             return epi.search_distributed(local_search, top_k)
         return eng.search(top_k)
@@ -222,7 +227,7 @@ def run_ours(args):
         "data": "synthetic (seeded HWE genotypes + planted 4-way interaction, SURVEY.md §8(d))",
         "config": {"workload": f"{args.config}: N={n} SNPs, M={m} samples ({d.n_controls} controls / "
                                f"{d.n_cases} cases), exhaustive C(N,4)={comb4(n)} quads, top_k={top_k}",
-                   "pipe": args.pipe, "parallelism": f"static LPT over (w-block, x) units x {world}",
+                   "pipe": args.pipe, "parallelism": f"static LPT over (w-block, x) units x {world}" + (", T3 sharded + NCCL all_gather" if shard else ""),
                    "l2": "flushed (512 MiB write) before every timed step"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": int(n * m + m),
                 "d2h_bytes_per_step": int(top_k * 16 + 4)},
@@ -289,6 +294,7 @@ def main():
     ap.add_argument("--pipe", default="tc", choices=["tc", "lop3"])
     ap.add_argument("--top-k", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-shard-t3", action="store_true", help="N > 1: build the whole 3-way table on every rank")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

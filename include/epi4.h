@@ -50,8 +50,16 @@ typedef struct {
     int32_t rank;     /* this process' rank and the world size: epi4_search evaluates only the     */
     int32_t world;    /*   work units the static LPT plan assigns to `rank`       */
     int32_t grid;     /* persistent-kernel CTAs (0 = 2 x number of SMs)                             */
-    int32_t reserved[3];
+    int32_t debug;    /* diagnostics only, 0 in production (debug modes disable warp roles; results  */
+                      /*   invalid except bit 16 = exact K2 for every quad, no filter)               */
+    int32_t flags;    /* EPI4_FLAG_* bits                                                          */
+    int32_t reserved;
 } epi4_opts;
+
+/* opts.flags: with world > 1, a load computes only this rank's contiguous share of the 3-way table T3
+ * (the triples [rank*S, (rank+1)*S) of the colex order, S = ceil(C(N,3) / world)); the caller all-gathers
+ * the shares (epi4_t3_shard / epi4_t3_ready) — the exchange that replaces building T3 on every GPU. */
+#define EPI4_FLAG_SHARD_T3 1
 
 /* Fill *opts with defaults (block 32, pipe TC, rank 0, world 1, grid 0). */
 void epi4_default_opts(epi4_opts* opts);
@@ -103,6 +111,16 @@ int epi4_search_units(epi4_ctx* ctx, int64_t unit_begin, int64_t unit_end, int32
  * n * 162 entries. */
 int epi4_tables(epi4_ctx* ctx, const uint64_t* quads, int64_t n, uint32_t* counts_out);
 
+/* Sharded T3 (opts.flags & EPI4_FLAG_SHARD_T3, world > 1, PAPER.md:L155 builds the tables on
+ * every GPU instead).  After a load, *t3_dev receives the device address of the packed T3 buffer (the
+ * context owns it), *shard_bytes the size of one rank's share and *total_bytes = world * shard_bytes; this
+ * rank's share is already computed at offset rank * shard_bytes.  The caller fills the other shares (an
+ * all-gather of equal-size chunks, e.g. NCCL over NVLink) on any stream, synchronizes, and calls
+ * epi4_t3_ready.  Until then epi4_search / epi4_tables fail with EPI4_ESTATE.  Without the flag the tables
+ * are complete after the load and both calls return EPI4_ESTATE. */
+int epi4_t3_shard(epi4_ctx* ctx, void** t3_dev, int64_t* shard_bytes, int64_t* total_bytes);
+int epi4_t3_ready(epi4_ctx* ctx);
+
 /* Debug/verification: make the next search also write the 162 counts of EVERY evaluated quad into
  * a device buffer indexed by the quad's colex rank C(l,4)+C(k,3)+C(j,2)+i (162 uint32 each);
  * counts_dev = NULL disables.  Only for small N (the buffer has C(N,4)*162 entries). */
@@ -127,7 +145,7 @@ typedef struct {
     int64_t launches;      /* kernels launched by the last search                  */
     int64_t launches_load; /* kernels launched by the last load                    */
     double executed_macs;  /* MACs issued by the last search's contraction (incl. padding/masking) */
-    double prof[8];        /* diagnostics: [0] exact-K2 evaluations (filter candidates); with opts.reserved[0]
+    double prof[8];        /* diagnostics: [0] exact-K2 evaluations (filter candidates); with opts.debug
                               & 8 (instrumented build, -DEPI4_PROF) also summed SM cycles: [1] epilogue busy,
                               [2] MMA waiting for the A operand, [3] producer busy, [4] producer waiting for a
                               free B stage, [5] MMA waiting for the B operand, [6] TMA waiting for a free A

@@ -12,7 +12,7 @@ import numpy as np
 from . import binding
 from .binding import Epi4Error, epi4_last_error, epi4_version  # noqa: F401
 
-__all__ = ["Epi4", "merge_topk", "search_distributed", "pack_index", "unpack_index", "binding", "Epi4Error"]
+__all__ = ["Epi4", "merge_topk", "search_distributed", "allgather_shares", "pack_index", "unpack_index", "binding", "Epi4Error"]
 
 
 def pack_index(i, j, k, l) -> int:
@@ -29,11 +29,13 @@ class Epi4:
     """One search context on one GPU (one per rank)."""
 
     def __init__(self, device: int = 0, pipe: str = "tc", rank: int = 0, world: int = 1, grid: int = 0,
-                 debug: int = 0):
+                 debug: int = 0, shard_t3: bool = False):
         o = binding.epi4_default_opts()
         o.pipe = binding.PIPES[pipe]
         o.rank, o.world, o.grid = int(rank), int(world), int(grid)
-        o.reserved[0] = int(debug)     # diagnostics only: disables warp roles, results invalid
+        o.debug = int(debug)           # diagnostics only: disables warp roles, results invalid
+        o.flags = binding.EPI4_FLAG_SHARD_T3 if shard_t3 else 0
+        self.shard_t3 = bool(shard_t3) and int(world) > 1
         self.pipe, self.rank, self.world = pipe, int(rank), int(world)
         self.ctx = binding.epi4_create(device, o)
 
@@ -71,11 +73,44 @@ class Epi4:
     def search_units(self, unit_begin: int, unit_end: int, top_k: int = 1):
         return binding.epi4_search_units(self.ctx, unit_begin, unit_end, top_k)
 
+    def t3_device_view(self):
+        """(full uint8 device tensor over the packed T3 buffer, share size in bytes) — sharded T3 only."""
+        import torch
+        ptr, shard, total = binding.epi4_t3_shard(self.ctx)
+        return torch.as_tensor(_CudaBuffer(ptr, total), device="cuda"), shard
+
+    def gather_t3(self, group=None, stream=None):
+        """Sharded T3: all-gather the ranks' equal-size shares of the 3-way table over
+        torch.distributed (NCCL over NVLink on GPUs), then release the context for searching."""
+        import torch
+        full, shard = self.t3_device_view()
+        allgather_shares(full, shard, group)
+        torch.cuda.current_stream().synchronize()
+        binding.epi4_t3_ready(self.ctx)
+
     def tables(self, quads):
         return binding.epi4_tables(self.ctx, quads)
 
     def stats(self) -> dict:
         return binding.epi4_get_stats(self.ctx)
+
+
+class _CudaBuffer:
+    """A raw device allocation exposed through __cuda_array_interface__ (uint8), for torch.as_tensor."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (int(nbytes),), "typestr": "|u1", "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
+def allgather_shares(full, shard: int, group=None):
+    """In-place assembly of equal-size shares: rank r's bytes live in full[r*shard:(r+1)*shard]; after the
+    call every rank holds all of them (one all_gather of `shard` bytes per rank; NCCL or gloo)."""
+    import torch.distributed as dist
+    r = dist.get_rank(group)
+    mine = full[r * shard:(r + 1) * shard].clone()
+    dist.all_gather_into_tensor(full, mine, group=group)
+    return full
 
 
 def merge_topk(parts, top_k: int):

@@ -20,6 +20,7 @@ HEADER = os.path.join(os.path.dirname(HERE), "include", "epi4.h")
 EPI4_OK, EPI4_EINVAL, EPI4_ENOMEM, EPI4_ECUDA, EPI4_ESTATE, EPI4_ENODEV = 0, -1, -2, -3, -4, -5
 EPI4_PIPE_TC, EPI4_PIPE_LOP3 = 0, 1
 EPI4_PTR_HOST, EPI4_PTR_DEVICE = 0, 1
+EPI4_FLAG_SHARD_T3 = 1
 EPI4_MAX_TOPK = 1024
 PIPES = {"tc": EPI4_PIPE_TC, "lop3": EPI4_PIPE_LOP3}
 
@@ -32,7 +33,8 @@ class Epi4Error(RuntimeError):
 
 class epi4_opts(ctypes.Structure):
     _fields_ = [("block", ctypes.c_int32), ("pipe", ctypes.c_int32), ("rank", ctypes.c_int32),
-                ("world", ctypes.c_int32), ("grid", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
+                ("world", ctypes.c_int32), ("grid", ctypes.c_int32), ("debug", ctypes.c_int32),
+                ("flags", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class epi4_stats(ctypes.Structure):
@@ -64,6 +66,8 @@ def _load():
         "epi4_search_units": (ctypes.c_int, [P, I64, I64, I32, P, P, P]),
         "epi4_tables": (ctypes.c_int, [P, P, I64, P]),
         "epi4_set_dump": (ctypes.c_int, [P, P]),
+        "epi4_t3_shard": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(I64), ctypes.POINTER(I64)]),
+        "epi4_t3_ready": (ctypes.c_int, [P]),
         "epi4_plan_count": (I64, [I32, I32, I32]),
         "epi4_plan_units": (ctypes.c_int, [I32, I32, I32, P, P]),
         "epi4_get_stats": (ctypes.c_int, [P, ctypes.POINTER(epi4_stats)]),
@@ -170,6 +174,17 @@ def epi4_tables(ctx, quads) -> np.ndarray:
     out = np.zeros((q.size, 2, 81), dtype=np.uint32)
     _check(_lib.epi4_tables(ctx, _ptr(q), q.size, _ptr(out)))
     return out
+
+
+def epi4_t3_shard(ctx):
+    """(device address of the packed T3 buffer, bytes of one rank's share, total bytes)."""
+    p, sb, tb = ctypes.c_void_p(), ctypes.c_int64(), ctypes.c_int64()
+    _check(_lib.epi4_t3_shard(ctx, ctypes.byref(p), ctypes.byref(sb), ctypes.byref(tb)))
+    return int(p.value or 0), int(sb.value), int(tb.value)
+
+
+def epi4_t3_ready(ctx) -> None:
+    _check(_lib.epi4_t3_ready(ctx))
 
 
 def epi4_set_dump(ctx, counts_dev) -> None:

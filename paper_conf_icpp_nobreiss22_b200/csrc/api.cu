@@ -66,6 +66,8 @@ struct epi4_ctx {
     cudaStream_t own_stream = nullptr, stream = nullptr;
     // dataset
     bool loaded = false;
+    bool t3_pending = false;       // sharded T3: the other ranks' shares are not in yet (epi4_t3_ready)
+    int64_t t3_shard = 0;          // triples per rank share (sharded) or C(N,3)
     int32_t n = 0, npad = 0;
     int64_t np[2] = {0, 0};
     int32_t nchunks[2] = {0, 0};
@@ -237,7 +239,9 @@ int finish_load(epi4_ctx* c) {
     const int64_t n = c->n;
     CU(grow(c->T1, c->cap_T1, (size_t)n * 2 * sizeof(uint32_t)));
     CU(grow(c->T2, c->cap_T2, (size_t)c2(n) * 4 * sizeof(uint32_t)));
-    const size_t t3b = (size_t)c3(n) * 8 * sizeof(uint32_t);
+    const bool shard = (c->opts.flags & EPI4_FLAG_SHARD_T3) && c->opts.world > 1;
+    c->t3_shard = shard ? (c3(n) + c->opts.world - 1) / c->opts.world : c3(n);
+    const size_t t3b = (size_t)c->t3_shard * (shard ? c->opts.world : 1) * 8 * sizeof(uint32_t);
     size_t freeb = 0, totb = 0;
     CU(cudaMemGetInfo(&freeb, &totb));
     if (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
@@ -260,15 +264,42 @@ int finish_load(epi4_ctx* c) {
         CU(grow(c->expl[p], c->cap_expl[p], (size_t)(((c->nchunks[p] + 1) / 2 + 1) / 2 * 2) * c->npad * 2 * 128));   // fp4 rows
         CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
     }
-    CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, c->stream, &c->stats.launches_load));
+    {
+        const int64_t lo = shard ? std::min<int64_t>(c3(n), (int64_t)c->opts.rank * c->t3_shard) : 0;
+        const int64_t hi = shard ? std::min<int64_t>(c3(n), lo + c->t3_shard) : c3(n);
+        CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, lo, hi, c->stream, &c->stats.launches_load));
+    }
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(cudaStreamSynchronize(c->stream));
     float ms = 0;
     CU(cudaEventElapsedTime(&ms, c->ev[2], c->ev[3]));
     c->stats.ms_pop = ms;
     c->loaded = true;
+    c->t3_pending = shard;
     return 0;
 }
+
+}  // namespace
+
+extern "C" int epi4_t3_shard(epi4_ctx* c, void** t3_dev, int64_t* shard_bytes, int64_t* total_bytes) {
+    if (!c || !t3_dev || !shard_bytes || !total_bytes) return fail(EPI4_EINVAL, "NULL argument");
+    if (!c->loaded) return fail(EPI4_ESTATE, "no data loaded");
+    if (!((c->opts.flags & EPI4_FLAG_SHARD_T3) && c->opts.world > 1))
+        return fail(EPI4_ESTATE, "T3 is not sharded (opts.flags & EPI4_FLAG_SHARD_T3 with world > 1)");
+    *t3_dev = c->T3;
+    *shard_bytes = c->t3_shard * 8 * (int64_t)sizeof(uint32_t);
+    *total_bytes = *shard_bytes * c->opts.world;
+    return 0;
+}
+
+extern "C" int epi4_t3_ready(epi4_ctx* c) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (!c->loaded || !c->t3_pending) return fail(EPI4_ESTATE, "no sharded T3 pending");
+    c->t3_pending = false;
+    return 0;
+}
+
+namespace {
 
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
     c->loaded = false;
@@ -515,6 +546,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
                       int32_t* n_out) {
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
+    if (c->t3_pending) return fail(EPI4_ESTATE, "sharded T3 incomplete: all-gather the shares, then epi4_t3_ready");
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!quads_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
     CU(cudaSetDevice(c->device));
@@ -570,7 +602,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.status = c->d_status;
     sp.quads_done = c->d_counters + 1;
     sp.prof = c->d_counters + 16;
-    sp.debug = c->opts.reserved[0];
+    sp.debug = c->opts.debug;
     sp.use_filter = !(sp.debug & 16);   // debug 16: exact K2 for every quad (no filter)
 
     c->stats.launches = 0;
@@ -621,6 +653,7 @@ int epi4_search(epi4_ctx* c, int32_t top_k, uint64_t* quads_out, double* k2_out,
 int epi4_tables(epi4_ctx* c, const uint64_t* quads, int64_t n, uint32_t* counts_out) {
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "tables before any load");
+    if (c->t3_pending) return fail(EPI4_ESTATE, "sharded T3 incomplete: all-gather the shares, then epi4_t3_ready");
     if (n < 0 || (n > 0 && (!quads || !counts_out))) return fail(EPI4_EINVAL, "bad quads/counts arguments");
     if (n == 0) return 0;
     CU(cudaSetDevice(c->device));

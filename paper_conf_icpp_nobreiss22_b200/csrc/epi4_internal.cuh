@@ -161,8 +161,8 @@ cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t
                           uint32_t* rows, cudaStream_t s, int64_t* launches);
 cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,
                           int64_t* launches);
-cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, cudaStream_t s,
-                       int64_t* launches);
+cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, int64_t t3_lo, int64_t t3_hi,
+                       cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches);

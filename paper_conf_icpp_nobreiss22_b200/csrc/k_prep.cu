@@ -269,9 +269,9 @@ __global__ void __launch_bounds__(256) k_pop2(DevData d, uint32_t* __restrict__ 
                                                  out[0][2] | (out[1][2] << s), out[0][3] | (out[1][3] << s));
 }
 
-__global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ T3, int64_t ntri) {
-    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= ntri) return;
+__global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ T3, int64_t lo, int64_t hi) {
+    const int64_t r = lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= hi) return;
     int i, j, k;
     decode3(r, i, j, k);
     uint32_t out[2][8];
@@ -304,15 +304,15 @@ __global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ 
                       out[0][7] | (out[1][7] << s));
 }
 
-cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, cudaStream_t s,
-                       int64_t* launches) {
+cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, int64_t t3_lo, int64_t t3_hi,
+                       cudaStream_t s, int64_t* launches) {
     k_pop1<<<(d.n + 255) / 256, 256, 0, s>>>(d, T1);
     if (launches) ++*launches;
-    const int64_t np2 = c2(d.n), np3 = c3(d.n);
+    const int64_t np2 = c2(d.n);
     k_pop2<<<(unsigned)((np2 + 255) / 256), 256, 0, s>>>(d, T2, np2);
     if (launches) ++*launches;
-    if (np3 > 0) {
-        k_pop3<<<(unsigned)((np3 + 255) / 256), 256, 0, s>>>(d, T3, np3);
+    if (t3_hi > t3_lo) {   // the triples [t3_lo, t3_hi) of the colex order (all of them unless sharded)
+        k_pop3<<<(unsigned)((t3_hi - t3_lo + 255) / 256), 256, 0, s>>>(d, T3, t3_lo, t3_hi);
         if (launches) ++*launches;
     }
     return cudaGetLastError();

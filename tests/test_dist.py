@@ -71,3 +71,36 @@ def test_two_rank_search_matches_single_process(world):
     for _, _, idx, k2 in res:                        # every rank holds the same merged answer
         assert idx == [int(v) for v in ref_idx]
         assert k2 == [float(v) for v in ref_k2]
+
+
+def _shard_worker(rank, world, port, shard, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_icpp_nobreiss22_b200 as epi
+        full = torch.zeros(world * shard, dtype=torch.uint8)
+        full[rank * shard:(rank + 1) * shard] = torch.arange(shard, dtype=torch.int64).remainder(251).to(torch.uint8) + rank
+        epi.allgather_shares(full, shard)
+        q.put((rank, full.numpy().tobytes()))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_sharded_table_allgather_assembles_every_share():
+    """The N > 1 sharded-T3 exchange (bench.py, Epi4.gather_t3): equal-size shares, in-place assembly."""
+    world, shard = 2, 1000
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_shard_worker, args=(r, world, port, shard, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    want = np.concatenate([(np.arange(shard) % 251 + r).astype(np.uint8) for r in range(world)]).tobytes()
+    assert res[0] == want and res[1] == want

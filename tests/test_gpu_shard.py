@@ -1,0 +1,60 @@
+"""Sharded 3-way table (multi-GPU path) on one GPU: two contexts play ranks 0 and 1 of a
+2-rank job, each builds its share of T3; rank 1's share is copied into rank 0's buffer (the byte movement
+the NCCL all_gather performs across GPUs) and rank 0 must then produce exactly what an unsharded context
+produces: all 162 counts of sampled quads and the rank-0 top-k."""
+import numpy as np
+import pytest
+
+import datagen
+
+pytestmark = pytest.mark.gpu
+
+
+def _epi():
+    import paper_conf_icpp_nobreiss22_b200 as epi
+    return epi
+
+
+@pytest.mark.parametrize("cfg,nsnp", [("C1", None), ("C2", 96), ("C5", 72)])
+def test_sharded_t3_assembles_to_the_full_table(cfg, nsnp):
+    import torch
+    epi = _epi()
+    d = datagen.make_config(cfg, n_snps=nsnp)
+    rng = np.random.default_rng(7)
+    quads = np.array([epi.pack_index(*sorted(rng.choice(d.n_snps, 4, replace=False))) for _ in range(300)],
+                     dtype=np.uint64)
+    with epi.Epi4(0, pipe="tc", rank=0, world=2) as ref:
+        ref.load_genotypes(d.geno, d.phen)
+        want_tab = ref.tables(quads)
+        want_idx, want_k2 = ref.search(16)
+    r0 = epi.Epi4(0, pipe="tc", rank=0, world=2, shard_t3=True)
+    r1 = epi.Epi4(0, pipe="tc", rank=1, world=2, shard_t3=True)
+    try:
+        r0.load_genotypes(d.geno, d.phen)
+        r1.load_genotypes(d.geno, d.phen)
+        with pytest.raises(epi.Epi4Error):          # tables incomplete until the shares are gathered
+            r0.search(16)
+        full0, shard = r0.t3_device_view()
+        full1, shard1 = r1.t3_device_view()
+        assert shard == shard1 and full0.numel() == full1.numel() == 2 * shard
+        full0[shard:2 * shard].copy_(full1[shard:2 * shard])
+        torch.cuda.synchronize()
+        epi.binding.epi4_t3_ready(r0.ctx)
+        np.testing.assert_array_equal(r0.tables(quads), want_tab)
+        idx, k2 = r0.search(16)
+        np.testing.assert_array_equal(idx, want_idx)
+        np.testing.assert_array_equal(k2, want_k2)
+    finally:
+        r0.close()
+        r1.close()
+
+
+def test_unsharded_context_refuses_shard_calls():
+    epi = _epi()
+    d = datagen.make_config("C1")
+    with epi.Epi4(0, pipe="tc", rank=0, world=2) as e:
+        e.load_genotypes(d.geno, d.phen)
+        with pytest.raises(epi.Epi4Error):
+            epi.binding.epi4_t3_shard(e.ctx)
+        with pytest.raises(epi.Epi4Error):
+            epi.binding.epi4_t3_ready(e.ctx)
