@@ -58,3 +58,22 @@ def test_unsharded_context_refuses_shard_calls():
             epi.binding.epi4_t3_shard(e.ctx)
         with pytest.raises(epi.Epi4Error):
             epi.binding.epi4_t3_ready(e.ctx)
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_rank_partition_merges_to_the_single_rank_result(world):
+    """SURVEY.md §4 T4 on one GPU: every rank of a `world`-rank plan searches only its LPT units; the
+    deterministic merge of the per-rank top-k equals the 1-rank search (bit-identical keys)."""
+    epi = _epi()
+    d = datagen.make_config("C2", n_snps=96)
+    with epi.Epi4(0, pipe="tc") as e:
+        e.load_genotypes(d.geno, d.phen)
+        want_idx, want_k2 = e.search(32)
+    parts = []
+    for r in range(world):
+        with epi.Epi4(0, pipe="tc", rank=r, world=world) as e:
+            e.load_genotypes(d.geno, d.phen)
+            parts.append(e.search(32))
+    idx, k2 = epi.merge_topk(parts, 32)
+    np.testing.assert_array_equal(idx, want_idx)
+    np.testing.assert_array_equal(k2, want_k2)
