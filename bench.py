@@ -243,6 +243,16 @@ def run_ours(args):
         "clocks": clk.summary(),
         "best": {"quad": epi.unpack_index(res[0][0]), "k2": float(res[1][0])},
     }
+    if args.pipe == "tc":
+        # second denominator: the microbenchmarked MMA rate at the clock logged during the timed region —
+        # kind::mxf4 M=256 K=64 issues in N/2 cycles per SM pair (tools/probe_mxf4b.cu), i.e. 128 x 64 x 2 MACs
+        # per SM and cycle whatever N = 2 x 16384 fp4 ops per SM and cycle
+        mhz = out["clocks"].get("sm_mhz") or pk.get("sm_max_mhz", 1965.0)
+        probe = 2.0 * 16384 * 148 * float(mhz) * 1e6 / 1e12
+        out["roofline"]["peak_probe"] = probe
+        out["roofline"]["frac_probe"] = achieved / probe
+        out["roofline"]["peak_probe_source"] = (f"tools/probe_mxf4b.cu MMA rate (16384 {{0,1}}-MACs/clk/SM) x 148 SMs x "
+                                                f"{mhz:.0f} MHz median SM clock of the timed region")
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_oracle_sample(d)
     if rank == 0:
