@@ -282,15 +282,20 @@ __global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ 
             ld_planes(d, p, kc, i, a);
             ld_planes(d, p, kc, j, b);
             ld_planes(d, p, kc, k, e);
+            // POPC-bound: the 4 words of a cell are summed with one carry-save step, x0 + x1 + x2 + x3 =
+            // popc(s ^ x3) + 2 (popc(maj(x0, x1, x2)) + popc(s & x3)) with s = x0 ^ x1 ^ x2: 3 POPC, not 4
 #pragma unroll
-            for (int w = 0; w < 4; ++w)
+            for (int x = 0; x < 2; ++x)
 #pragma unroll
                 for (int y = 0; y < 2; ++y)
 #pragma unroll
                     for (int z = 0; z < 2; ++z) {
-                        const uint32_t yz = b[y][w] & e[z][w];
-                        c[0 * 4 + y * 2 + z] += __popc(a[0][w] & yz);
-                        c[1 * 4 + y * 2 + z] += __popc(a[1][w] & yz);
+                        uint32_t v[4];
+#pragma unroll
+                        for (int w = 0; w < 4; ++w) v[w] = a[x][w] & b[y][w] & e[z][w];
+                        const uint32_t s3 = v[0] ^ v[1] ^ v[2];
+                        const uint32_t cy = (v[0] & v[1]) | (v[2] & (v[0] ^ v[1]));
+                        c[x * 4 + y * 2 + z] += __popc(s3 ^ v[3]) + 2 * (__popc(cy) + __popc(s3 & v[3]));
                     }
         }
 #pragma unroll
