@@ -108,6 +108,11 @@ def allgather_shares(full, shard: int, group=None):
     call every rank holds all of them (one all_gather of `shard` bytes per rank; NCCL or gloo)."""
     import torch.distributed as dist
     r = dist.get_rank(group)
+    if full.is_cuda and dist.get_backend(group) != "nccl":   # gloo (tests, one-GPU runs): stage through the host
+        host = full.cpu()
+        allgather_shares(host, shard, group)
+        full.copy_(host)
+        return full
     mine = full[r * shard:(r + 1) * shard].clone()
     dist.all_gather_into_tensor(full, mine, group=group)
     return full

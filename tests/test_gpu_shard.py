@@ -77,3 +77,17 @@ def test_rank_partition_merges_to_the_single_rank_result(world):
     idx, k2 = epi.merge_topk(parts, 32)
     np.testing.assert_array_equal(idx, want_idx)
     np.testing.assert_array_equal(k2, want_k2)
+
+
+def test_multirank_path_on_one_gpu():
+    """bench.py's N > 1 flow end to end (torchrun, 2 ranks on cuda:0 over gloo — NCCL refuses two ranks on
+    one device): sharded T3 + all_gather, per-rank LPT units, all_gather + merge of the top-k."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--standalone", "--nproc-per-node", "2",
+                        os.path.join(root, "tools", "multirank_one_gpu.py"), "--n-snps", "128"],
+                       capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    assert "OK" in r.stdout
