@@ -92,13 +92,15 @@ constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 512 with 4 prod
 #endif
 constexpr bool REGSPLIT = EPI4_REGSPLIT && PROD_WARPS == 4 && MMA_WARPS + TMA_WARPS == 4 && EPI_WARPS == 8;
 #ifndef EPI4_REGS_CTL
-#define EPI4_REGS_CTL 56
+#define EPI4_REGS_CTL 40
 #endif
 #ifndef EPI4_REGS_PROD
-#define EPI4_REGS_PROD 104
+#define EPI4_REGS_PROD 120
 #endif
 constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
-constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 56 / 96
+constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 40 / 120
+// measured (C2 kernel, same box): control/producers 56/104 520 ms, 48/112 503, 40/120 499, 32/128 504; the
+// epilogue needs >= 176 (48/120 -> 168: 561 ms); control 24 does not fit its code (illegal instruction)
 constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
 constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
 constexpr int TMEM_COLS = 512;
