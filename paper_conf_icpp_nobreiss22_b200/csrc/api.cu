@@ -260,14 +260,48 @@ int finish_load(epi4_ctx* c) {
     CU(cudaMemcpyAsync(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
     CU(cudaStreamSynchronize(c->stream));   // the host table must outlive the async copy
     CU(cudaEventRecord(c->ev[2], c->stream));
+    // the tensor-core pipe builds T3 on the tensor cores (k_quad_tc's 3-way-table mode, the paper's
+    // tensorOp_3way) against the all-ones SNP n; the CUDA-core pipe and the sharded
+    // multi-GPU load keep the POPC kernel (k_pop3), an independent path
+    const bool t3_tc = c->opts.pipe == EPI4_PIPE_TC && !shard && n >= 3;
     for (int p = 0; p < 2; ++p) {
+        if (t3_tc) CU(launch_ones_plane(c->planes[p], (int32_t)n, c->npad, c->nchunks[p], c->np[p], c->stream,
+                                        &c->stats.launches_load));
         CU(grow(c->expl[p], c->cap_expl[p], (size_t)(((c->nchunks[p] + 1) / 2 + 1) / 2 * 2) * c->npad * 2 * 128));   // fp4 rows
         CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
     }
     {
         const int64_t lo = shard ? std::min<int64_t>(c3(n), (int64_t)c->opts.rank * c->t3_shard) : 0;
-        const int64_t hi = shard ? std::min<int64_t>(c3(n), lo + c->t3_shard) : c3(n);
-        CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, lo, hi, c->stream, &c->stats.launches_load));
+        const int64_t hi = t3_tc ? 0 : shard ? std::min<int64_t>(c3(n), lo + c->t3_shard) : c3(n);
+        CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, t3_tc ? 0 : lo, hi, c->stream, &c->stats.launches_load));
+    }
+    if (t3_tc) {
+        // tiles (w-range wp, x, y-range y0, z = n): every w < x < y < n exactly once
+        std::vector<uint64_t> tiles;
+        for (int32_t x = 1; x <= (int32_t)n - 2; ++x)
+            for (int32_t wp = 0; wp * EPI4_WP < x; ++wp)
+                for (int32_t y0 = x + 1; y0 <= (int32_t)n - 1; y0 += EPI4_YR_TC)
+                    tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
+                                    ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
+        CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
+        CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice,
+                           c->stream));
+        const int32_t grid = std::max(2, (c->opts.grid > 0 ? c->opts.grid : c->sm_count) / 2 * 2);
+        if (int r = ensure_lists(c, grid, 1)) return r;
+        SearchParams sp{};
+        sp.d = devdata(c);
+        sp.tile_info = c->d_tiles;
+        sp.ntiles = (int64_t)tiles.size();
+        sp.t3_out = c->T3;
+        sp.topk = 1;
+        sp.list_k2 = c->d_list_k2;
+        sp.list_idx = c->d_list_idx;
+        sp.list_cnt = c->d_list_cnt;
+        sp.status = c->d_status;
+        sp.quads_done = c->d_counters + 1;
+        sp.prof = c->d_counters + 16;
+        CU(launch_quad_tc(sp, grid, c->stream, &c->stats.launches_load));
+        CU(cudaStreamSynchronize(c->stream));   // the host tile list must outlive the async copy
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(cudaStreamSynchronize(c->stream));
@@ -591,6 +625,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.units = c->d_units;
     sp.prefix = c->d_prefix;
     sp.tile_info = nullptr;
+    sp.t3_out = nullptr;
     sp.nunits = nu;
     sp.ntiles = acc;
     sp.tile_counter = c->d_counters;

@@ -130,6 +130,7 @@ struct SearchParams {
     const Unit* units;
     const int64_t* prefix;     // inclusive prefix of tiles per unit
     const uint64_t* tile_info; // (tensor-core pipe) decoded tiles: wp | x << 16 | y0 << 32 | z << 48 (k_tile_table)
+    uint32_t* t3_out;          // non-NULL: 3-way-table mode of k_quad_tc (z = the all-ones SNP n, writes T3)
     int64_t nunits;
     int64_t ntiles;
     unsigned long long* tile_counter;   // dynamic scheduler
@@ -161,6 +162,8 @@ cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t
                           uint32_t* rows, cudaStream_t s, int64_t* launches);
 cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,
                           int64_t* launches);
+cudaError_t launch_ones_plane(uint32_t* planes, int32_t n, int32_t npad, int32_t nchunks, int64_t np, cudaStream_t s,
+                              int64_t* launches);
 cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, int64_t t3_lo, int64_t t3_hi,
                        cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);

@@ -205,6 +205,28 @@ cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks,
     return cudaGetLastError();
 }
 
+// The all-ones SNP: padding row n (AA plane = every real sample, Aa = 0), the virtual z of k_quad_tc's 3-way-table
+// mode (its columns x_b & y_c & z_AA are then x_b & y_c: T3(w, x, y) on the tensor cores
+// "tensorOp_3way").  Row n exists (npad >= n + 16) and lies outside every real quad.
+__global__ void k_ones_plane(uint32_t* __restrict__ planes, int32_t n, int32_t npad, int32_t nchunks, int64_t np) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;   // (chunk, word)
+    if (t >= (int64_t)nchunks * EPI4_CHUNK_WORDS) return;
+    const int64_t kc = t / EPI4_CHUNK_WORDS;
+    const int w = (int)(t % EPI4_CHUNK_WORDS);
+    const int64_t s0 = kc * EPI4_CHUNK_SAMPLES + 32 * w;
+    const uint32_t ones = s0 + 32 <= np ? 0xFFFFFFFFu : (s0 >= np ? 0u : ((1u << (np - s0)) - 1u));
+    planes[plane_off(kc, npad, n, 0, w)] = ones;
+    planes[plane_off(kc, npad, n, 1, w)] = 0u;
+}
+cudaError_t launch_ones_plane(uint32_t* planes, int32_t n, int32_t npad, int32_t nchunks, int64_t np, cudaStream_t s,
+                              int64_t* launches) {
+    const int64_t tot = (int64_t)nchunks * EPI4_CHUNK_WORDS;
+    if (tot <= 0) return cudaSuccess;
+    k_ones_plane<<<(unsigned)((tot + 255) / 256), 256, 0, s>>>(planes, n, npad, nchunks, np);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
 // ---- lower-order tables ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_pop1(DevData d, uint32_t* __restrict__ T1) {
     const int snp = blockIdx.x * blockDim.x + threadIdx.x;

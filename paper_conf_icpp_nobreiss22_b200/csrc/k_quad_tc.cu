@@ -417,7 +417,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                      "r"(tc::TMEM_COLS));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
     }
-    topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);
+    if (!sp.t3_out) topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);
     // Accumulators are zeroed by the epilogue after it reads them (and once here), so every MMA accumulates:
     // the two issuers' MMAs into one tile may then complete in any order.
     __syncthreads();                     // TMEM address visible
@@ -754,6 +754,16 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     c16[8 + k] = a ? v[8 + k] : rv;
                 }
                 const int y = ti.y0 + 2 * g + a;
+                if (sp.t3_out) {
+                    // 3-way-table mode (z = the all-ones SNP n): the d = AA columns are T3(w, x, y)[a b c]
+                    // (PAPER.md:L118 tensorOp_3way); already packed (control | case), written in the T3 layout
+                    if (w < ti.x && y < ti.z) {
+                        uint4* o = reinterpret_cast<uint4*>(sp.t3_out + rank3(w, ti.x, y) * 8);
+                        o[0] = make_uint4(c16[0], c16[2], c16[4], c16[6]);
+                        o[1] = make_uint4(c16[8], c16[10], c16[12], c16[14]);
+                    }
+                    continue;
+                }
                 const bool valid = (w < ti.x) && (y < ti.z) && score;
                 double key = 0.0;
                 uint64_t idx = 0;
@@ -806,7 +816,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     tc_fence_after();
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tc::TMEM_COLS));
-    topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
+    if (!sp.t3_out) topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
 #if EPI4_PROF
     if (tracing && tid == 0) {
         for (int k = 0; k < TR_STEPS; ++k)
