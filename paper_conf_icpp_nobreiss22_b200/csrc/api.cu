@@ -107,14 +107,16 @@ namespace {
 // remainder) and E(M) bounds ln2 |A - A_exact| from fp32 arithmetic (A in log2 units).  Over a quad's 243
 // terms, sum (k + 1/2) <= 2M + 203 and every argument is <= M + 2:
 //   lg2.approx: absolute error <= 2^-21 max(1, log2(M + 2)), times the coefficient (k + 1/2);
-//   per cell: FMUL + 2 FFMA, 3 roundings of relative 2^-24 of at most (n + 3/2) log2(M + 2);
-//   81-term sum (two interleaved partial sums + 1 add): 81 roundings of at most M + 81 (log2(M + 2) + 2).
+//   accumulation: every cell adds its three terms to one of three running sums by FFMA (243 roundings); a
+//   running sum is at most P = M + 81 (log2(M + 2) + 2) between cells and at most P + (n + 3/2) log2(M + 2)
+//   inside a cell, so the roundings total <= u (243 P + 3 (M + 122) log2(M + 2)); + 2 final adds of <= P.
 // E is doubled for safety; at M = 16384 E ~ 0.6, at M = 100003 ~ 4.
 double filter_offset(int64_t m) {
     const double M = (double)m, u = std::ldexp(1.0, -24), l2M = std::log2(M + 2.0), ln2 = std::log(2.0);
     const double e_log = std::ldexp(1.0, -21) * std::max(1.0, l2M) * (2.0 * M + 203.0);
+    const double P = M + 81.0 * (l2M + 2.0);
     const double e_cell = 3.0 * u * (M + 122.0) * l2M;
-    const double e_acc = 81.0 * u * (M + 81.0 * (l2M + 2.0));
+    const double e_acc = (243.0 + 2.0) * u * P;
     const double E = 2.0 * ln2 * (e_log + e_cell + e_acc);
     const double C0 = 0.5 * std::log(2.0 * M_PI) - 1.0;
     return -81.0 - 81.0 * C0 - 13.5 - E;
@@ -132,7 +134,7 @@ DevData devdata(const epi4_ctx* c) {
     d.nsteps[1] = (d.nchunks4[1] + 1) / 2;
     d.nrb = c->npad / 64;
     // c0 <= n0 < 2^pk_shift; 16 whenever both counts fit 16 bits (the epilogue then unpacks each half into a
-    // float with one byte permute, epilogue.cuh cell_T<true>)
+    // float with one byte permute, epilogue.cuh cell_T_acc<true>)
     d.pk_shift = 1;
     while (d.pk_shift < 31 && ((int64_t)1 << d.pk_shift) <= c->np[0]) ++d.pk_shift;
     if (c->np[0] < 65536 && c->np[1] < 65536) d.pk_shift = 16;

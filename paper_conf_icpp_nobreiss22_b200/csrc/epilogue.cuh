@@ -139,7 +139,8 @@ __device__ __forceinline__ void mobius3(uint32_t (&g)[27]) {
 // K2 - (ln2 sum T_c - 81 - 81 C0) lies in (-13.5, 3.375).  With the fp32 rounding bound E(M) computed on the
 // host (api.cu: filter_offset), K2 > ln2 A - 81 - 81 C0 - 13.5 - E for the computed A = sum T_c, so a quad is
 // scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
-// is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + FMUL + 2 FFMA + 1 FADD, 3 MUFU;
+// is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + 3 FFMA into one of three
+// running sums, 3 MUFU;
 // no table and no conversion instruction (a count r < 2^22 becomes the float 2^23 + r by setting the exponent
 // bits).
 __device__ __forceinline__ float lg2_approx(float x) {
@@ -148,16 +149,16 @@ __device__ __forceinline__ float lg2_approx(float x) {
     return y;
 }
 template <bool PK16>
-__device__ __forceinline__ float cell_T(uint32_t v, uint32_t pks, uint32_t pkm) {
+__device__ __forceinline__ void cell_T_acc(uint32_t v, uint32_t pks, uint32_t pkm, float& acc) {
     // 2^23 + r0, 2^23 + r1 (with pks = 16 one byte permute each: [r.lo, r.hi, 0x00, 0x4B])
     const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
     const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
     const float f0 = m0 - 8388607.0f, f1 = m1 - 8388607.0f;     // r + 1
     const float h0 = m0 - 8388607.5f, h1 = m1 - 8388607.5f;     // r + 1/2
     const float fn = f0 + f1, hn = h0 + f1;                     // n + 2, n + 3/2
-    float t = hn * lg2_approx(fn);
-    t = fmaf(-h0, lg2_approx(f0), t);
-    return fmaf(-h1, lg2_approx(f1), t);
+    acc = fmaf(hn, lg2_approx(fn), acc);   // the cell's three terms go straight into the running sum
+    acc = fmaf(-h0, lg2_approx(f0), acc);  // (rounding bound: api.cu filter_offset)
+    acc = fmaf(-h1, lg2_approx(f1), acc);
 }
 
 // Per-quad evaluation from the 16 packed contraction counts c16[8a + 4b + 2c + d] of quad (w, x, y, z).
@@ -179,14 +180,13 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
     const uint4 twxy1 = t3_half(d, q.wxy, 1), twxz1 = t3_half(d, q.wxz, 1), twyz1 = t3_half(d, q.wyz, 1);
     const uint4 pwx = t2_all(d, q.wx), pwy = t2_all(d, q.wy), pwz = t2_all(d, q.wz);
     const uint2 sw = t1_all(d, w);
-    float fa = 0.0f, fb = 0.0f;
+    float fa = 0.0f, fb = 0.0f, fc = 0.0f;
     double kk = 0.0;
     auto consume = [&](const uint32_t (&S)[27], int base) {
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
-                const float t = cell_T<PK16>(S[c], pks, pkm);
-                if (c & 1) fb += t; else fa += t;
+                cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
             } else {
                 const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
                 const double t = __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1));
@@ -218,7 +218,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) R2[c] -= S[c];
     }
     consume(R2, 54);
-    flt = fa + fb;
+    flt = fa + fb + fc;
     k2 = kk;
 }
 
