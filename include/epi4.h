@@ -60,6 +60,11 @@ typedef struct {
  * (the triples [rank*S, (rank+1)*S) of the colex order, S = ceil(C(N,3) / world)); the caller all-gathers
  * the shares (epi4_t3_shard / epi4_t3_ready) — the exchange that replaces building T3 on every GPU. */
 #define EPI4_FLAG_SHARD_T3 1
+/* opts.flags: windowed 3-way table (tensor-core pipe): instead of all C(N,3) triples (32 B each) only two
+ * slabs of 128 x C(N,2) triples are resident, rebuilt on the tensor cores during the search;
+ * chosen automatically when the resident table does not fit in HBM (e.g. N = 4096), forced by this flag.
+ * epi4_tables is unavailable (EPI4_ESTATE) with a windowed table. */
+#define EPI4_FLAG_T3_WINDOWED 2
 
 /* Fill *opts with defaults (block 32, pipe TC, rank 0, world 1, grid 0). */
 void epi4_default_opts(epi4_opts* opts);

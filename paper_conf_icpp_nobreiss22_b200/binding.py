@@ -21,6 +21,7 @@ EPI4_OK, EPI4_EINVAL, EPI4_ENOMEM, EPI4_ECUDA, EPI4_ESTATE, EPI4_ENODEV = 0, -1,
 EPI4_PIPE_TC, EPI4_PIPE_LOP3 = 0, 1
 EPI4_PTR_HOST, EPI4_PTR_DEVICE = 0, 1
 EPI4_FLAG_SHARD_T3 = 1
+EPI4_FLAG_T3_WINDOWED = 2
 EPI4_MAX_TOPK = 1024
 PIPES = {"tc": EPI4_PIPE_TC, "lop3": EPI4_PIPE_LOP3}
 

@@ -73,11 +73,15 @@ struct epi4_ctx {
     int32_t nchunks[2] = {0, 0};
     uint32_t* planes[2] = {nullptr, nullptr};
     uint32_t *T1 = nullptr, *T2 = nullptr, *T3 = nullptr;
+    uint32_t* T3x = nullptr;       // windowed T3: the slab FIRST(X) (T3 then holds FIRST(R))
+    size_t cap_T3x = 0;
+    bool t3_windowed = false;
     double* lgam = nullptr;
     uint8_t* expl[2] = {nullptr, nullptr};
     size_t cap_planes[2] = {0, 0}, cap_T1 = 0, cap_T2 = 0, cap_T3 = 0, cap_lgam = 0, cap_expl[2] = {0, 0};
     unsigned char* scratch = nullptr;     // H2D staging / pack indices
     std::vector<double> host_L;           // lgamma(n + 1), grown on demand
+    std::vector<uint64_t> host_tiles;     // 3-way-table mode tile list (build_t3_tc)
     size_t cap_scratch = 0;
     // search workspace
     Unit* d_units = nullptr;
@@ -146,6 +150,9 @@ DevData devdata(const epi4_ctx* c) {
     d.T1 = c->T1;
     d.T2 = c->T2;
     d.T3 = c->T3;
+    d.T3x = c->T3;
+    d.t3_win = 0;
+    d.t3_w0 = d.t3_x0 = 0;
     d.lgam = c->lgam;
     d.expl[0] = c->expl[0];
     d.expl[1] = c->expl[1];
@@ -160,6 +167,7 @@ void release_data(epi4_ctx* c) {
     dfree(c->T1);
     dfree(c->T2);
     dfree(c->T3);
+    dfree(c->T3x);
     dfree(c->lgam);
     dfree(c->expl[0]);
     dfree(c->expl[1]);
@@ -221,6 +229,47 @@ int ensure_lists(epi4_ctx* c, int32_t slots, int32_t cap) {
     return 0;
 }
 
+// bytes of one windowed-T3 slab: 128 first SNPs x C(n, 2) pairs x 8 packed cells
+size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * sizeof(uint32_t); }
+
+// T3 on the tensor cores (k_quad_tc's 3-way-table mode against the all-ones SNP n, the paper's
+// tensorOp_3way): tiles (w-range wp, x, y-range y0, z = n) cover every w < x < y < n exactly
+// once.  slab_w0 < 0: all w-ranges, resident colex layout; else only the w-range starting at slab_w0, written
+// as the slab FIRST([slab_w0, slab_w0 + 128)) (DevData t3_win).
+int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) {
+    const int32_t n = c->n;
+    std::vector<uint64_t>& tiles = c->host_tiles;
+    tiles.clear();
+    for (int32_t x = 1; x <= n - 2; ++x)
+        for (int32_t wp = 0; wp * EPI4_WP < x; ++wp) {
+            if (slab_w0 >= 0 && wp * EPI4_WP != slab_w0) continue;
+            for (int32_t y0 = x + 1; y0 <= n - 1; y0 += EPI4_YR_TC)
+                tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
+                                ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
+        }
+    if (tiles.empty()) return 0;
+    CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
+    CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice, c->stream));
+    const int32_t grid = std::max(2, (c->opts.grid > 0 ? c->opts.grid : c->sm_count) / 2 * 2);
+    if (int r = ensure_lists(c, grid, 1)) return r;
+    SearchParams sp{};
+    sp.d = devdata(c);
+    sp.tile_info = c->d_tiles;
+    sp.ntiles = (int64_t)tiles.size();
+    sp.t3_out = out;
+    sp.t3_slab_w0 = slab_w0;
+    sp.topk = 1;
+    sp.list_k2 = c->d_list_k2;
+    sp.list_idx = c->d_list_idx;
+    sp.list_cnt = c->d_list_cnt;
+    sp.status = c->d_status;
+    sp.quads_done = c->d_counters + 2;
+    sp.prof = c->d_counters + 24;
+    CU(launch_quad_tc(sp, grid, c->stream, launches));
+    CU(cudaStreamSynchronize(c->stream));   // the host tile list must outlive the async copy
+    return 0;
+}
+
 int finish_load(epi4_ctx* c) {
     // status of the pack / retile kernels
     unsigned int st = 0;
@@ -246,10 +295,19 @@ int finish_load(epi4_ctx* c) {
     const size_t t3b = (size_t)c->t3_shard * (shard ? c->opts.world : 1) * 8 * sizeof(uint32_t);
     size_t freeb = 0, totb = 0;
     CU(cudaMemGetInfo(&freeb, &totb));
-    if (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
+    // windowed T3 (tensor-core pipe): when the resident table does not fit, or on request
+    c->t3_windowed = c->opts.pipe == EPI4_PIPE_TC && !shard && n >= 3 &&
+                     ((c->opts.flags & EPI4_FLAG_T3_WINDOWED) ||
+                      (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3));
+    if (c->t3_windowed) {
+        const size_t slab = t3_slab_bytes(n);
+        CU(grow(c->T3, c->cap_T3, slab));
+        CU(grow(c->T3x, c->cap_T3x, slab));
+    }
+    if (!c->t3_windowed && t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
         return fail(EPI4_ENOMEM, "3-way tables need %.1f GB but only %.1f GB of HBM are free (N=%d); "
                     "the windowed T3 path for larger N is not built yet", t3b / 1e9, freeb / 1e9, c->n);
-    CU(grow(c->T3, c->cap_T3, t3b));
+    if (!c->t3_windowed) CU(grow(c->T3, c->cap_T3, t3b));
     // lgamma table L[k] = lgamma(k + 1) for k in [0, M + 1]
     const int64_t m = c->np[0] + c->np[1];
     std::vector<double>& L = c->host_L;
@@ -277,33 +335,8 @@ int finish_load(epi4_ctx* c) {
         const int64_t hi = t3_tc ? 0 : shard ? std::min<int64_t>(c3(n), lo + c->t3_shard) : c3(n);
         CU(launch_pop(devdata(c), c->T1, c->T2, c->T3, t3_tc ? 0 : lo, hi, c->stream, &c->stats.launches_load));
     }
-    if (t3_tc) {
-        // tiles (w-range wp, x, y-range y0, z = n): every w < x < y < n exactly once
-        std::vector<uint64_t> tiles;
-        for (int32_t x = 1; x <= (int32_t)n - 2; ++x)
-            for (int32_t wp = 0; wp * EPI4_WP < x; ++wp)
-                for (int32_t y0 = x + 1; y0 <= (int32_t)n - 1; y0 += EPI4_YR_TC)
-                    tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
-                                    ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
-        CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
-        CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice,
-                           c->stream));
-        const int32_t grid = std::max(2, (c->opts.grid > 0 ? c->opts.grid : c->sm_count) / 2 * 2);
-        if (int r = ensure_lists(c, grid, 1)) return r;
-        SearchParams sp{};
-        sp.d = devdata(c);
-        sp.tile_info = c->d_tiles;
-        sp.ntiles = (int64_t)tiles.size();
-        sp.t3_out = c->T3;
-        sp.topk = 1;
-        sp.list_k2 = c->d_list_k2;
-        sp.list_idx = c->d_list_idx;
-        sp.list_cnt = c->d_list_cnt;
-        sp.status = c->d_status;
-        sp.quads_done = c->d_counters + 1;
-        sp.prof = c->d_counters + 16;
-        CU(launch_quad_tc(sp, grid, c->stream, &c->stats.launches_load));
-        CU(cudaStreamSynchronize(c->stream));   // the host tile list must outlive the async copy
+    if (t3_tc && !c->t3_windowed) {
+        if (int r = build_t3_tc(c, c->T3, -1, &c->stats.launches_load)) return r;
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(cudaStreamSynchronize(c->stream));
@@ -597,12 +630,24 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
                                  "(%lld, %lld); use EPI4_PIPE_LOP3", (long long)c->np[0], (long long)c->np[1]);
     const int32_t G = quad_split(c->opts.pipe), YR = quad_yr(c->opts.pipe);
     std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
-    std::vector<int64_t> prefix((size_t)std::max<int64_t>(nu, 1));
-    int64_t acc = 0;
-    for (int64_t i = 0; i < nu; ++i) {
-        units[(size_t)i] = plan[(size_t)(ub + i)].u;
-        acc += unit_tiles(c->n, units[(size_t)i].x, YR) * G;
-        prefix[(size_t)i] = acc;
+    for (int64_t i = 0; i < nu; ++i) units[(size_t)i] = plan[(size_t)(ub + i)].u;
+    // Windowed T3: the units are taken grouped by (w-range R, 128-SNP x-range X) so that each launch reads
+    // only the slabs FIRST(R) and FIRST(X) (rebuilt on the tensor cores when R or X changes); the result does
+    // not depend on the order (top-k by (K2, index)).  Resident T3: one group, the plan order.
+    struct Group { int64_t b, e; int32_t wr, xr; };
+    std::vector<Group> groups;
+    if (c->t3_windowed && nu > 0) {
+        std::stable_sort(units.begin(), units.begin() + nu, [](const Unit& p, const Unit& q) {
+            return p.wr != q.wr ? p.wr < q.wr : p.x < q.x;
+        });
+        for (int64_t i = 0; i < nu; ++i) {
+            const int32_t xr = units[(size_t)i].x / EPI4_WP;
+            if (groups.empty() || groups.back().wr != units[(size_t)i].wr || groups.back().xr != xr)
+                groups.push_back(Group{i, i, units[(size_t)i].wr, xr});
+            groups.back().e = i + 1;
+        }
+    } else if (nu > 0) {
+        groups.push_back(Group{0, nu, -1, -1});
     }
     if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
         dfree(c->d_units);
@@ -610,10 +655,6 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
         c->units_cap = (size_t)std::max<int64_t>(nu, 1);
         CU(cudaMalloc(&c->d_units, c->units_cap * sizeof(Unit)));
         CU(cudaMalloc(&c->d_prefix, c->units_cap * sizeof(int64_t)));
-    }
-    if (nu > 0) {
-        CU(cudaMemcpyAsync(c->d_units, units.data(), nu * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
-        CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), nu * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
     }
     int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
     grid = std::max(2, grid / 2 * 2);                 // whole CTA pairs
@@ -628,8 +669,9 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.prefix = c->d_prefix;
     sp.tile_info = nullptr;
     sp.t3_out = nullptr;
-    sp.nunits = nu;
-    sp.ntiles = acc;
+    sp.t3_slab_w0 = -1;
+    sp.nunits = 0;
+    sp.ntiles = 0;
     sp.tile_counter = c->d_counters;
     sp.topk = top_k;
     sp.list_k2 = c->d_list_k2;
@@ -643,16 +685,50 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.use_filter = !(sp.debug & 16);   // debug 16: exact K2 for every quad (no filter)
 
     c->stats.launches = 0;
-    if (c->opts.pipe != EPI4_PIPE_LOP3 && acc > 0) {
-        CU(grow(c->d_tiles, c->cap_tiles, (size_t)acc * sizeof(uint64_t)));
-        sp.tile_info = c->d_tiles;
-        CU(launch_tile_table(sp, c->d_tiles, c->stream, &c->stats.launches));
-    }
     CU(cudaEventRecord(c->ev[2], c->stream));
-    if (acc > 0) {
+    int64_t acc = 0;
+    int32_t slab_r = -1, slab_x = -1;
+    std::vector<int64_t> prefix;
+    for (const Group& gr : groups) {
+        const int64_t gn = gr.e - gr.b;
+        prefix.assign((size_t)gn, 0);
+        int64_t gacc = 0;
+        for (int64_t i = 0; i < gn; ++i) {
+            gacc += unit_tiles(c->n, units[(size_t)(gr.b + i)].x, YR) * G;
+            prefix[(size_t)i] = gacc;
+        }
+        if (gacc == 0) continue;
+        if (c->t3_windowed) {
+            if (gr.wr != slab_r) {            // FIRST(R) into T3
+                if (int r = build_t3_tc(c, c->T3, gr.wr * EPI4_WP, &c->stats.launches)) return r;
+                slab_r = gr.wr;
+                if (slab_x == slab_r) slab_x = -1;
+            }
+            if (gr.xr != gr.wr && gr.xr != slab_x) {   // FIRST(X) into T3x
+                if (int r = build_t3_tc(c, c->T3x, gr.xr * EPI4_WP, &c->stats.launches)) return r;
+                slab_x = gr.xr;
+            }
+            sp.d.t3_win = 1;
+            sp.d.t3_w0 = gr.wr * EPI4_WP;
+            sp.d.t3_x0 = gr.xr * EPI4_WP;
+            sp.d.T3 = c->T3;
+            sp.d.T3x = gr.xr == gr.wr ? c->T3 : c->T3x;
+        }
+        // pageable host source: the copy has completed when cudaMemcpyAsync returns, so `prefix` may be reused
+        CU(cudaMemcpyAsync(c->d_units, units.data() + gr.b, gn * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
+        CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), gn * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
+        sp.nunits = gn;
+        sp.ntiles = gacc;
+        sp.tile_info = nullptr;
+        if (c->opts.pipe != EPI4_PIPE_LOP3) {
+            CU(grow(c->d_tiles, c->cap_tiles, (size_t)gacc * sizeof(uint64_t)));
+            sp.tile_info = c->d_tiles;
+            CU(launch_tile_table(sp, c->d_tiles, c->stream, &c->stats.launches));
+        }
         cudaError_t e = c->opts.pipe == EPI4_PIPE_LOP3 ? launch_quad_lop3(sp, grid, c->stream, &c->stats.launches)
                                                        : launch_quad_tc(sp, grid, c->stream, &c->stats.launches);
         CU(e);
+        acc += gacc;
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(launch_merge(sp, grid, c->d_out_k2, c->d_out_idx, c->d_out_n, c->stream, &c->stats.launches));
@@ -691,6 +767,7 @@ int epi4_tables(epi4_ctx* c, const uint64_t* quads, int64_t n, uint32_t* counts_
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "tables before any load");
     if (c->t3_pending) return fail(EPI4_ESTATE, "sharded T3 incomplete: all-gather the shares, then epi4_t3_ready");
+    if (c->t3_windowed) return fail(EPI4_ESTATE, "epi4_tables needs the resident 3-way table (windowed T3 in use)");
     if (n < 0 || (n > 0 && (!quads || !counts_out))) return fail(EPI4_EINVAL, "bad quads/counts arguments");
     if (n == 0) return 0;
     CU(cudaSetDevice(c->device));

@@ -67,7 +67,13 @@ struct DevData {
     uint32_t npk;                // n0 | n1 << pk_shift
     const uint32_t* T1;
     const uint32_t* T2;
-    const uint32_t* T3;
+    const uint32_t* T3;          // resident: all triples, colex rank; windowed: the slab FIRST(R) (below)
+    // Windowed T3 (t3_win = 1): every triple a quad w < x < y < z reads starts with w (wxy, wxz,
+    // wyz) or with x (xyz).  T3 holds FIRST(R) = {(w, j, k): w in the 128-SNP w-range R = [t3_w0, t3_w0 + 128)} at
+    // entry (w - t3_w0) * C(n,2) + rank2(j, k); T3x holds FIRST(X) for the x-range X = [t3_x0, t3_x0 + 128) the
+    // same way (T3x == T3 when X == R).
+    const uint32_t* T3x;
+    int32_t t3_win, t3_w0, t3_x0;
     const double* lgam;          // M + 2 entries
     const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
     double flt_off;              // fp32 K2 filter: exact-score a quad iff ln2 A + flt_off <= threshold (epilogue.cuh)
@@ -131,6 +137,7 @@ struct SearchParams {
     const int64_t* prefix;     // inclusive prefix of tiles per unit
     const uint64_t* tile_info; // (tensor-core pipe) decoded tiles: wp | x << 16 | y0 << 32 | z << 48 (k_tile_table)
     uint32_t* t3_out;          // non-NULL: 3-way-table mode of k_quad_tc (z = the all-ones SNP n, writes T3)
+    int32_t t3_slab_w0;        // 3-way-table mode: < 0 resident colex layout, else the slab FIRST([w0, w0+128))
     int64_t nunits;
     int64_t ntiles;
     unsigned long long* tile_counter;   // dynamic scheduler

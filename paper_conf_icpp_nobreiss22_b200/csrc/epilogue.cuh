@@ -49,13 +49,23 @@ struct QuadRanks {
     int64_t wxy, wxz, wyz, xyz;   // T3
     int64_t wx, wy, wz, xy, xz, yz;   // T2
 };
-__device__ __forceinline__ QuadRanks quad_ranks(int w, int x, int y, int z) {
+// T3 entries: resident (colex rank3) or windowed (slab entries, epi4_internal.cuh DevData); xyz is read from T3x
+__device__ __forceinline__ QuadRanks quad_ranks(const DevData& d, int w, int x, int y, int z) {
     QuadRanks q;
-    const int64_t c2x = c2(x), c2y = c2(y), c2z = c2(z), c3y = c3(y), c3z = c3(z);
-    q.wxy = c3y + c2x + w;
-    q.wxz = c3z + c2x + w;
-    q.wyz = c3z + c2y + w;
-    q.xyz = c3z + c2y + x;
+    const int64_t c2x = c2(x), c2y = c2(y), c2z = c2(z);
+    if (d.t3_win) {
+        const int64_t pn = c2(d.n), bw = (int64_t)(w - d.t3_w0) * pn;
+        q.wxy = bw + c2y + x;
+        q.wxz = bw + c2z + x;
+        q.wyz = bw + c2z + y;
+        q.xyz = (int64_t)(x - d.t3_x0) * pn + c2z + y;
+    } else {
+        const int64_t c3y = c3(y), c3z = c3(z);
+        q.wxy = c3y + c2x + w;
+        q.wxz = c3z + c2x + w;
+        q.wyz = c3z + c2y + w;
+        q.xyz = c3z + c2y + x;
+    }
     q.wx = c2x + w;
     q.wy = c2y + w;
     q.wz = c2z + w;
@@ -173,7 +183,8 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
                                           const uint32_t (&c16)[16], float& flt, double& k2, uint32_t* dump) {
     const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
     // all table reads up front (one round of load latency per quad)
-    const uint4 txyz0 = t3_half(d, q.xyz, 0), txyz1 = t3_half(d, q.xyz, 1);
+    const uint4 txyz0 = __ldg(reinterpret_cast<const uint4*>(d.T3x + q.xyz * 8)),
+                txyz1 = __ldg(reinterpret_cast<const uint4*>(d.T3x + q.xyz * 8 + 4));
     const uint4 pxy = t2_all(d, q.xy), pxz = t2_all(d, q.xz), pyz = t2_all(d, q.yz);
     const uint2 sx = t1_all(d, x), sy = t1_all(d, y), sz = t1_all(d, z);
     const uint4 twxy0 = t3_half(d, q.wxy, 0), twxz0 = t3_half(d, q.wxz, 0), twyz0 = t3_half(d, q.wyz, 0);
@@ -229,7 +240,7 @@ static __device__ __noinline__ double score_quad(const DevData& d, int w, int x,
                                                  const uint32_t (&c16)[16], uint32_t* dump_row) {
     float flt;
     double k2;
-    const QuadRanks q = quad_ranks(w, x, y, z);
+    const QuadRanks q = quad_ranks(d, w, x, y, z);
     if (dump_row) quad_eval<2>(d, q, w, x, y, z, c16, flt, k2, dump_row);
     else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;

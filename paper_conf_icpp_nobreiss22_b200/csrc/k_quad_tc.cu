@@ -758,7 +758,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     // 3-way-table mode (z = the all-ones SNP n): the d = AA columns are T3(w, x, y)[a b c]
                     // (PAPER.md:L118 tensorOp_3way); already packed (control | case), written in the T3 layout
                     if (w < ti.x && y < ti.z) {
-                        uint4* o = reinterpret_cast<uint4*>(sp.t3_out + rank3(w, ti.x, y) * 8);
+                        // resident: colex rank; windowed slab FIRST(R): (w - w0) * C(n,2) + rank2(x, y)
+                        const int64_t e = sp.t3_slab_w0 >= 0
+                                              ? (int64_t)(w - sp.t3_slab_w0) * c2(d.n) + c2(y) + ti.x
+                                              : rank3(w, ti.x, y);
+                        uint4* o = reinterpret_cast<uint4*>(sp.t3_out + e * 8);
                         o[0] = make_uint4(c16[0], c16[2], c16[4], c16[6]);
                         o[1] = make_uint4(c16[8], c16[10], c16[12], c16[14]);
                     }
@@ -777,7 +781,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         // fp32 Stirling filter (epilogue.cuh); only possible top-k members get the exact K2
                         float flt;
                         double unused;
-                        quad_eval<0, PK16>(d, quad_ranks(w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt, unused, nullptr);
+                        quad_eval<0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt, unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
                         offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
