@@ -109,6 +109,14 @@ int epi4_search(epi4_ctx* ctx, int32_t top_k, uint64_t* quads_out, double* k2_ou
 int epi4_search_units(epi4_ctx* ctx, int64_t unit_begin, int64_t unit_end, int32_t top_k,
                       uint64_t* quads_out, double* k2_out, int32_t* n_out);
 
+/* Third-order search (the paper's predecessors): every triple
+ * i < j < k of this rank's share (the 4-way plan's units, rank/world as for epi4_search), its 2 x 27 table
+ * (8 non-aa counts on the tensor cores against an all-ones SNP, the other 19 recovered from T2/T1/n as in
+ * PAPER.md:L126) scored by K2 over 27 cells in double, canonical order c = 9a + 3b + c.  Output as
+ * epi4_search: the top_k smallest (K2, index) keys ascending, index = i<<48 | j<<32 | k<<16.
+ * Tensor-core pipe only (EPI4_EINVAL otherwise); host arrays of top_k entries. */
+int epi4_search3(epi4_ctx* ctx, int32_t top_k, uint64_t* triples_out, double* k2_out, int32_t* n_out);
+
 /* Verification hook: the 2 x 81 contingency table (controls row first, cell 27a+9b+3c+d,
  * 0=AA 1=Aa 2=aa) of each listed quad (packed, any SNP order), computed from the device planes:
  * 16 cells by AND+POPC of the planes and the other 65 by the same lower-order recovery the search

@@ -51,6 +51,10 @@ def _load():
         lib.oracle_score.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, P, ctypes.c_int64, P, ctypes.c_int32]
         lib.oracle_search.restype = ctypes.c_int
         lib.oracle_search.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P, ctypes.c_int32]
+        lib.oracle_tables3.restype = ctypes.c_int
+        lib.oracle_tables3.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, P, ctypes.c_int64, P]
+        lib.oracle_search3.restype = ctypes.c_int
+        lib.oracle_search3.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P, ctypes.c_int32]
         lib.oracle_max_threads.restype = ctypes.c_int32
         lib.oracle_max_threads.argtypes = [ctypes.c_int32]
         _lib = lib
@@ -120,6 +124,33 @@ def search(geno, phen, top_k: int = 1, n_snps: int | None = None, n_threads: int
                                _ptr(k2v), _ptr(nout), n_threads)
     if rc:
         raise ValueError(f"oracle_search failed: {rc}")
+    return idx[: nout[0]], k2v[: nout[0]]
+
+
+def tables3(geno, phen, triples) -> np.ndarray:
+    """Per-sample brute-force 2 x 27 tables (cell 9a + 3b + c) of the given triples -> uint32 [nt, 2, 27]."""
+    geno, phen = _prep(geno, phen)
+    t = np.ascontiguousarray(np.asarray(triples, dtype=np.int32).reshape(-1, 3))
+    out = np.zeros((t.shape[0], 2, 27), dtype=np.uint32)
+    rc = _load().oracle_tables3(_ptr(geno), _ptr(phen), geno.shape[0], geno.shape[1], _ptr(t), t.shape[0], _ptr(out))
+    if rc:
+        raise ValueError(f"oracle_tables3 failed: {rc}")
+    return out
+
+
+def search3(geno, phen, top_k: int = 1, n_snps: int | None = None, n_threads: int = 0):
+    """Exhaustive third-order search over all triples of SNPs [0, n_snps) -> (packed idx i<<48|j<<32|k<<16,
+    K2 over 27 cells), the top_k smallest (K2, idx) keys ascending."""
+    geno, phen = _prep(geno, phen)
+    n = geno.shape[0] if n_snps is None else int(n_snps)
+    geno = np.ascontiguousarray(geno[:n])
+    idx = np.zeros(top_k, dtype=np.uint64)
+    k2v = np.zeros(top_k, dtype=np.float64)
+    nout = np.zeros(1, dtype=np.int32)
+    rc = _load().oracle_search3(_ptr(geno), _ptr(phen), n, geno.shape[1], int(top_k), _ptr(idx), _ptr(k2v),
+                                _ptr(nout), n_threads)
+    if rc:
+        raise ValueError(f"oracle_search3 failed: {rc}")
     return idx[: nout[0]], k2v[: nout[0]]
 
 

@@ -77,7 +77,7 @@ static void count_quad(const uint8_t *geno, const uint8_t *phen, int64_t m,
 }
 
 static int validate(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m) {
-    if (n < 4 || n > 65536 || m < 1) return -1;
+    if (n < 3 || n > 65536 || m < 1) return -1;
     for (int64_t s = 0; s < m; ++s) if (phen[s] > 1) return -2;
     for (int64_t x = 0; x < (int64_t)n * m; ++x) if (geno[x] > 2) return -3;
     return 0;
@@ -184,6 +184,87 @@ int oracle_search(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m
         }
     }
     /* deterministic merge of the per-thread lists */
+    int32_t len = 0;
+    double *fk = (double *)malloc(sizeof(double) * top_k);
+    uint64_t *fi = (uint64_t *)malloc(sizeof(uint64_t) * top_k);
+    for (int32_t t = 0; t < nthr; ++t)
+        for (int32_t e = 0; e < tl[t]; ++e)
+            topk_insert(fk, fi, &len, top_k, tk[(size_t)t * top_k + e], ti[(size_t)t * top_k + e]);
+    memcpy(k2_out, fk, sizeof(double) * len);
+    memcpy(idx_out, fi, sizeof(uint64_t) * len);
+    *n_out = len;
+    free(fk); free(fi); free(tk); free(ti); free(tl);
+    return 0;
+}
+
+/* ---- third-order search (the paper's predecessors) ----------
+ * The same definition one order lower: every triple i<j<k, its 2 x 27 genotype table by a per-sample loop
+ * (cell = 9 g_i + 3 g_j + g_k), K2 = sum_{c=0}^{26} [(L(r_c + 1) - L(r_c0)) - L(r_c1)] in canonical cell order,
+ * top-k smallest (K2, index) keys with index = i<<48 | j<<32 | k<<16 (the quad packing with l = 0). */
+#define NCELL3 27
+static void count_triple(const uint8_t *geno, const uint8_t *phen, int64_t m, int32_t i, int32_t j, int32_t k,
+                         uint32_t *r) {
+    const uint8_t *gi = geno + (int64_t)i * m, *gj = geno + (int64_t)j * m, *gk = geno + (int64_t)k * m;
+    memset(r, 0, sizeof(uint32_t) * 2 * NCELL3);
+    for (int64_t s = 0; s < m; ++s) r[phen[s] * NCELL3 + 9 * gi[s] + 3 * gj[s] + gk[s]] += 1;
+}
+static double k2_27(const uint32_t *r) {
+    double k2 = 0.0;
+    for (int c = 0; c < NCELL3; ++c) {
+        uint32_t r0 = r[c], r1 = r[NCELL3 + c];
+        double t = (log_factorial(r0 + r1 + 1) - log_factorial(r0)) - log_factorial(r1);
+        k2 = k2 + t;
+    }
+    return k2;
+}
+
+/* 2 x 27 tables of an explicit triple list (indices used as given). counts: nt x 2 x 27 */
+int oracle_tables3(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m, const int32_t *tri, int64_t nt,
+                   uint32_t *counts) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    for (int64_t t = 0; t < nt; ++t) {
+        for (int u = 0; u < 3; ++u)
+            if (tri[3 * t + u] < 0 || tri[3 * t + u] >= n) return -4;
+        count_triple(geno, phen, m, tri[3 * t], tri[3 * t + 1], tri[3 * t + 2], counts + t * 2 * NCELL3);
+    }
+    return 0;
+}
+
+int oracle_search3(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m, int32_t top_k,
+                   uint64_t *idx_out, double *k2_out, int32_t *n_out, int32_t n_threads) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    if (top_k < 1) return -5;
+    int32_t nthr = 1;
+#ifdef _OPENMP
+    if (n_threads > 0) omp_set_num_threads(n_threads);
+    nthr = omp_get_max_threads();
+#endif
+    double *tk = (double *)malloc(sizeof(double) * (size_t)top_k * nthr);
+    uint64_t *ti = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)top_k * nthr);
+    int32_t *tl = (int32_t *)calloc(nthr, sizeof(int32_t));
+    if (!tk || !ti || !tl) { free(tk); free(ti); free(tl); return -6; }
+#ifdef _OPENMP
+#pragma omp parallel
+#endif
+    {
+        int32_t tid = 0;
+#ifdef _OPENMP
+        tid = omp_get_thread_num();
+#endif
+        uint32_t r[2 * NCELL3];
+#ifdef _OPENMP
+#pragma omp for schedule(dynamic, 1)
+#endif
+        for (int32_t i = 0; i < n; ++i)
+            for (int32_t j = i + 1; j < n; ++j)
+                for (int32_t k = j + 1; k < n; ++k) {
+                    count_triple(geno, phen, m, i, j, k, r);
+                    topk_insert(tk + (size_t)tid * top_k, ti + (size_t)tid * top_k, &tl[tid], top_k, k2_27(r),
+                                oracle_pack(i, j, k, 0));
+                }
+    }
     int32_t len = 0;
     double *fk = (double *)malloc(sizeof(double) * top_k);
     uint64_t *fi = (uint64_t *)malloc(sizeof(uint64_t) * top_k);

@@ -70,6 +70,10 @@ class Epi4:
     def search(self, top_k: int = 1):
         return binding.epi4_search(self.ctx, top_k)
 
+    def search3(self, top_k: int = 1):
+        """Third-order search: (packed i<<48|j<<32|k<<16, K2 over 27 cells)."""
+        return binding.epi4_search3(self.ctx, top_k)
+
     def search_units(self, unit_begin: int, unit_end: int, top_k: int = 1):
         return binding.epi4_search_units(self.ctx, unit_begin, unit_end, top_k)
 

@@ -65,6 +65,7 @@ def _load():
         "epi4_get_bits": (ctypes.c_int, [P, P, P]),
         "epi4_search": (ctypes.c_int, [P, I32, P, P, P]),
         "epi4_search_units": (ctypes.c_int, [P, I64, I64, I32, P, P, P]),
+        "epi4_search3": (ctypes.c_int, [P, I32, P, P, P]),
         "epi4_tables": (ctypes.c_int, [P, P, I64, P]),
         "epi4_set_dump": (ctypes.c_int, [P, P]),
         "epi4_t3_shard": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(I64), ctypes.POINTER(I64)]),
@@ -159,6 +160,14 @@ def epi4_search(ctx, top_k: int):
     k = np.zeros(top_k, dtype=np.float64)
     n = np.zeros(1, dtype=np.int32)
     _check(_lib.epi4_search(ctx, int(top_k), _ptr(q), _ptr(k), _ptr(n)))
+    return q[: n[0]], k[: n[0]]
+
+
+def epi4_search3(ctx, top_k: int):
+    q = np.zeros(top_k, dtype=np.uint64)
+    k = np.zeros(top_k, dtype=np.float64)
+    n = np.zeros(1, dtype=np.int32)
+    _check(_lib.epi4_search3(ctx, int(top_k), _ptr(q), _ptr(k), _ptr(n)))
     return q[: n[0]], k[: n[0]]
 
 

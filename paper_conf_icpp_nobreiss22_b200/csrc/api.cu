@@ -325,8 +325,9 @@ int finish_load(epi4_ctx* c) {
     // multi-GPU load keep the POPC kernel (k_pop3), an independent path
     const bool t3_tc = c->opts.pipe == EPI4_PIPE_TC && !shard && n >= 3;
     for (int p = 0; p < 2; ++p) {
-        if (t3_tc) CU(launch_ones_plane(c->planes[p], (int32_t)n, c->npad, c->nchunks[p], c->np[p], c->stream,
-                                        &c->stats.launches_load));
+        if (c->opts.pipe == EPI4_PIPE_TC && n >= 3)   // z of the 3-way-table mode and the third-order search
+            CU(launch_ones_plane(c->planes[p], (int32_t)n, c->npad, c->nchunks[p], c->np[p], c->stream,
+                                 &c->stats.launches_load));
         CU(grow(c->expl[p], c->cap_expl[p], (size_t)(((c->nchunks[p] + 1) / 2 + 1) / 2 * 2) * c->npad * 2 * 128));   // fp4 rows
         CU(launch_expand(c->planes[p], c->npad, c->nchunks[p], c->expl[p], c->stream, &c->stats.launches_load));
     }
@@ -670,6 +671,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.tile_info = nullptr;
     sp.t3_out = nullptr;
     sp.t3_slab_w0 = -1;
+    sp.search3 = 0;
     sp.nunits = 0;
     sp.ntiles = 0;
     sp.tile_counter = c->d_counters;
@@ -755,6 +757,72 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
                                 ? (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES
                                 : (double)(sp.d.nsteps[0] + sp.d.nsteps[1]) * 512.0;
     c->stats.executed_macs = (double)(acc / G) * 256.0 * 8.0 * YR * ksamples;
+    *n_out = nout;
+    return 0;
+}
+
+int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_out, int32_t* n_out) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
+    if (c->opts.pipe != EPI4_PIPE_TC) return fail(EPI4_EINVAL, "the third-order search runs on the tensor-core pipe");
+    if (c->n < 3) return fail(EPI4_EINVAL, "N=%d < 3", c->n);
+    if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
+    if (!triples_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
+    CU(cudaSetDevice(c->device));
+    // this rank's units (the 4-way plan: w-range x second SNP) with z = the all-ones SNP n: each triple
+    // w < x < y once across ranks
+    std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
+    std::vector<uint64_t>& tiles = c->host_tiles;
+    tiles.clear();
+    auto add = [&](int32_t wr, int32_t x) {
+        for (int32_t y0 = x + 1; y0 <= c->n - 1; y0 += EPI4_YR_TC)
+            tiles.push_back((uint64_t)(uint16_t)wr | ((uint64_t)(uint16_t)x << 16) | ((uint64_t)(uint16_t)y0 << 32) |
+                            ((uint64_t)(uint16_t)c->n << 48));
+    };
+    for (const PlanEntry& pe : plan) add(pe.u.wr, pe.u.x);
+    // the 4-way plan has no units with x = n - 2 (no room for z); their triples (w, n - 2, n - 1) go to rank 0
+    if (c->opts.rank == 0)
+        for (int32_t wr = 0; wr * EPI4_WP < c->n - 2; ++wr) add(wr, c->n - 2);
+    int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
+    grid = std::max(2, grid / 2 * 2);
+    if (int r = ensure_lists(c, grid, top_k)) return r;
+    CU(cudaMemsetAsync(c->d_list_cnt, 0, (size_t)grid * sizeof(int32_t), c->stream));
+    CU(cudaMemsetAsync(c->d_counters, 0, 32 * sizeof(unsigned long long), c->stream));
+    SearchParams sp{};
+    sp.d = devdata(c);
+    sp.t3_slab_w0 = -1;
+    sp.search3 = 1;
+    sp.topk = top_k;
+    sp.list_k2 = c->d_list_k2;
+    sp.list_idx = c->d_list_idx;
+    sp.list_cnt = c->d_list_cnt;
+    sp.status = c->d_status;
+    sp.quads_done = c->d_counters + 1;
+    sp.prof = c->d_counters + 16;
+    c->stats.launches = 0;
+    CU(cudaEventRecord(c->ev[2], c->stream));
+    if (!tiles.empty()) {
+        CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
+        CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice,
+                           c->stream));
+        sp.tile_info = c->d_tiles;
+        sp.ntiles = (int64_t)tiles.size();
+        CU(launch_quad_tc(sp, grid, c->stream, &c->stats.launches));
+    }
+    CU(cudaEventRecord(c->ev[3], c->stream));
+    CU(launch_merge(sp, grid, c->d_out_k2, c->d_out_idx, c->d_out_n, c->stream, &c->stats.launches));
+    int32_t nout = 0;
+    unsigned long long ctr[32] = {0};
+    CU(cudaMemcpyAsync(&nout, c->d_out_n, sizeof nout, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(triples_out, c->d_out_idx, (size_t)top_k * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(k2_out, c->d_out_k2, (size_t)top_k * sizeof(double), cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(ctr, c->d_counters, sizeof ctr, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaStreamSynchronize(c->stream));   // also keeps the host tile list alive for the copy
+    float ms = 0;
+    CU(cudaEventElapsedTime(&ms, c->ev[2], c->ev[3]));
+    c->stats.ms_quad = ms;
+    c->stats.quads = (int64_t)ctr[1];
+    c->stats.tiles = (int64_t)tiles.size();
     *n_out = nout;
     return 0;
 }

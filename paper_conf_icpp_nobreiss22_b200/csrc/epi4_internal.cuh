@@ -138,6 +138,7 @@ struct SearchParams {
     const uint64_t* tile_info; // (tensor-core pipe) decoded tiles: wp | x << 16 | y0 << 32 | z << 48 (k_tile_table)
     uint32_t* t3_out;          // non-NULL: 3-way-table mode of k_quad_tc (z = the all-ones SNP n, writes T3)
     int32_t t3_slab_w0;        // 3-way-table mode: < 0 resident colex layout, else the slab FIRST([w0, w0+128))
+    int32_t search3;           // third-order search mode (z = the all-ones SNP n, epi4_search3)
     int64_t nunits;
     int64_t ntiles;
     unsigned long long* tile_counter;   // dynamic scheduler

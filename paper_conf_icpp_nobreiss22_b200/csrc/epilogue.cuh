@@ -245,6 +245,44 @@ static __device__ __noinline__ double score_quad(const DevData& d, int w, int x,
     else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;
 }
+// Third-order search: exact K2 of triple w < x < y from its 8 packed non-aa counts
+// c8[4a + 2b + c] (the 3-way-table mode's d = AA columns), the same recovery one order lower: generalized
+// cells S[9a + 3b + c] (digit 2 = '*') from c8, T2, T1 and n, aa recovered on the three axes,
+// K2 = sum_c ((L[r_c + 1] - L[r_c0]) - L[r_c1]) in canonical order c = 9a + 3b + c (reading #4).
+static __device__ __noinline__ double score_triple(const DevData& d, int w, int x, int y, const uint32_t (&c8)[8]) {
+    const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
+    const uint4 pwx = t2_all(d, c2(x) + w), pwy = t2_all(d, c2(y) + w), pxy = t2_all(d, c2(y) + x);
+    const uint2 sw = t1_all(d, w), sx = t1_all(d, x), sy = t1_all(d, y);
+    uint32_t S[27];
+#pragma unroll
+    for (int c = 0; c < 27; ++c) {
+        const int a = c / 9, b = (c / 3) % 3, e = c % 3;
+        const int ns = (a == 2) + (b == 2) + (e == 2);
+        uint32_t v;
+        if (ns == 0) v = c8[4 * a + 2 * b + e];
+        else if (ns == 1) {
+            if (a == 2) v = u4(pxy, 2 * b + e);
+            else if (b == 2) v = u4(pwy, 2 * a + e);
+            else v = u4(pwx, 2 * a + b);
+        } else if (ns == 2) {
+            if (a != 2) v = u2(sw, a);
+            else if (b != 2) v = u2(sx, b);
+            else v = u2(sy, e);
+        } else {
+            v = d.npk;
+        }
+        S[c] = v;
+    }
+    mobius3(S);
+    double kk = 0.0;
+#pragma unroll
+    for (int c = 0; c < 27; ++c) {
+        const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+        kk = __dadd_rn(kk, __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1)));
+    }
+    return kk;
+}
+
 // pack separate control / case counts (CUDA-core kernels)
 __device__ __forceinline__ void pack16(const DevData& d, const uint32_t (&c0)[16], const uint32_t (&c1)[16],
                                        uint32_t (&c16)[16]) {

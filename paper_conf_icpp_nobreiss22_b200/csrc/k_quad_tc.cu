@@ -417,7 +417,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                      "r"(tc::TMEM_COLS));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
     }
-    if (!sp.t3_out) topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);
+    if (!sp.t3_out) topk_load(tk, sp, blockIdx.x, tid, tc::THREADS);   // (also the third-order search)
     // Accumulators are zeroed by the epilogue after it reads them (and once here), so every MMA accumulates:
     // the two issuers' MMAs into one tile may then complete in any order.
     __syncthreads();                     // TMEM address visible
@@ -766,6 +766,20 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         o[0] = make_uint4(c16[0], c16[2], c16[4], c16[6]);
                         o[1] = make_uint4(c16[8], c16[10], c16[12], c16[14]);
                     }
+                    continue;
+                }
+                if (sp.search3) {
+                    // third-order search (z = the all-ones SNP n): triple (w, x, y) from the d = AA columns
+                    const bool v3 = (w < ti.x) && (y < ti.z) && score;
+                    double key3 = 0.0;
+                    uint64_t idx3 = 0;
+                    if (v3) {
+                        const uint32_t c8[8] = {c16[0], c16[2], c16[4], c16[6], c16[8], c16[10], c16[12], c16[14]};
+                        key3 = score_triple(d, w, ti.x, y, c8);
+                        idx3 = pack_quad(w, ti.x, y, 0);
+                        ++my_quads;
+                    }
+                    warp_offer(tk, v3, key3, idx3);
                     continue;
                 }
                 const bool valid = (w < ti.x) && (y < ti.z) && score;

@@ -1,0 +1,44 @@
+"""Pins of the third-order oracle (oracle.search3 / tables3) against things other
+than itself: the 4-way oracle tables marginalised over the fourth SNP (a separately written per-sample loop),
+a closed form, and an independent numpy K2 over all triples of a tiny dataset."""
+import itertools
+import math
+
+import numpy as np
+
+import datagen
+import oracle
+
+
+def _k2_numpy(t):
+    r0, r1 = t[0].astype(np.int64), t[1].astype(np.int64)
+    return sum(math.lgamma(a + b + 2) - math.lgamma(a + 1) - math.lgamma(b + 1) for a, b in zip(r0, r1))
+
+
+def test_triple_tables_are_quad_marginals():
+    d = datagen.make_config("C1")
+    rng = np.random.default_rng(3)
+    for _ in range(20):
+        i, j, k, l = sorted(rng.choice(d.n_snps, 4, replace=False))
+        t3 = oracle.tables3(d.geno, d.phen, [[i, j, k]])[0]
+        q = oracle.tables(d.geno, d.phen, [[i, j, k, l]])[0].reshape(2, 27, 3).sum(axis=2)
+        np.testing.assert_array_equal(t3, q)
+        assert t3[0].sum() == d.n_controls and t3[1].sum() == d.n_cases
+
+
+def test_triple_k2_closed_form_identical_samples():
+    geno = np.zeros((3, 40), dtype=np.uint8)
+    phen = np.array([0] * 15 + [1] * 25, dtype=np.uint8)
+    idx, k2 = oracle.search3(geno, phen, top_k=1)
+    want = math.lgamma(40 + 2) - math.lgamma(15 + 1) - math.lgamma(25 + 1)
+    assert abs(k2[0] - want) < 1e-9 * want and int(idx[0]) == oracle.pack_index(0, 1, 2, 0)
+
+
+def test_triple_search_equals_numpy_brute_force():
+    d = datagen.make_dataset(12, 30, 34, 99, planted=None, name="tiny3")
+    tri = list(itertools.combinations(range(12), 3))
+    tabs = oracle.tables3(d.geno, d.phen, tri)
+    keys = sorted((_k2_numpy(t), oracle.pack_index(i, j, k, 0)) for t, (i, j, k) in zip(tabs, tri))
+    idx, k2 = oracle.search3(d.geno, d.phen, top_k=10)
+    assert [int(v) for v in idx] == [kk[1] for kk in keys[:10]]
+    np.testing.assert_allclose(k2, [kk[0] for kk in keys[:10]], rtol=1e-12)

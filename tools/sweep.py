@@ -68,6 +68,11 @@ def main():
                 n1 = int(round(0.3 * m))
                 todo.append((f"C5-sweep M={m}", lambda m=m, n1=n1: datagen.make_dataset(
                     1024, m - n1, n1, 2000 + m, planted=datagen.planted_quad_for(1024), name=f"sweep{m}")))
+        elif w == "paper2048":
+            # the paper's single-GPU shape (2048 SNPs, balanced; P:L264-266 used M = 524288) at the largest M the
+            # packed 32-bit counts allow (65535 per class)
+            todo.append(("paper-shape N=2048 M=131070", lambda: datagen.make_dataset(
+                2048, 65535, 65535, 3000, planted=datagen.planted_quad_for(2048), name="paper2048")))
         else:
             todo.append((w, lambda w=w: datagen.make_config(w)))
     with open(a.out, "a") as f:
