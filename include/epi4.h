@@ -53,7 +53,7 @@ typedef struct {
     int32_t debug;    /* diagnostics only, 0 in production (debug modes disable warp roles; results  */
                       /*   invalid except bit 16 = exact K2 for every quad, no filter)               */
     int32_t flags;    /* EPI4_FLAG_* bits                                                          */
-    int32_t reserved;
+    int32_t objective; /* EPI4_OBJ_K2 (default) or EPI4_OBJ_MI  */
 } epi4_opts;
 
 /* opts.flags: with world > 1, a load computes only this rank's contiguous share of the 3-way table T3
@@ -65,6 +65,16 @@ typedef struct {
  * chosen automatically when the resident table does not fit in HBM (e.g. N = 4096), forced by this flag.
  * epi4_tables is unavailable (EPI4_ESTATE) with a windowed table. */
 #define EPI4_FLAG_T3_WINDOWED 2
+
+/* opts.objective (the table construction does not depend on the score):
+ *   EPI4_OBJ_K2: K2 (the paper's), smallest first.
+ *   EPI4_OBJ_MI: mutual information between the quad's 81-cell genotype and the phenotype, largest first.
+ *     Computed exactly as M*I = sum_c [(X(r_c0) + X(r_c1)) - X(r_c)] + (X(M) - X(n0) - X(n1)) with
+ *     X(k) = k ln k (X(0) = 0) from a host-built double table, summed in canonical cell order; the key
+ *     returned in k2_out is -M*I (so "smallest key first" ranks by largest MI).  No fp32 filter: every quad is
+ *     scored exactly.  epi4_search3 supports K2 only. */
+#define EPI4_OBJ_K2 0
+#define EPI4_OBJ_MI 1
 
 /* Fill *opts with defaults (block 32, pipe TC, rank 0, world 1, grid 0). */
 void epi4_default_opts(epi4_opts* opts);

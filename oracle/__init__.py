@@ -55,6 +55,10 @@ def _load():
         lib.oracle_tables3.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, P, ctypes.c_int64, P]
         lib.oracle_search3.restype = ctypes.c_int
         lib.oracle_search3.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P, ctypes.c_int32]
+        lib.oracle_mi.restype = ctypes.c_double
+        lib.oracle_mi.argtypes = [P]
+        lib.oracle_search_mi.restype = ctypes.c_int
+        lib.oracle_search_mi.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P]
         lib.oracle_max_threads.restype = ctypes.c_int32
         lib.oracle_max_threads.argtypes = [ctypes.c_int32]
         _lib = lib
@@ -125,6 +129,28 @@ def search(geno, phen, top_k: int = 1, n_snps: int | None = None, n_threads: int
     if rc:
         raise ValueError(f"oracle_search failed: {rc}")
     return idx[: nout[0]], k2v[: nout[0]]
+
+
+def mi(table) -> float:
+    """M * I (mutual information of the 81-cell genotype and the phenotype, nats) of a 2 x 81 table."""
+    t = np.ascontiguousarray(np.asarray(table, dtype=np.uint32).reshape(2, 81))
+    return float(_load().oracle_mi(_ptr(t)))
+
+
+def search_mi(geno, phen, top_k: int = 1, n_snps: int | None = None):
+    """Exhaustive search ranked by mutual information -> (packed idx, key = -M*I),
+    the top_k smallest keys ascending (single-threaded: for small test problems)."""
+    geno, phen = _prep(geno, phen)
+    n = geno.shape[0] if n_snps is None else int(n_snps)
+    geno = np.ascontiguousarray(geno[:n])
+    idx = np.zeros(top_k, dtype=np.uint64)
+    key = np.zeros(top_k, dtype=np.float64)
+    nout = np.zeros(1, dtype=np.int32)
+    rc = _load().oracle_search_mi(_ptr(geno), _ptr(phen), n, geno.shape[1], int(top_k), _ptr(idx), _ptr(key),
+                                  _ptr(nout))
+    if rc:
+        raise ValueError(f"oracle_search_mi failed: {rc}")
+    return idx[: nout[0]], key[: nout[0]]
 
 
 def tables3(geno, phen, triples) -> np.ndarray:

@@ -197,6 +197,43 @@ int oracle_search(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m
     return 0;
 }
 
+/* ---- alternative objective (the table does not depend on the
+ * score): mutual information between the 81-cell genotype of the quad and the phenotype, by its definition
+ * I = sum_{c,p} (r_cp / M) ln(r_cp M / (r_c n_p)), written as M*I = sum_c [(X(r_c0) + X(r_c1)) - X(r_c)]
+ * + (X(M) - X(n0) - X(n1)) with X(k) = k ln k, X(0) = 0 (0 ln 0 = 0), in canonical cell order.  Ranked
+ * largest first: the key is -M*I, ties by the smallest packed index. */
+static double xlogx(uint32_t k) { return k ? (double)k * log((double)k) : 0.0; }
+double oracle_mi(const uint32_t *r) {   /* M * I of one 2 x 81 table */
+    uint32_t n0 = 0, n1 = 0;
+    for (int c = 0; c < NCELL; ++c) { n0 += r[c]; n1 += r[NCELL + c]; }
+    double acc = 0.0;
+    for (int c = 0; c < NCELL; ++c) {
+        uint32_t r0 = r[c], r1 = r[NCELL + c];
+        acc = acc + ((xlogx(r0) + xlogx(r1)) - xlogx(r0 + r1));
+    }
+    const double M = (double)(n0 + n1);
+    const double cst = (M > 0 ? M * log(M) : 0.0) - xlogx(n0) - xlogx(n1);
+    return acc + cst;
+}
+
+int oracle_search_mi(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m, int32_t top_k,
+                     uint64_t *idx_out, double *key_out, int32_t *n_out) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    if (top_k < 1) return -5;
+    int32_t len = 0;
+    uint32_t r[2 * NCELL];
+    for (int32_t i = 0; i < n; ++i)
+        for (int32_t j = i + 1; j < n; ++j)
+            for (int32_t k = j + 1; k < n; ++k)
+                for (int32_t l = k + 1; l < n; ++l) {
+                    count_quad(geno, phen, m, i, j, k, l, r);
+                    topk_insert(key_out, idx_out, &len, top_k, -oracle_mi(r), oracle_pack(i, j, k, l));
+                }
+    *n_out = len;
+    return 0;
+}
+
 /* ---- third-order search (the paper's predecessors) ----------
  * The same definition one order lower: every triple i<j<k, its 2 x 27 genotype table by a per-sample loop
  * (cell = 9 g_i + 3 g_j + g_k), K2 = sum_{c=0}^{26} [(L(r_c + 1) - L(r_c0)) - L(r_c1)] in canonical cell order,

@@ -22,6 +22,7 @@ EPI4_PIPE_TC, EPI4_PIPE_LOP3 = 0, 1
 EPI4_PTR_HOST, EPI4_PTR_DEVICE = 0, 1
 EPI4_FLAG_SHARD_T3 = 1
 EPI4_FLAG_T3_WINDOWED = 2
+EPI4_OBJ_K2, EPI4_OBJ_MI = 0, 1
 EPI4_MAX_TOPK = 1024
 PIPES = {"tc": EPI4_PIPE_TC, "lop3": EPI4_PIPE_LOP3}
 
@@ -35,7 +36,7 @@ class Epi4Error(RuntimeError):
 class epi4_opts(ctypes.Structure):
     _fields_ = [("block", ctypes.c_int32), ("pipe", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("world", ctypes.c_int32), ("grid", ctypes.c_int32), ("debug", ctypes.c_int32),
-                ("flags", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("flags", ctypes.c_int32), ("objective", ctypes.c_int32)]
 
 
 class epi4_stats(ctypes.Structure):

@@ -77,6 +77,9 @@ struct epi4_ctx {
     size_t cap_T3x = 0;
     bool t3_windowed = false;
     double* lgam = nullptr;
+    double* xlx = nullptr;         // X(k) = k ln k (EPI4_OBJ_MI)
+    size_t cap_xlx = 0;
+    std::vector<double> host_X;
     uint8_t* expl[2] = {nullptr, nullptr};
     size_t cap_planes[2] = {0, 0}, cap_T1 = 0, cap_T2 = 0, cap_T3 = 0, cap_lgam = 0, cap_expl[2] = {0, 0};
     unsigned char* scratch = nullptr;     // H2D staging / pack indices
@@ -154,6 +157,12 @@ DevData devdata(const epi4_ctx* c) {
     d.t3_win = 0;
     d.t3_w0 = d.t3_x0 = 0;
     d.lgam = c->lgam;
+    d.xlx = c->xlx;
+    d.objective = c->opts.objective;
+    {
+        const double M = (double)(c->np[0] + c->np[1]), a = (double)c->np[0], b = (double)c->np[1];
+        d.mi_const = (M > 0 ? M * std::log(M) : 0.0) - (a > 0 ? a * std::log(a) : 0.0) - (b > 0 ? b * std::log(b) : 0.0);
+    }
     d.expl[0] = c->expl[0];
     d.expl[1] = c->expl[1];
     d.flt_off = filter_offset(c->np[0] + c->np[1]);
@@ -169,6 +178,7 @@ void release_data(epi4_ctx* c) {
     dfree(c->T3);
     dfree(c->T3x);
     dfree(c->lgam);
+    dfree(c->xlx);
     dfree(c->expl[0]);
     dfree(c->expl[1]);
     c->loaded = false;
@@ -306,7 +316,7 @@ int finish_load(epi4_ctx* c) {
     }
     if (!c->t3_windowed && t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
         return fail(EPI4_ENOMEM, "3-way tables need %.1f GB but only %.1f GB of HBM are free (N=%d); "
-                    "the windowed T3 path for larger N is not built yet", t3b / 1e9, freeb / 1e9, c->n);
+                    "the windowed T3 needs the tensor-core pipe without sharding", t3b / 1e9, freeb / 1e9, c->n);
     if (!c->t3_windowed) CU(grow(c->T3, c->cap_T3, t3b));
     // lgamma table L[k] = lgamma(k + 1) for k in [0, M + 1]
     const int64_t m = c->np[0] + c->np[1];
@@ -318,6 +328,16 @@ int finish_load(epi4_ctx* c) {
     }
     CU(grow(c->lgam, c->cap_lgam, ((size_t)m + 2) * sizeof(double)));
     CU(cudaMemcpyAsync(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+    if (c->opts.objective == EPI4_OBJ_MI) {   // X(k) = k ln k, X(0) = 0
+        std::vector<double>& X = c->host_X;
+        const size_t hx = X.size();
+        if (hx < (size_t)m + 2) {
+            X.resize((size_t)m + 2);
+            for (size_t k = hx; k < X.size(); ++k) X[k] = k ? (double)k * std::log((double)k) : 0.0;
+        }
+        CU(grow(c->xlx, c->cap_xlx, ((size_t)m + 2) * sizeof(double)));
+        CU(cudaMemcpyAsync(c->xlx, X.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+    }
     CU(cudaStreamSynchronize(c->stream));   // the host table must outlive the async copy
     CU(cudaEventRecord(c->ev[2], c->stream));
     // the tensor-core pipe builds T3 on the tensor cores (k_quad_tc's 3-way-table mode, the paper's
@@ -423,6 +443,8 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
     epi4_default_opts(&o);
     if (opts) o = *opts;
     if (o.block != EPI4_B) return fail(EPI4_EINVAL, "block=%d: only B=32 is supported", o.block);
+    if (o.objective != EPI4_OBJ_K2 && o.objective != EPI4_OBJ_MI)
+        return fail(EPI4_EINVAL, "objective=%d: EPI4_OBJ_K2 or EPI4_OBJ_MI", o.objective);
     if (o.pipe != EPI4_PIPE_TC && o.pipe != EPI4_PIPE_LOP3) return fail(EPI4_EINVAL, "unknown pipe %d", o.pipe);
     if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return fail(EPI4_EINVAL, "bad rank/world %d/%d", o.rank, o.world);
     int ndev = 0;
@@ -684,7 +706,8 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.quads_done = c->d_counters + 1;
     sp.prof = c->d_counters + 16;
     sp.debug = c->opts.debug;
-    sp.use_filter = !(sp.debug & 16);   // debug 16: exact K2 for every quad (no filter)
+    // debug 16: exact K2 for every quad; the fp32 filter bounds K2 only, other objectives are scored exactly
+    sp.use_filter = !(sp.debug & 16) && c->opts.objective == EPI4_OBJ_K2;
 
     c->stats.launches = 0;
     CU(cudaEventRecord(c->ev[2], c->stream));
@@ -765,6 +788,7 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
     if (c->opts.pipe != EPI4_PIPE_TC) return fail(EPI4_EINVAL, "the third-order search runs on the tensor-core pipe");
+    if (c->opts.objective != EPI4_OBJ_K2) return fail(EPI4_EINVAL, "the third-order search scores K2 only");
     if (c->n < 3) return fail(EPI4_EINVAL, "N=%d < 3", c->n);
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!triples_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");

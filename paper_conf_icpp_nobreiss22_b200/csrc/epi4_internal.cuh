@@ -75,6 +75,9 @@ struct DevData {
     const uint32_t* T3x;
     int32_t t3_win, t3_w0, t3_x0;
     const double* lgam;          // M + 2 entries
+    const double* xlx;           // X(k) = k ln k, M + 2 entries (EPI4_OBJ_MI)
+    double mi_const;             // X(M) - X(n0) - X(n1)
+    int32_t objective;           // EPI4_OBJ_*
     const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
     double flt_off;              // fp32 K2 filter: exact-score a quad iff ln2 A + flt_off <= threshold (epilogue.cuh)
 };

@@ -198,6 +198,10 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
                 cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
+            } else if (MODE == 3) {
+                // mutual information (EPI4_OBJ_MI): (X(r0) + X(r1)) - X(r0 + r1), X(k) = k ln k
+                const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+                kk = __dadd_rn(kk, __dsub_rn(__dadd_rn(__ldg(d.xlx + r0), __ldg(d.xlx + r1)), __ldg(d.xlx + (r0 + r1))));
             } else {
                 const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
                 const double t = __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1));
@@ -230,7 +234,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
     }
     consume(R2, 54);
     flt = fa + fb + fc;
-    k2 = kk;
+    k2 = MODE == 3 ? -__dadd_rn(kk, d.mi_const) : kk;   // MI: key = -M*I (largest MI first)
 }
 
 // exact K2 of one quad (double, canonical order) from its packed contraction counts; optionally dumps its 162
@@ -242,6 +246,7 @@ static __device__ __noinline__ double score_quad(const DevData& d, int w, int x,
     double k2;
     const QuadRanks q = quad_ranks(d, w, x, y, z);
     if (dump_row) quad_eval<2>(d, q, w, x, y, z, c16, flt, k2, dump_row);
+    else if (d.objective == EPI4_OBJ_MI) quad_eval<3>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;
 }

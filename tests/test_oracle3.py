@@ -42,3 +42,45 @@ def test_triple_search_equals_numpy_brute_force():
     idx, k2 = oracle.search3(d.geno, d.phen, top_k=10)
     assert [int(v) for v in idx] == [kk[1] for kk in keys[:10]]
     np.testing.assert_allclose(k2, [kk[0] for kk in keys[:10]], rtol=1e-12)
+
+
+# ---- mutual-information objective ----------------------------------------------
+def _mi_numpy(t):
+    """M * I from the definition sum p(g, y) ln(p(g, y) / (p(g) p(y))), numpy, cells with r > 0 only."""
+    t = t.astype(np.float64)
+    M = t.sum()
+    pg = t.sum(axis=0) / M
+    py = t.sum(axis=1) / M
+    s = 0.0
+    for p in range(2):
+        for c in range(t.shape[1]):
+            if t[p, c] > 0:
+                pj = t[p, c] / M
+                s += pj * math.log(pj / (pg[c] * py[p]))
+    return M * s
+
+
+def test_mi_matches_definition_and_closed_forms():
+    d = datagen.make_config("C1")
+    tabs = oracle.tables(d.geno, d.phen, [[0, 1, 2, 3], [3, 11, 22, 35], [5, 9, 17, 30]])
+    for t in tabs:
+        assert abs(oracle.mi(t) - _mi_numpy(t)) < 1e-9 * max(1.0, abs(_mi_numpy(t)))
+    # independence: every cell split in the class ratio -> MI = 0; perfect association -> M * H(phenotype)
+    ind = np.zeros((2, 81), dtype=np.uint32)
+    ind[0, :10], ind[1, :10] = 3, 1
+    assert abs(oracle.mi(ind)) < 1e-9
+    perf = np.zeros((2, 81), dtype=np.uint32)
+    perf[0, 0], perf[1, 80] = 30, 10
+    want = -(30 * math.log(30 / 40) + 10 * math.log(10 / 40))
+    assert abs(oracle.mi(perf) - want) < 1e-9 * want
+
+
+def test_mi_search_equals_numpy_ranking():
+    d = datagen.make_dataset(9, 20, 24, 5, planted=None, name="tinymi")
+    quads = list(itertools.combinations(range(9), 4))
+    tabs = oracle.tables(d.geno, d.phen, quads)
+    keys = sorted((-_mi_numpy(t), oracle.pack_index(*q)) for t, q in zip(tabs, quads))
+    idx, key = oracle.search_mi(d.geno, d.phen, top_k=8)
+    np.testing.assert_allclose(key, [k[0] for k in keys[:8]], rtol=1e-9)
+    # the same quads, up to near-ties the two rounding orders may swap
+    assert set(int(v) for v in idx[:5]) <= set(k[1] for k in keys[:8])
