@@ -59,6 +59,10 @@ def _load():
         lib.oracle_mi.argtypes = [P]
         lib.oracle_search_mi.restype = ctypes.c_int
         lib.oracle_search_mi.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P]
+        lib.oracle_chi2.restype = ctypes.c_double
+        lib.oracle_chi2.argtypes = [P]
+        lib.oracle_search_chi2.restype = ctypes.c_int
+        lib.oracle_search_chi2.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P]
         lib.oracle_max_threads.restype = ctypes.c_int32
         lib.oracle_max_threads.argtypes = [ctypes.c_int32]
         _lib = lib
@@ -150,6 +154,28 @@ def search_mi(geno, phen, top_k: int = 1, n_snps: int | None = None):
                                   _ptr(nout))
     if rc:
         raise ValueError(f"oracle_search_mi failed: {rc}")
+    return idx[: nout[0]], key[: nout[0]]
+
+
+def chi2(table) -> float:
+    """Pearson chi-square (no continuity correction) of a 2 x 81 table over its non-empty genotype cells."""
+    t = np.ascontiguousarray(np.asarray(table, dtype=np.uint32).reshape(2, 81))
+    return float(_load().oracle_chi2(_ptr(t)))
+
+
+def search_chi2(geno, phen, top_k: int = 1, n_snps: int | None = None):
+    """Exhaustive search ranked by Pearson chi-square -> (packed idx, key = -X^2),
+    the top_k smallest keys ascending (single-threaded: for small test problems)."""
+    geno, phen = _prep(geno, phen)
+    n = geno.shape[0] if n_snps is None else int(n_snps)
+    geno = np.ascontiguousarray(geno[:n])
+    idx = np.zeros(top_k, dtype=np.uint64)
+    key = np.zeros(top_k, dtype=np.float64)
+    nout = np.zeros(1, dtype=np.int32)
+    rc = _load().oracle_search_chi2(_ptr(geno), _ptr(phen), n, geno.shape[1], int(top_k), _ptr(idx), _ptr(key),
+                                    _ptr(nout))
+    if rc:
+        raise ValueError(f"oracle_search_chi2 failed: {rc}")
     return idx[: nout[0]], key[: nout[0]]
 
 

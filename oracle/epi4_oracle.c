@@ -234,6 +234,50 @@ int oracle_search_mi(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_
     return 0;
 }
 
+/* ---- second alternative objective ("e.g. mutual information, chi^2"): Pearson's
+ * chi-square statistic of the 2 x 81 (phenotype x genotype cell) table, no continuity correction, over the
+ * cells with r_c = r_c0 + r_c1 > 0 (an empty genotype column has no expected count and is dropped, the usual
+ * contingency-table convention):  X^2 = sum_{c: r_c > 0} sum_p (r_cp - E_cp)^2 / E_cp,  E_cp = r_c n_p / M.
+ * Expanding the square, sum_p (r_cp - E_cp)^2 / E_cp = (M / r_c) sum_p r_cp^2 / n_p - r_c, so
+ *     X^2 = M * S / (n0 n1) - M,   S = sum_{c: r_c > 0} (r_c0^2 n1 + r_c1^2 n0) / r_c,
+ * with the numerator an exact integer (< n0 n1 M < 2^53 whenever the counts pack into 32 bits with room; the
+ * GPU library checks the bound) and one correctly rounded division per cell, summed in canonical cell order.
+ * X^2 := 0 when a phenotype is empty (no variation).  Ranked largest first: key = -X^2, ties by the smallest
+ * packed index.  Pinned in tests/test_oracle3.py against scipy.stats.chi2_contingency (correction=False) and
+ * closed forms (independence -> 0; perfect association -> M). */
+double oracle_chi2(const uint32_t *r) {   /* X^2 of one 2 x 81 table */
+    uint32_t n0 = 0, n1 = 0;
+    for (int c = 0; c < NCELL; ++c) { n0 += r[c]; n1 += r[NCELL + c]; }
+    if (n0 == 0 || n1 == 0) return 0.0;
+    double s = 0.0;
+    for (int c = 0; c < NCELL; ++c) {
+        const uint64_t r0 = r[c], r1 = r[NCELL + c], rc = r0 + r1;
+        if (rc == 0) continue;
+        const uint64_t num = r0 * r0 * n1 + r1 * r1 * n0;
+        s = s + (double)num / (double)rc;
+    }
+    const double M = (double)n0 + (double)n1;
+    return (M * s) / ((double)n0 * (double)n1) - M;
+}
+
+int oracle_search_chi2(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m, int32_t top_k,
+                       uint64_t *idx_out, double *key_out, int32_t *n_out) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    if (top_k < 1) return -5;
+    int32_t len = 0;
+    uint32_t r[2 * NCELL];
+    for (int32_t i = 0; i < n; ++i)
+        for (int32_t j = i + 1; j < n; ++j)
+            for (int32_t k = j + 1; k < n; ++k)
+                for (int32_t l = k + 1; l < n; ++l) {
+                    count_quad(geno, phen, m, i, j, k, l, r);
+                    topk_insert(key_out, idx_out, &len, top_k, -oracle_chi2(r), oracle_pack(i, j, k, l));
+                }
+    *n_out = len;
+    return 0;
+}
+
 /* ---- third-order search (the paper's predecessors) ----------
  * The same definition one order lower: every triple i<j<k, its 2 x 27 genotype table by a per-sample loop
  * (cell = 9 g_i + 3 g_j + g_k), K2 = sum_{c=0}^{26} [(L(r_c + 1) - L(r_c0)) - L(r_c1)] in canonical cell order,

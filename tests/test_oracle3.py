@@ -84,3 +84,56 @@ def test_mi_search_equals_numpy_ranking():
     np.testing.assert_allclose(key, [k[0] for k in keys[:8]], rtol=1e-9)
     # the same quads, up to near-ties the two rounding orders may swap
     assert set(int(v) for v in idx[:5]) <= set(k[1] for k in keys[:8])
+
+
+# ---- chi-square objective ("e.g. mutual information, chi^2") ---------------------
+def _chi2_scipy(t):
+    """Pearson X^2 from scipy's textbook routine on the 2 x (non-empty cells) table, no continuity correction."""
+    from scipy.stats import chi2_contingency
+    t = np.asarray(t, dtype=np.float64)
+    t = t[:, t.sum(axis=0) > 0]
+    return float(chi2_contingency(t, correction=False)[0])
+
+
+def test_chi2_matches_scipy_and_closed_forms():
+    d = datagen.make_config("C1")
+    quads = [[0, 1, 2, 3], [3, 11, 22, 35], [5, 9, 17, 30], [1, 20, 30, 39]]
+    for t in oracle.tables(d.geno, d.phen, quads):
+        want = _chi2_scipy(t)
+        assert abs(oracle.chi2(t) - want) < 1e-10 * max(1.0, want)
+    # unbalanced ragged workload (C5 shape, 30/70) on a few quads
+    d5 = datagen.make_config("C5", n_snps=12)
+    for t in oracle.tables(d5.geno, d5.phen, [[0, 1, 2, 3], [2, 5, 7, 11]]):
+        want = _chi2_scipy(t)
+        assert abs(oracle.chi2(t) - want) < 1e-10 * max(1.0, want)
+    # independence: every non-empty cell split in the class ratio -> 0; perfect association -> M;
+    # an empty phenotype -> 0 (defined, no variation)
+    ind = np.zeros((2, 81), dtype=np.uint32)
+    ind[0, :10], ind[1, :10] = 3, 1
+    assert abs(oracle.chi2(ind)) < 1e-9
+    perf = np.zeros((2, 81), dtype=np.uint32)
+    perf[0, 0], perf[1, 80] = 30, 10
+    assert abs(oracle.chi2(perf) - 40.0) < 1e-12
+    one = np.zeros((2, 81), dtype=np.uint32)
+    one[0, :5] = 7
+    assert oracle.chi2(one) == 0.0
+    # 2 x 2 textbook value: [[10, 20], [30, 40]] -> X^2 = 100 * (10*40 - 20*30)^2 / (30 * 70 * 40 * 60)
+    tb = np.zeros((2, 81), dtype=np.uint32)
+    tb[0, 4], tb[0, 60], tb[1, 4], tb[1, 60] = 10, 20, 30, 40
+    assert abs(oracle.chi2(tb) - 100 * 200.0 ** 2 / (30 * 70 * 40 * 60)) < 1e-12
+
+
+def test_chi2_search_equals_scipy_ranking():
+    d = datagen.make_dataset(9, 20, 24, 5, planted=None, name="tinychi")
+    quads = list(itertools.combinations(range(9), 4))
+    tabs = oracle.tables(d.geno, d.phen, quads)
+    keys = sorted((-_chi2_scipy(t), oracle.pack_index(*q)) for t, q in zip(tabs, quads))
+    idx, key = oracle.search_chi2(d.geno, d.phen, top_k=8)
+    np.testing.assert_allclose(key, [k[0] for k in keys[:8]], rtol=1e-9)
+    assert set(int(v) for v in idx[:5]) <= set(k[1] for k in keys[:8])
+
+
+def test_chi2_search_recovers_planted_quad():
+    d = datagen.make_config("C1")
+    idx, _ = oracle.search_chi2(d.geno, d.phen, top_k=1)
+    assert oracle.unpack_index(int(idx[0])) == tuple(d.planted)
