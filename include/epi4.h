@@ -53,7 +53,7 @@ typedef struct {
     int32_t debug;    /* diagnostics only, 0 in production (debug modes disable warp roles; results  */
                       /*   invalid except bit 16 = exact K2 for every quad, no filter)               */
     int32_t flags;    /* EPI4_FLAG_* bits                                                          */
-    int32_t objective; /* EPI4_OBJ_K2 (default) or EPI4_OBJ_MI  */
+    int32_t objective; /* EPI4_OBJ_K2 (default), EPI4_OBJ_MI or EPI4_OBJ_CHI2 (§8(f) NEXT-4) */
 } epi4_opts;
 
 /* opts.flags: with world > 1, a load computes only this rank's contiguous share of the 3-way table T3
@@ -75,6 +75,12 @@ typedef struct {
  *     scored exactly.  epi4_search3 supports K2 only. */
 #define EPI4_OBJ_K2 0
 #define EPI4_OBJ_MI 1
+/*   EPI4_OBJ_CHI2: Pearson's chi-square of the 2 x 81 table (no continuity correction, cells with r_c > 0),
+ *     largest first, computed as X^2 = M*S/(n0 n1) - M with S = sum_{c: r_c>0} (r_c0^2 n1 + r_c1^2 n0) / r_c:
+ *     an exact integer numerator (uint64, < n0 n1 M), one correctly rounded double division per cell, summed in
+ *     canonical cell order; X^2 = 0 if a phenotype is empty.  The key in k2_out is -X^2.  epi4_load_* returns
+ *     EPI4_EINVAL if n0 n1 M >= 2^53 (the numerator would not be exact in double).  No fp32 filter. */
+#define EPI4_OBJ_CHI2 2
 
 /* Fill *opts with defaults (block 32, pipe TC, rank 0, world 1, grid 0). */
 void epi4_default_opts(epi4_opts* opts);

@@ -35,7 +35,8 @@ class Epi4:
         o.rank, o.world, o.grid = int(rank), int(world), int(grid)
         o.debug = int(debug)           # diagnostics only: disables warp roles, results invalid
         o.flags = (binding.EPI4_FLAG_SHARD_T3 if shard_t3 else 0) | (binding.EPI4_FLAG_T3_WINDOWED if t3_windowed else 0)
-        o.objective = {"k2": binding.EPI4_OBJ_K2, "mi": binding.EPI4_OBJ_MI}[objective]
+        o.objective = {"k2": binding.EPI4_OBJ_K2, "mi": binding.EPI4_OBJ_MI,
+                       "chi2": binding.EPI4_OBJ_CHI2}[objective]
         self.shard_t3 = bool(shard_t3) and int(world) > 1
         self.pipe, self.rank, self.world = pipe, int(rank), int(world)
         self.ctx = binding.epi4_create(device, o)

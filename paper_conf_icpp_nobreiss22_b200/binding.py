@@ -22,7 +22,7 @@ EPI4_PIPE_TC, EPI4_PIPE_LOP3 = 0, 1
 EPI4_PTR_HOST, EPI4_PTR_DEVICE = 0, 1
 EPI4_FLAG_SHARD_T3 = 1
 EPI4_FLAG_T3_WINDOWED = 2
-EPI4_OBJ_K2, EPI4_OBJ_MI = 0, 1
+EPI4_OBJ_K2, EPI4_OBJ_MI, EPI4_OBJ_CHI2 = 0, 1, 2
 EPI4_MAX_TOPK = 1024
 PIPES = {"tc": EPI4_PIPE_TC, "lop3": EPI4_PIPE_LOP3}
 

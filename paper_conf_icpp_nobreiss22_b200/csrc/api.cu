@@ -296,6 +296,11 @@ int finish_load(epi4_ctx* c) {
             c->np[1] >= ((int64_t)1 << (32 - dd.pk_shift)))
             return fail(EPI4_EINVAL, "n0=%lld / n1=%lld: counts are packed (control | case) into one 32-bit word, which "
                         "needs bits(n0) + bits(n1) <= 32 and each < 2^22", (long long)c->np[0], (long long)c->np[1]);
+        // chi-square: per-cell numerator r_c0^2 n1 + r_c1^2 n0 <= n0 n1 M must be exact in double (epi4.h)
+        if (c->opts.objective == EPI4_OBJ_CHI2 &&
+            (double)c->np[0] * (double)c->np[1] * (double)(c->np[0] + c->np[1]) >= 9007199254740992.0)
+            return fail(EPI4_EINVAL, "EPI4_OBJ_CHI2 needs n0 n1 M < 2^53 (n0=%lld, n1=%lld)", (long long)c->np[0],
+                        (long long)c->np[1]);
     }
     const int64_t n = c->n;
     CU(grow(c->T1, c->cap_T1, (size_t)n * 2 * sizeof(uint32_t)));
@@ -443,8 +448,8 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
     epi4_default_opts(&o);
     if (opts) o = *opts;
     if (o.block != EPI4_B) return fail(EPI4_EINVAL, "block=%d: only B=32 is supported", o.block);
-    if (o.objective != EPI4_OBJ_K2 && o.objective != EPI4_OBJ_MI)
-        return fail(EPI4_EINVAL, "objective=%d: EPI4_OBJ_K2 or EPI4_OBJ_MI", o.objective);
+    if (o.objective != EPI4_OBJ_K2 && o.objective != EPI4_OBJ_MI && o.objective != EPI4_OBJ_CHI2)
+        return fail(EPI4_EINVAL, "objective=%d: EPI4_OBJ_K2, EPI4_OBJ_MI or EPI4_OBJ_CHI2", o.objective);
     if (o.pipe != EPI4_PIPE_TC && o.pipe != EPI4_PIPE_LOP3) return fail(EPI4_EINVAL, "unknown pipe %d", o.pipe);
     if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return fail(EPI4_EINVAL, "bad rank/world %d/%d", o.rank, o.world);
     int ndev = 0;

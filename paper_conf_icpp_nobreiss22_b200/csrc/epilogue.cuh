@@ -198,6 +198,15 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
                 cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
+            } else if (MODE == 4) {
+                // Pearson chi-square (EPI4_OBJ_CHI2): S += (r0^2 n1 + r1^2 n0) / r_c over cells with r_c > 0,
+                // exact uint64 numerator, one correctly rounded division (oracle_chi2's order)
+                const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks, rc = r0 + r1;
+                if (rc) {
+                    const unsigned long long num = (unsigned long long)r0 * r0 * d.np[1] +
+                                                   (unsigned long long)r1 * r1 * d.np[0];
+                    kk = __dadd_rn(kk, __ddiv_rn(__ull2double_rn(num), __uint2double_rn(rc)));
+                }
             } else if (MODE == 3) {
                 // mutual information (EPI4_OBJ_MI): (X(r0) + X(r1)) - X(r0 + r1), X(k) = k ln k
                 const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
@@ -234,7 +243,12 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
     }
     consume(R2, 54);
     flt = fa + fb + fc;
-    k2 = MODE == 3 ? -__dadd_rn(kk, d.mi_const) : kk;   // MI: key = -M*I (largest MI first)
+    if (MODE == 4) {   // chi-square: X^2 = M S / (n0 n1) - M (0 with an empty phenotype); key = -X^2
+        const double n0 = __uint2double_rn(d.np[0]), n1 = __uint2double_rn(d.np[1]), M = __dadd_rn(n0, n1);
+        k2 = (d.np[0] == 0 || d.np[1] == 0) ? 0.0 : -__dsub_rn(__ddiv_rn(__dmul_rn(M, kk), __dmul_rn(n0, n1)), M);
+    } else {
+        k2 = MODE == 3 ? -__dadd_rn(kk, d.mi_const) : kk;   // MI: key = -M*I (largest MI first)
+    }
 }
 
 // exact K2 of one quad (double, canonical order) from its packed contraction counts; optionally dumps its 162
@@ -247,6 +261,7 @@ static __device__ __noinline__ double score_quad(const DevData& d, int w, int x,
     const QuadRanks q = quad_ranks(d, w, x, y, z);
     if (dump_row) quad_eval<2>(d, q, w, x, y, z, c16, flt, k2, dump_row);
     else if (d.objective == EPI4_OBJ_MI) quad_eval<3>(d, q, w, x, y, z, c16, flt, k2, nullptr);
+    else if (d.objective == EPI4_OBJ_CHI2) quad_eval<4>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;
 }

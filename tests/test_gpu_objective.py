@@ -1,6 +1,7 @@
 """Alternative objective: the search ranked by mutual information (EPI4_OBJ_MI),
 scored exactly for every quad on the GPU from the same host-built k ln k table and in the same canonical
-order as the oracle, so the keys are bit-identical; both pipes."""
+order as the oracle, so the keys are bit-identical; both pipes.  The same for Pearson chi-square
+(EPI4_OBJ_CHI2): exact integer numerators and one correctly rounded division per cell on both sides."""
 import numpy as np
 import pytest
 
@@ -21,6 +22,33 @@ def test_mi_search_matches_oracle(pipe, cfg, nsnp):
         idx, key = e.search(32)
     np.testing.assert_array_equal(idx, want_idx)
     np.testing.assert_array_equal(key, want_key)
+
+
+@pytest.mark.parametrize("pipe", ["tc", "lop3"])
+@pytest.mark.parametrize("cfg,nsnp", [("C1", None), ("C5", 24)])
+def test_chi2_search_matches_oracle(pipe, cfg, nsnp):
+    import paper_conf_icpp_nobreiss22_b200 as epi
+    d = datagen.make_config(cfg, n_snps=nsnp)
+    want_idx, want_key = oracle.search_chi2(d.geno, d.phen, top_k=32)
+    with epi.Epi4(0, pipe=pipe, objective="chi2") as e:
+        e.load_genotypes(d.geno, d.phen)
+        idx, key = e.search(32)
+    np.testing.assert_array_equal(idx, want_idx)
+    np.testing.assert_array_equal(key, want_key)
+
+
+def test_chi2_planted_quad_on_a_multi_tile_problem():
+    """N = 160 (several 128-SNP w-ranges, a ragged tail): the chi-square search's best quad is the planted one
+    and its key equals the oracle's chi-square of the oracle's table for that quad."""
+    import paper_conf_icpp_nobreiss22_b200 as epi
+    d = datagen.make_dataset(160, 4096, 4096, 77, planted=datagen.planted_quad_for(160), name="chi2-160")
+    with epi.Epi4(0, pipe="tc", objective="chi2") as e:
+        e.load_genotypes(d.geno, d.phen)
+        idx, key = e.search(4)
+    best = oracle.unpack_index(int(idx[0]))
+    assert best == tuple(d.planted)
+    t = oracle.tables(d.geno, d.phen, [list(best)])[0]
+    assert key[0] == -oracle.chi2(t)
 
 
 def test_mi_objective_rejected_by_the_third_order_search():
