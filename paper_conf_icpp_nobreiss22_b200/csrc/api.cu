@@ -166,6 +166,12 @@ DevData devdata(const epi4_ctx* c) {
     d.expl[0] = c->expl[0];
     d.expl[1] = c->expl[1];
     d.flt_off = filter_offset(c->np[0] + c->np[1]);
+    {
+        const double M = (double)(c->np[0] + c->np[1]);
+        d.chi_a = c->np[0] ? (float)(M / (double)c->np[0]) : 0.0f;
+        d.chi_b = c->np[1] ? (float)(M / (double)c->np[1]) : 0.0f;
+        d.chi_M = M;
+    }
     return d;
 }
 
@@ -711,8 +717,11 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.quads_done = c->d_counters + 1;
     sp.prof = c->d_counters + 16;
     sp.debug = c->opts.debug;
-    // debug 16: exact K2 for every quad; the fp32 filter bounds K2 only, other objectives are scored exactly
-    sp.use_filter = !(sp.debug & 16) && c->opts.objective == EPI4_OBJ_K2;
+    // debug 16: exact score for every quad.  K2: fp32 Stirling filter; chi-square: fp32 upper bound on X^2
+    // (both phenotypes non-empty); MI: every quad scored exactly
+    sp.use_filter = (sp.debug & 16) ? 0
+                    : c->opts.objective == EPI4_OBJ_K2 ? 1
+                    : (c->opts.objective == EPI4_OBJ_CHI2 && c->np[0] > 0 && c->np[1] > 0) ? 2 : 0;
 
     c->stats.launches = 0;
     CU(cudaEventRecord(c->ev[2], c->stream));

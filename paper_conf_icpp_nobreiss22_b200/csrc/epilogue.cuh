@@ -171,11 +171,32 @@ __device__ __forceinline__ void cell_T_acc(uint32_t v, uint32_t pks, uint32_t pk
     acc = fmaf(-h1, lg2_approx(f1), acc);
 }
 
+// ---- the fp32 chi-square filter (EPI4_OBJ_CHI2) ---------------------------------------------------------
+// X^2 + M = sum_{c} u_c with u_c = (r0^2 (M/n0) + r1^2 (M/n1)) / r_c (cells with r_c = 0 give 0: the
+// numerator is 0 and the divisor is clamped to 1).  In fp32 every count is exact (< 2^23, exponent-bit
+// conversion as in cell_T_acc), each u_c carries at most ~8 roundings (alpha/beta, 2 products, FMA, rcp.approx,
+// product; each <= 2^-23 relative), and the three running sums of positive terms add <= 29 more, so the
+// computed sum U satisfies |U - (X^2 + M)| <= 40 * 2^-23 (X^2 + M) < 2^-17 (X^2 + M).  The kernel scores a
+// quad exactly only if -(U (1 + 2^-12) - M) <= the current k-th best key: 2^-12 is 32x the bound.
+__device__ __forceinline__ float rcp_approx(float x) {
+    float y;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+template <bool PK16>
+__device__ __forceinline__ void cell_chi_acc(uint32_t v, uint32_t pks, uint32_t pkm, float ca, float cb, float& acc) {
+    const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
+    const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
+    const float f0 = m0 - 8388608.0f, f1 = m1 - 8388608.0f;     // r0, r1 (exact)
+    const float num = fmaf(f0 * ca, f0, (f1 * cb) * f1);
+    acc = fmaf(num, rcp_approx(fmaxf(f0 + f1, 1.0f)), acc);
+}
+
 // Per-quad evaluation from the 16 packed contraction counts c16[8a + 4b + 2c + d] of quad (w, x, y, z).
 // Slabs along w: R2 := M3(S_*) (the recovered (x, y, z) table); for A = AA, Aa: r_A = M3(S_A) is consumed
 // and subtracted from R2, which ends as r_aa = M3(S_*) - M3(S_AA) - M3(S_Aa) (linearity of the recovery,
 // PAPER.md:L126 applied on axis w).  Cells are consumed slab by slab in canonical order c = 27a + 9b + 3c + d.
-// MODE 0: the fp32 filter value A = sum T_c (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
+// MODE 0: the fp32 filter value A = sum T_c (above); MODE 5: the fp32 chi-square sum U ~ X^2 + M (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
 // L[r_c0]) - L[r_c1], K2 += t_c, c = 0..80 (reading #4); MODE 2: exact K2 and the
 // 2 x 81 cells written to dump (controls first).
 template <int MODE, bool PK16 = false>
@@ -198,6 +219,8 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
                 cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
+            } else if (MODE == 5) {
+                cell_chi_acc<PK16>(S[c], pks, pkm, d.chi_a, d.chi_b, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
             } else if (MODE == 4) {
                 // Pearson chi-square (EPI4_OBJ_CHI2): S += (r0^2 n1 + r1^2 n0) / r_c over cells with r_c > 0,
                 // exact uint64 numerator, one correctly rounded division (oracle_chi2's order)

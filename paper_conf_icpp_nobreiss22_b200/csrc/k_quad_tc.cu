@@ -368,7 +368,7 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 // issuers may issue (and complete) the steps of the other parity out of order, so a waiter is only protected
 // from phase aliasing if its previous wait on a ring was on the same issuer's steps: both ring sizes must be
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
-template <int SA, int SB, bool PK16>
+template <int SA, int SB, bool PK16, int FILT>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     static_assert(tc::MMA_ISSUERS == 1 ||
                   (SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2),
@@ -792,12 +792,17 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     if (dump) {
                         key = score_quad(d, w, ti.x, y, ti.z, c16, dump);
                     } else if (sp.use_filter) {
-                        // fp32 Stirling filter (epilogue.cuh); only possible top-k members get the exact K2
+                        // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
+                        // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2)
                         float flt;
                         double unused;
-                        quad_eval<0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt, unused, nullptr);
+                        quad_eval<FILT == 1 ? 5 : 0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt,
+                                                           unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
-                        offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
+                        if (FILT == 1)
+                            offer = d.chi_M - (double)flt * (1.0 + 1.0 / 4096.0) <= thr;
+                        else
+                            offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
                             // rare path: the noinline exact scorer takes the counts through local memory
                             key = score_quad(d, w, ti.x, y, ti.z, c16, nullptr);
@@ -847,9 +852,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 #endif
 }
 
-template <int SA, int SB, bool PK16>
+template <int SA, int SB, bool PK16, int FILT>
 static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
-    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16, FILT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
@@ -863,7 +868,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16>, sp);
+    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16, FILT>, sp);
 }
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
@@ -896,16 +901,18 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
                 tc::PROD_WARPS, pick.sa, pick.sb, tc::A_SPLIT, sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
     const bool pk16 = sp.d.pk_shift == 16;
+    const bool chi = sp.use_filter == 2;   // FILT 1: the chi-square filter
+#define EPI4_LAUNCH(A_, B_)                                                                        \
+    e = chi ? (pk16 ? launch_cfg<A_, B_, true, 1>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1>(sp, smem, grid, s)) \
+            : (pk16 ? launch_cfg<A_, B_, true, 0>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0>(sp, smem, grid, s))
     if (pick.sa == 5 && pick.sb == 3) {
-        if constexpr (tc::MMA_ISSUERS == 1)
-            e = pk16 ? launch_cfg<5, 3, true>(sp, smem, grid, s) : launch_cfg<5, 3, false>(sp, smem, grid, s);
-    } else if (pick.sa == 4 && pick.sb == 6) {
-        e = pk16 ? launch_cfg<4, 6, true>(sp, smem, grid, s) : launch_cfg<4, 6, false>(sp, smem, grid, s);
-    } else if (pick.sa == 6 && pick.sb == 2) {
-        e = pk16 ? launch_cfg<6, 2, true>(sp, smem, grid, s) : launch_cfg<6, 2, false>(sp, smem, grid, s);
-    } else if (pick.sa == 4 && pick.sb == 4) e = pk16 ? launch_cfg<4, 4, true>(sp, smem, grid, s) : launch_cfg<4, 4, false>(sp, smem, grid, s);
-    else if (pick.sa == 4 && pick.sb == 2) e = pk16 ? launch_cfg<4, 2, true>(sp, smem, grid, s) : launch_cfg<4, 2, false>(sp, smem, grid, s);
-    else if (pick.sa == 2 && pick.sb == 2) e = pk16 ? launch_cfg<2, 2, true>(sp, smem, grid, s) : launch_cfg<2, 2, false>(sp, smem, grid, s);
+        if constexpr (tc::MMA_ISSUERS == 1) EPI4_LAUNCH(5, 3);
+    } else if (pick.sa == 4 && pick.sb == 6) EPI4_LAUNCH(4, 6);
+    else if (pick.sa == 6 && pick.sb == 2) EPI4_LAUNCH(6, 2);
+    else if (pick.sa == 4 && pick.sb == 4) EPI4_LAUNCH(4, 4);
+    else if (pick.sa == 4 && pick.sb == 2) EPI4_LAUNCH(4, 2);
+    else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
+#undef EPI4_LAUNCH
     if (launches) ++*launches;
     return e;
 }

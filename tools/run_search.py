@@ -16,14 +16,15 @@ ap.add_argument("--top-k", type=int, default=16)
 ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--debug", type=int, default=0)
 ap.add_argument("--grid", type=int, default=0)
+ap.add_argument("--objective", default="k2", choices=["k2", "mi", "chi2"])
 a = ap.parse_args()
 d = datagen.make_config(a.config)
-with epi.Epi4(0, pipe=a.pipe, debug=a.debug, grid=a.grid) as e:
+with epi.Epi4(0, pipe=a.pipe, debug=a.debug, grid=a.grid, objective=a.objective) as e:
     e.load_genotypes(d.geno, d.phen)
     for _ in range(a.repeat):
         t0 = time.time()
         idx, k2 = e.search_units(0, a.units, a.top_k) if a.units >= 0 else e.search(a.top_k)
         st = e.stats()
         best = (epi.unpack_index(idx[0]), float(k2[0])) if len(idx) else None
-        print(f"{a.config} {a.pipe} dbg={a.debug}: best {best} quad {st['ms_quad']:.2f} ms "
+        print(f"{a.config} {a.pipe} {a.objective} dbg={a.debug}: best {best} quad {st['ms_quad']:.2f} ms "
               f"tiles {st['tiles']} quads {st['quads']} wall {time.time() - t0:.2f}s prof {[f'{v:.3g}' for v in st['prof']]}", flush=True)
