@@ -71,15 +71,16 @@ typedef struct {
  *   EPI4_OBJ_MI: mutual information between the quad's 81-cell genotype and the phenotype, largest first.
  *     Computed exactly as M*I = sum_c [(X(r_c0) + X(r_c1)) - X(r_c)] + (X(M) - X(n0) - X(n1)) with
  *     X(k) = k ln k (X(0) = 0) from a host-built double table, summed in canonical cell order; the key
- *     returned in k2_out is -M*I (so "smallest key first" ranks by largest MI).  No fp32 filter: every quad is
- *     scored exactly.  epi4_search3 supports K2 only. */
+ *     returned in k2_out is -M*I (so "smallest key first" ranks by largest MI).  The tensor-core pipe skips
+ *     quads whose fp32 upper bound on M*I cannot reach the top-k (rigorous rounding bound; exact result).  epi4_search3 supports K2 only. */
 #define EPI4_OBJ_K2 0
 #define EPI4_OBJ_MI 1
 /*   EPI4_OBJ_CHI2: Pearson's chi-square of the 2 x 81 table (no continuity correction, cells with r_c > 0),
  *     largest first, computed as X^2 = M*S/(n0 n1) - M with S = sum_{c: r_c>0} (r_c0^2 n1 + r_c1^2 n0) / r_c:
  *     an exact integer numerator (uint64, < n0 n1 M), one correctly rounded double division per cell, summed in
  *     canonical cell order; X^2 = 0 if a phenotype is empty.  The key in k2_out is -X^2.  epi4_load_* returns
- *     EPI4_EINVAL if n0 n1 M >= 2^53 (the numerator would not be exact in double).  No fp32 filter. */
+ *     EPI4_EINVAL if n0 n1 M >= 2^53 (the numerator would not be exact in double).  The tensor-core
+ *     pipe skips quads whose fp32 upper bound on X^2 cannot reach the top-k (exact result). */
 #define EPI4_OBJ_CHI2 2
 
 /* Fill *opts with defaults (block 32, pipe TC, rank 0, world 1, grid 0). */

@@ -171,6 +171,12 @@ DevData devdata(const epi4_ctx* c) {
         d.chi_a = c->np[0] ? (float)(M / (double)c->np[0]) : 0.0f;
         d.chi_b = c->np[1] ? (float)(M / (double)c->np[1]) : 0.0f;
         d.chi_M = M;
+        // MI filter bound (epilogue.cuh cell_mi): lg2.approx calls (coefficients sum to 2M), the three
+        // roundings of each cell (each <= u * r_c lg2 r_c, sum <= 3 u M lg2 M), and 29 additions of the cell
+        // values (|cell| <= r_c bits, so the partial sums are <= M); doubled, as for the K2 filter
+        const double u = std::ldexp(1.0, -24), l2M = std::log2(M + 2.0);
+        d.mi_E = 2.0 * (std::ldexp(1.0, -21) * std::max(1.0, l2M) * (2.0 * M + 243.0) + 3.0 * u * (M + 81.0) * l2M +
+                        29.0 * u * (M + 81.0));
     }
     return d;
 }
@@ -718,10 +724,11 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.prof = c->d_counters + 16;
     sp.debug = c->opts.debug;
     // debug 16: exact score for every quad.  K2: fp32 Stirling filter; chi-square: fp32 upper bound on X^2
-    // (both phenotypes non-empty); MI: every quad scored exactly
+    // (both phenotypes non-empty); MI: fp32 upper bound on M*I
     sp.use_filter = (sp.debug & 16) ? 0
                     : c->opts.objective == EPI4_OBJ_K2 ? 1
-                    : (c->opts.objective == EPI4_OBJ_CHI2 && c->np[0] > 0 && c->np[1] > 0) ? 2 : 0;
+                    : (c->opts.objective == EPI4_OBJ_CHI2 && c->np[0] > 0 && c->np[1] > 0) ? 2
+                    : c->opts.objective == EPI4_OBJ_MI ? 3 : 0;
 
     c->stats.launches = 0;
     CU(cudaEventRecord(c->ev[2], c->stream));

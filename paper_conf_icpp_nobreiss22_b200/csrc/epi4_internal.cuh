@@ -82,6 +82,7 @@ struct DevData {
     double flt_off;              // fp32 K2 filter: exact-score a quad iff ln2 A + flt_off <= threshold (epilogue.cuh)
     float chi_a, chi_b;          // fp32 chi-square filter: M / n0, M / n1 (epilogue.cuh, cell_chi_acc)
     double chi_M;                // M
+    double mi_E;                 // fp32 MI filter: rounding bound (bits) on V = sum_c [X2(r0) + X2(r1) - X2(r_c)]
 };
 
 // byte offset of (fp4 chunk C, row r = 2 snp + g) in expl: blocked [chunk pair][128-row block][C & 1][row][128 B]
@@ -156,7 +157,8 @@ struct SearchParams {
     unsigned long long* quads_done;   // useful quads evaluated (atomicAdd once per CTA)
     unsigned long long* prof;  // [16] diagnostics: [0] exact K2 evaluations, [1..] per-role cycle counters
     int32_t use_filter;        // fp32 filter before the exact double score: 1 = Stirling K2 filter, 2 = chi-square
-                               // upper bound (EPI4_OBJ_CHI2) (epilogue.cuh); 0 = every quad scored exactly
+                               // upper bound (EPI4_OBJ_CHI2), 3 = MI upper bound (EPI4_OBJ_MI) (epilogue.cuh);
+                               // 0 = every quad scored exactly
 
     int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA,
                                // 128 no A copies (16: exact K2 for every quad, 64: trace)

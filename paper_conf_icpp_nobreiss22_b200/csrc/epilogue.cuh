@@ -192,11 +192,27 @@ __device__ __forceinline__ void cell_chi_acc(uint32_t v, uint32_t pks, uint32_t 
     acc = fmaf(num, rcp_approx(fmaxf(f0 + f1, 1.0f)), acc);
 }
 
+// ---- the fp32 mutual-information filter (EPI4_OBJ_MI) ----------------------------------------------------
+// M*I = ln2 V + mi_const with V = sum_c [X2(r0) + X2(r1) - X2(r_c)], X2(k) = k lg2 k (X2(0) = 0: lg2 of
+// max(k, 1)).  Each cell value is formed first (two FMAs onto -r_c lg2 r_c; |value| <= r_c bits), then added
+// to a running sum, so |V_computed - V| <= mi_E (api.cu: lg2.approx, the cell roundings, the additions).
+// The kernel scores a quad exactly only if -(ln2 (V + mi_E) + mi_const) <= the current k-th best key.
+template <bool PK16>
+__device__ __forceinline__ void cell_mi_acc(uint32_t v, uint32_t pks, uint32_t pkm, float& acc) {
+    const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
+    const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
+    const float f0 = m0 - 8388608.0f, f1 = m1 - 8388608.0f, fn = f0 + f1;   // r0, r1, r_c (exact)
+    const float cell = fmaf(f0, lg2_approx(fmaxf(f0, 1.0f)), fmaf(f1, lg2_approx(fmaxf(f1, 1.0f)),
+                                                                  -fn * lg2_approx(fmaxf(fn, 1.0f))));
+    acc += cell;
+}
+
 // Per-quad evaluation from the 16 packed contraction counts c16[8a + 4b + 2c + d] of quad (w, x, y, z).
 // Slabs along w: R2 := M3(S_*) (the recovered (x, y, z) table); for A = AA, Aa: r_A = M3(S_A) is consumed
 // and subtracted from R2, which ends as r_aa = M3(S_*) - M3(S_AA) - M3(S_Aa) (linearity of the recovery,
 // PAPER.md:L126 applied on axis w).  Cells are consumed slab by slab in canonical order c = 27a + 9b + 3c + d.
-// MODE 0: the fp32 filter value A = sum T_c (above); MODE 5: the fp32 chi-square sum U ~ X^2 + M (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
+// MODE 0: the fp32 filter value A = sum T_c (above); MODE 5: the fp32 chi-square sum U ~ X^2 + M (above);
+// MODE 6: the fp32 MI sum V (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
 // L[r_c0]) - L[r_c1], K2 += t_c, c = 0..80 (reading #4); MODE 2: exact K2 and the
 // 2 x 81 cells written to dump (controls first).
 template <int MODE, bool PK16 = false>
@@ -219,6 +235,8 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
                 cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
+            } else if (MODE == 6) {
+                cell_mi_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
             } else if (MODE == 5) {
                 cell_chi_acc<PK16>(S[c], pks, pkm, d.chi_a, d.chi_b, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
             } else if (MODE == 4) {

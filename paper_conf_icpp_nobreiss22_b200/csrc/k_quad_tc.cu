@@ -793,14 +793,17 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         key = score_quad(d, w, ti.x, y, ti.z, c16, dump);
                     } else if (sp.use_filter) {
                         // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
-                        // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2)
+                        // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2); FILT 2: MI
+                        // upper bound (key = -M*I)
                         float flt;
                         double unused;
-                        quad_eval<FILT == 1 ? 5 : 0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt,
+                        quad_eval<FILT == 1 ? 5 : FILT == 2 ? 6 : 0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt,
                                                            unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
                         if (FILT == 1)
                             offer = d.chi_M - (double)flt * (1.0 + 1.0 / 4096.0) <= thr;
+                        else if (FILT == 2)
+                            offer = -(((double)flt + d.mi_E) * 0.69314718055994530942 + d.mi_const) <= thr;
                         else
                             offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
@@ -901,10 +904,11 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
                 tc::PROD_WARPS, pick.sa, pick.sb, tc::A_SPLIT, sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
     const bool pk16 = sp.d.pk_shift == 16;
-    const bool chi = sp.use_filter == 2;   // FILT 1: the chi-square filter
+    const int filt = sp.use_filter == 2 ? 1 : sp.use_filter == 3 ? 2 : 0;   // FILT 1: chi-square, 2: MI
 #define EPI4_LAUNCH(A_, B_)                                                                        \
-    e = chi ? (pk16 ? launch_cfg<A_, B_, true, 1>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1>(sp, smem, grid, s)) \
-            : (pk16 ? launch_cfg<A_, B_, true, 0>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0>(sp, smem, grid, s))
+    e = filt == 1 ? (pk16 ? launch_cfg<A_, B_, true, 1>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1>(sp, smem, grid, s)) \
+      : filt == 2 ? (pk16 ? launch_cfg<A_, B_, true, 2>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 2>(sp, smem, grid, s)) \
+                  : (pk16 ? launch_cfg<A_, B_, true, 0>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0>(sp, smem, grid, s))
     if (pick.sa == 5 && pick.sb == 3) {
         if constexpr (tc::MMA_ISSUERS == 1) EPI4_LAUNCH(5, 3);
     } else if (pick.sa == 4 && pick.sb == 6) EPI4_LAUNCH(4, 6);

@@ -51,20 +51,21 @@ def test_chi2_planted_quad_on_a_multi_tile_problem():
     assert key[0] == -oracle.chi2(t)
 
 
+@pytest.mark.parametrize("objective", ["chi2", "mi"])
 @pytest.mark.parametrize("cfg,nsnp,k", [("C5", 32, 64), ("C2", 48, 1024)])
-def test_chi2_fp32_filter_keeps_exact_topk(cfg, nsnp, k):
-    """The tensor-core epilogue scores a quad's exact chi-square only when its fp32 upper bound on X^2 can beat
-    the CTA's k-th best key (epilogue.cuh, cell_chi_acc).  With a large k (a loose threshold for most of the
+def test_fp32_objective_filter_keeps_exact_topk(objective, cfg, nsnp, k):
+    """The tensor-core epilogue scores a quad's exact chi-square / MI only when its fp32 upper bound on X^2 /
+    M*I can beat the CTA's k-th best key (epilogue.cuh, cell_chi_acc / cell_mi_acc).  With a large k (a loose threshold for most of the
     run) and the largest M (C5, unbalanced), the top-k must equal the oracle's and the unfiltered run's
     (debug flag 16: exact score for every quad), and the filter must have skipped quads."""
     import paper_conf_icpp_nobreiss22_b200 as epi
     d = datagen.make_config(cfg, n_snps=nsnp, planted=False)
-    ref_idx, ref_key = oracle.search_chi2(d.geno, d.phen, top_k=k)
-    with epi.Epi4(0, pipe="tc", objective="chi2") as e:
+    ref_idx, ref_key = (oracle.search_chi2 if objective == "chi2" else oracle.search_mi)(d.geno, d.phen, top_k=k)
+    with epi.Epi4(0, pipe="tc", objective=objective) as e:
         e.load_genotypes(d.geno, d.phen)
         idx, key = e.search(k)
         n_exact = e.stats()["prof"][0]
-    with epi.Epi4(0, pipe="tc", objective="chi2", debug=16) as e:
+    with epi.Epi4(0, pipe="tc", objective=objective, debug=16) as e:
         e.load_genotypes(d.geno, d.phen)
         idx_u, key_u = e.search(k)
     np.testing.assert_array_equal(idx, ref_idx)
