@@ -72,7 +72,8 @@ typedef struct {
  *     Computed exactly as M*I = sum_c [(X(r_c0) + X(r_c1)) - X(r_c)] + (X(M) - X(n0) - X(n1)) with
  *     X(k) = k ln k (X(0) = 0) from a host-built double table, summed in canonical cell order; the key
  *     returned in k2_out is -M*I (so "smallest key first" ranks by largest MI).  The tensor-core pipe skips
- *     quads whose fp32 upper bound on M*I cannot reach the top-k (rigorous rounding bound; exact result).  epi4_search3 supports K2 only. */
+ *     quads whose fp32 upper bound on M*I cannot reach the top-k (rigorous rounding bound; exact result).
+ *     epi4_search3 supports K2 only. */
 #define EPI4_OBJ_K2 0
 #define EPI4_OBJ_MI 1
 /*   EPI4_OBJ_CHI2: Pearson's chi-square of the 2 x 81 table (no continuity correction, cells with r_c > 0),
