@@ -87,3 +87,15 @@ def test_merge_topk_orders_by_key_then_index():
     idx, k2 = epi.merge_topk(parts, 4)
     assert list(idx) == [9, 2, 5, 3]
     assert list(k2) == [0.5, 1.0, 1.0, 2.0]
+
+
+def test_binding_constants_match_the_header():
+    """Every EPI4_* integer #define in include/epi4.h that the binding mirrors has the same value."""
+    import os
+    import re
+    hdr = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include", "epi4.h")).read()
+    defs = {m.group(1): int(m.group(2), 0) for m in re.finditer(r"#define\s+(EPI4_\w+)\s+\(?(-?(?:0x)?[0-9A-Fa-f]+)\)?", hdr)}
+    for name in ("EPI4_OBJ_K2", "EPI4_OBJ_MI", "EPI4_OBJ_CHI2", "EPI4_FLAG_SHARD_T3", "EPI4_FLAG_T3_WINDOWED",
+                 "EPI4_EINVAL", "EPI4_ENODEV", "EPI4_PIPE_TC", "EPI4_PIPE_LOP3"):
+        assert name in defs, name
+        assert getattr(binding, name) == defs[name], name
