@@ -63,6 +63,10 @@ def _load():
         lib.oracle_chi2.argtypes = [P]
         lib.oracle_search_chi2.restype = ctypes.c_int
         lib.oracle_search_chi2.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, P, P, P]
+        lib.oracle_score3_obj.restype = ctypes.c_double
+        lib.oracle_score3_obj.argtypes = [P, ctypes.c_int32]
+        lib.oracle_search3_obj.restype = ctypes.c_int
+        lib.oracle_search3_obj.argtypes = [P, P, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, P, P, P]
         lib.oracle_max_threads.restype = ctypes.c_int32
         lib.oracle_max_threads.argtypes = [ctypes.c_int32]
         _lib = lib
@@ -204,6 +208,31 @@ def search3(geno, phen, top_k: int = 1, n_snps: int | None = None, n_threads: in
     if rc:
         raise ValueError(f"oracle_search3 failed: {rc}")
     return idx[: nout[0]], k2v[: nout[0]]
+
+
+_OBJ3 = {"mi": 1, "chi2": 2}
+
+
+def score3(table, objective: str) -> float:
+    """M * I ("mi") or Pearson X^2 ("chi2") of a 2 x 27 triple table."""
+    t = np.ascontiguousarray(np.asarray(table, dtype=np.uint32).reshape(2, 27))
+    return float(_load().oracle_score3_obj(_ptr(t), _OBJ3[objective]))
+
+
+def search3_obj(geno, phen, objective: str, top_k: int = 1, n_snps: int | None = None):
+    """Exhaustive third-order search ranked by "mi" or "chi2" (SURVEY.md §8(f) NEXT-3 x NEXT-4) -> (packed idx,
+    key = -score), the top_k smallest keys ascending (single-threaded: for small test problems)."""
+    geno, phen = _prep(geno, phen)
+    n = geno.shape[0] if n_snps is None else int(n_snps)
+    geno = np.ascontiguousarray(geno[:n])
+    idx = np.zeros(top_k, dtype=np.uint64)
+    key = np.zeros(top_k, dtype=np.float64)
+    nout = np.zeros(1, dtype=np.int32)
+    rc = _load().oracle_search3_obj(_ptr(geno), _ptr(phen), n, geno.shape[1], int(top_k), _OBJ3[objective],
+                                    _ptr(idx), _ptr(key), _ptr(nout))
+    if rc:
+        raise ValueError(f"oracle_search3_obj failed: {rc}")
+    return idx[: nout[0]], key[: nout[0]]
 
 
 def max_threads(n_threads: int = 0) -> int:

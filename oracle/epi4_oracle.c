@@ -369,3 +369,53 @@ int32_t oracle_max_threads(int32_t n_threads) {
     return 1;
 #endif
 }
+
+/* ---- third-order search with the alternative objectives (SURVEY.md §8(f) NEXT-3 x NEXT-4) ---------------
+ * The same definitions as oracle_mi / oracle_chi2 on the 2 x 27 table of a triple (cell 9a + 3b + c), in
+ * canonical cell order: objective 1 = mutual information (key -M*I), 2 = Pearson chi-square (key -X^2);
+ * top-k smallest (key, index) with index = i<<48 | j<<32 | k<<16.  Single-threaded (small test problems). */
+static double mi_27(const uint32_t *r) {
+    uint32_t n0 = 0, n1 = 0;
+    for (int c = 0; c < NCELL3; ++c) { n0 += r[c]; n1 += r[NCELL3 + c]; }
+    double acc = 0.0;
+    for (int c = 0; c < NCELL3; ++c) {
+        uint32_t r0 = r[c], r1 = r[NCELL3 + c];
+        acc = acc + ((xlogx(r0) + xlogx(r1)) - xlogx(r0 + r1));
+    }
+    const double M = (double)(n0 + n1);
+    const double cst = (M > 0 ? M * log(M) : 0.0) - xlogx(n0) - xlogx(n1);
+    return acc + cst;
+}
+static double chi2_27(const uint32_t *r) {
+    uint32_t n0 = 0, n1 = 0;
+    for (int c = 0; c < NCELL3; ++c) { n0 += r[c]; n1 += r[NCELL3 + c]; }
+    if (n0 == 0 || n1 == 0) return 0.0;
+    double s = 0.0;
+    for (int c = 0; c < NCELL3; ++c) {
+        const uint64_t r0 = r[c], r1 = r[NCELL3 + c], rc = r0 + r1;
+        if (rc == 0) continue;
+        const uint64_t num = r0 * r0 * n1 + r1 * r1 * n0;
+        s = s + (double)num / (double)rc;
+    }
+    const double M = (double)n0 + (double)n1;
+    return (M * s) / ((double)n0 * (double)n1) - M;
+}
+double oracle_score3_obj(const uint32_t *r, int32_t objective) {
+    return objective == 1 ? mi_27(r) : objective == 2 ? chi2_27(r) : k2_27(r);
+}
+int oracle_search3_obj(const uint8_t *geno, const uint8_t *phen, int32_t n, int64_t m, int32_t top_k,
+                       int32_t objective, uint64_t *idx_out, double *key_out, int32_t *n_out) {
+    int rc = validate(geno, phen, n, m);
+    if (rc) return rc;
+    if (top_k < 1 || objective < 1 || objective > 2) return -5;
+    int32_t len = 0;
+    uint32_t r[2 * NCELL3];
+    for (int32_t i = 0; i < n; ++i)
+        for (int32_t j = i + 1; j < n; ++j)
+            for (int32_t k = j + 1; k < n; ++k) {
+                count_triple(geno, phen, m, i, j, k, r);
+                topk_insert(key_out, idx_out, &len, top_k, -oracle_score3_obj(r, objective), oracle_pack(i, j, k, 0));
+            }
+    *n_out = len;
+    return 0;
+}

@@ -137,3 +137,24 @@ def test_chi2_search_recovers_planted_quad():
     d = datagen.make_config("C1")
     idx, _ = oracle.search_chi2(d.geno, d.phen, top_k=1)
     assert oracle.unpack_index(int(idx[0])) == tuple(d.planted)
+
+
+# ---- third-order search with the alternative objectives (NEXT-3 x NEXT-4) ---------------------------------
+def test_triple_objectives_match_scipy_and_definition():
+    d = datagen.make_config("C5", n_snps=10)
+    for t in oracle.tables3(d.geno, d.phen, [[0, 1, 2], [2, 5, 9], [1, 4, 7]]):
+        want = _chi2_scipy(t)
+        assert abs(oracle.score3(t, "chi2") - want) < 1e-10 * max(1.0, want)
+        want = _mi_numpy(t)
+        assert abs(oracle.score3(t, "mi") - want) < 1e-9 * max(1.0, abs(want))
+
+
+def test_triple_objective_search_equals_scipy_ranking():
+    d = datagen.make_dataset(12, 30, 34, 8, planted=None, name="tiny3obj")
+    tri = list(itertools.combinations(range(12), 3))
+    tabs = oracle.tables3(d.geno, d.phen, tri)
+    for obj, f in (("chi2", _chi2_scipy), ("mi", _mi_numpy)):
+        keys = sorted((-f(t), oracle.pack_index(i, j, k, 0)) for t, (i, j, k) in zip(tabs, tri))
+        idx, key = oracle.search3_obj(d.geno, d.phen, obj, top_k=8)
+        np.testing.assert_allclose(key, [k[0] for k in keys[:8]], rtol=1e-9)
+        assert set(int(v) for v in idx[:5]) <= set(k[1] for k in keys[:8])
