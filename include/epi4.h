@@ -73,7 +73,7 @@ typedef struct {
  *     X(k) = k ln k (X(0) = 0) from a host-built double table, summed in canonical cell order; the key
  *     returned in k2_out is -M*I (so "smallest key first" ranks by largest MI).  The tensor-core pipe skips
  *     quads whose fp32 upper bound on M*I cannot reach the top-k (rigorous rounding bound; exact result).
- *     epi4_search3 supports K2 only. */
+ *     epi4_search3 ranks triples by the same objective (27 cells, exact, no filter). */
 #define EPI4_OBJ_K2 0
 #define EPI4_OBJ_MI 1
 /*   EPI4_OBJ_CHI2: Pearson's chi-square of the 2 x 81 table (no continuity correction, cells with r_c > 0),
@@ -130,7 +130,7 @@ int epi4_search_units(epi4_ctx* ctx, int64_t unit_begin, int64_t unit_end, int32
 /* Third-order search (the paper's predecessors): every triple
  * i < j < k of this rank's share (the 4-way plan's units, rank/world as for epi4_search), its 2 x 27 table
  * (8 non-aa counts on the tensor cores against an all-ones SNP, the other 19 recovered from T2/T1/n as in
- * PAPER.md:L126) scored by K2 over 27 cells in double, canonical order c = 9a + 3b + c.  Output as
+ * PAPER.md:L126) scored by K2 (or opts.objective) over 27 cells in double, canonical order c = 9a + 3b + c.  Output as
  * epi4_search: the top_k smallest (K2, index) keys ascending, index = i<<48 | j<<32 | k<<16.
  * Tensor-core pipe only (EPI4_EINVAL otherwise); host arrays of top_k entries. */
 int epi4_search3(epi4_ctx* ctx, int32_t top_k, uint64_t* triples_out, double* k2_out, int32_t* n_out);

@@ -809,7 +809,6 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
     if (c->opts.pipe != EPI4_PIPE_TC) return fail(EPI4_EINVAL, "the third-order search runs on the tensor-core pipe");
-    if (c->opts.objective != EPI4_OBJ_K2) return fail(EPI4_EINVAL, "the third-order search scores K2 only");
     if (c->n < 3) return fail(EPI4_EINVAL, "N=%d < 3", c->n);
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!triples_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");

@@ -306,10 +306,21 @@ static __device__ __noinline__ double score_quad(const DevData& d, int w, int x,
     else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;
 }
+// Call-site wrapper for the hot loops: the counts are copied into an array local to the (rare) branch that
+// calls the noinline scorer, so the loop's own c16 never has its address taken and stays in registers (passing
+// c16 itself made the compiler store all 16 counts to the stack on every quad: 1.5 G STL per C2 slice, ncu).
+static __device__ __forceinline__ double score_quad_rare(const DevData& d, int w, int x, int y, int z,
+                                                         const uint32_t (&c16)[16], uint32_t* dump_row) {
+    uint32_t t[16];
+#pragma unroll
+    for (int k = 0; k < 16; ++k) t[k] = c16[k];
+    return score_quad(d, w, x, y, z, t, dump_row);
+}
 // Third-order search: exact K2 of triple w < x < y from its 8 packed non-aa counts
 // c8[4a + 2b + c] (the 3-way-table mode's d = AA columns), the same recovery one order lower: generalized
 // cells S[9a + 3b + c] (digit 2 = '*') from c8, T2, T1 and n, aa recovered on the three axes,
-// K2 = sum_c ((L[r_c + 1] - L[r_c0]) - L[r_c1]) in canonical order c = 9a + 3b + c (reading #4).
+// K2 = sum_c ((L[r_c + 1] - L[r_c0]) - L[r_c1]) in canonical order c = 9a + 3b + c (reading #4); with
+// EPI4_OBJ_MI / EPI4_OBJ_CHI2 the key is -M*I / -X^2 of the 2 x 27 table, as in quad_eval MODE 3 / 4.
 static __device__ __noinline__ double score_triple(const DevData& d, int w, int x, int y, const uint32_t (&c8)[8]) {
     const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
     const uint4 pwx = t2_all(d, c2(x) + w), pwy = t2_all(d, c2(y) + w), pxy = t2_all(d, c2(y) + x);
@@ -336,6 +347,28 @@ static __device__ __noinline__ double score_triple(const DevData& d, int w, int 
     }
     mobius3(S);
     double kk = 0.0;
+    if (d.objective == EPI4_OBJ_MI) {   // -M*I over the 27 cells (oracle mi_27's order)
+#pragma unroll
+        for (int c = 0; c < 27; ++c) {
+            const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+            kk = __dadd_rn(kk, __dsub_rn(__dadd_rn(__ldg(d.xlx + r0), __ldg(d.xlx + r1)), __ldg(d.xlx + (r0 + r1))));
+        }
+        return -__dadd_rn(kk, d.mi_const);
+    }
+    if (d.objective == EPI4_OBJ_CHI2) {   // -X^2 over the 27 cells (oracle chi2_27's order)
+        if (d.np[0] == 0 || d.np[1] == 0) return 0.0;
+#pragma unroll
+        for (int c = 0; c < 27; ++c) {
+            const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks, rc = r0 + r1;
+            if (rc) {
+                const unsigned long long num = (unsigned long long)r0 * r0 * d.np[1] +
+                                               (unsigned long long)r1 * r1 * d.np[0];
+                kk = __dadd_rn(kk, __ddiv_rn(__ull2double_rn(num), __uint2double_rn(rc)));
+            }
+        }
+        const double n0 = __uint2double_rn(d.np[0]), n1 = __uint2double_rn(d.np[1]), M = __dadd_rn(n0, n1);
+        return -__dsub_rn(__ddiv_rn(__dmul_rn(M, kk), __dmul_rn(n0, n1)), M);
+    }
 #pragma unroll
     for (int c = 0; c < 27; ++c) {
         const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;

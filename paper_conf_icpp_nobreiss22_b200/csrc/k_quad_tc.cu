@@ -790,7 +790,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     uint32_t* dump = sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
                     offer = true;
                     if (dump) {
-                        key = score_quad(d, w, ti.x, y, ti.z, c16, dump);
+                        key = score_quad_rare(d, w, ti.x, y, ti.z, c16, dump);
                     } else if (sp.use_filter) {
                         // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
                         // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2); FILT 2: MI
@@ -808,11 +808,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                             offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
                             // rare path: the noinline exact scorer takes the counts through local memory
-                            key = score_quad(d, w, ti.x, y, ti.z, c16, nullptr);
+                            key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
                             ++n_exact;
                         }
                     } else {
-                        key = score_quad(d, w, ti.x, y, ti.z, c16, nullptr);
+                        key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
                     }
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;

@@ -76,10 +76,15 @@ def test_fp32_objective_filter_keeps_exact_topk(objective, cfg, nsnp, k):
     assert k <= n_exact < nq
 
 
-def test_mi_objective_rejected_by_the_third_order_search():
+@pytest.mark.parametrize("objective", ["mi", "chi2"])
+@pytest.mark.parametrize("cfg,nsnp,k", [("C1", None, 64), ("C5", 40, 32), ("C2", 100, 16)])
+def test_search3_objectives_match_oracle(objective, cfg, nsnp, k):
+    """Third-order search ranked by MI / chi-square: keys bit-identical to oracle.search3_obj."""
     import paper_conf_icpp_nobreiss22_b200 as epi
-    d = datagen.make_config("C1")
-    with epi.Epi4(0, pipe="tc", objective="mi") as e:
+    d = datagen.make_config(cfg, n_snps=nsnp)
+    want_idx, want_key = oracle.search3_obj(d.geno, d.phen, objective, top_k=k)
+    with epi.Epi4(0, pipe="tc", objective=objective) as e:
         e.load_genotypes(d.geno, d.phen)
-        with pytest.raises(epi.Epi4Error):
-            e.search3(4)
+        idx, key = e.search3(k)
+    np.testing.assert_array_equal(idx, want_idx)
+    np.testing.assert_array_equal(key, want_key)
