@@ -239,6 +239,7 @@ def run_ours(args):
                      "peak_source": peak_note},
         "breakdown_ms": {"pack": st["ms_pack"], "pop_T1T2T3": st["ms_pop"], "quad": st["ms_quad"],
                          "merge_d2h": st["ms_merge"]},
+        "step_ms": [round(t, 3) for t in times], "e2e_step_ms": [round(t, 3) for t in e2e_times],
         "useful_over_executed": (16.0 * st["quads"] * (d.n_controls + d.n_cases)) / max(st["executed_macs"], 1.0),
         "clocks": clk.summary(),
         "best": {"quad": epi.unpack_index(res[0][0]), "k2": float(res[1][0])},
