@@ -58,6 +58,8 @@ class ClockSampler:
         self.proc = None
 
     def __enter__(self):
+        if os.environ.get("EPI4_BENCH_NO_CLOCKS"):   # diagnostics only: no sampler (the line reports "unsampled")
+            return self
         q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
              "clocks_event_reasons.sw_power_cap")
@@ -240,6 +242,7 @@ def run_ours(args):
         "breakdown_ms": {"pack": st["ms_pack"], "pop_T1T2T3": st["ms_pop"], "quad": st["ms_quad"],
                          "merge_d2h": st["ms_merge"]},
         "step_ms": [round(t, 3) for t in times], "e2e_step_ms": [round(t, 3) for t in e2e_times],
+        "quad_step_ms": [round(t, 3) for t in quad_ms],
         "useful_over_executed": (16.0 * st["quads"] * (d.n_controls + d.n_cases)) / max(st["executed_macs"], 1.0),
         "clocks": clk.summary(),
         "best": {"quad": epi.unpack_index(res[0][0]), "k2": float(res[1][0])},
