@@ -16,6 +16,7 @@ total work is fixed -> "scaling": "strong" (the paper's Fig. 3 experiment, PAPER
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import math
 import os
@@ -165,6 +166,8 @@ def run_ours(args):
             return epi.search_distributed(local_search, top_k)
         return eng.search(top_k)
 
+    other_ms = []   # per timed step (device steps, then e2e steps): pack + T1/T2/T3 + merge time (library events)
+
     def timed(host, steps):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         times, quad_ms, launches, res = [], [], 0, None
@@ -180,15 +183,23 @@ def run_ours(args):
             times.append(ev0.elapsed_time(ev1))
             st = eng.stats()
             quad_ms.append(st["ms_quad"])
+            other_ms.append(round(st["ms_pack"] + st["ms_pop"] + st["ms_merge"], 3))
             launches += st["launches"] + st["launches_load"]
         return times, quad_ms, launches, res
 
     for _ in range(args.warmup):
         step(False)
     torch.cuda.synchronize()
-    with ClockSampler(local) as clk:
-        times, quad_ms, launches, res = timed(False, args.steps)
-    e2e_times, _, _, _ = timed(True, max(1, min(args.steps, 3)))
+    # Python's cyclic GC is paused over the timed steps (collected just before): a full collection in a process
+    # holding torch takes tens of ms and landed inside random steps (profiles/r01i_step_jitter.txt)
+    gc.collect()
+    gc.disable()
+    try:
+        with ClockSampler(local) as clk:
+            times, quad_ms, launches, res = timed(False, args.steps)
+        e2e_times, _, _, _ = timed(True, max(1, min(args.steps, 3)))
+    finally:
+        gc.enable()
     t_step = statistics.mean(times)
     t_e2e = statistics.mean(e2e_times)
     t_quad = statistics.mean(quad_ms)
@@ -242,7 +253,7 @@ def run_ours(args):
         "breakdown_ms": {"pack": st["ms_pack"], "pop_T1T2T3": st["ms_pop"], "quad": st["ms_quad"],
                          "merge_d2h": st["ms_merge"]},
         "step_ms": [round(t, 3) for t in times], "e2e_step_ms": [round(t, 3) for t in e2e_times],
-        "quad_step_ms": [round(t, 3) for t in quad_ms],
+        "quad_step_ms": [round(t, 3) for t in quad_ms], "load_merge_step_ms": other_ms,
         "useful_over_executed": (16.0 * st["quads"] * (d.n_controls + d.n_cases)) / max(st["executed_macs"], 1.0),
         "clocks": clk.summary(),
         "best": {"quad": epi.unpack_index(res[0][0]), "k2": float(res[1][0])},
