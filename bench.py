@@ -142,7 +142,7 @@ def run_ours(args):
     # N > 1: every rank builds the 3-way table on its tensor cores (~3 ms at C2, tiny next to the search);
     # --shard-t3 instead builds 1/world of it per rank (POPC kernel) and all-gathers the shares over NCCL
     shard = world > 1 and args.shard_t3
-    eng = epi.Epi4(local, pipe=args.pipe, rank=rank, world=world, shard_t3=shard)
+    eng = epi.Epi4(local, pipe=args.pipe, rank=rank, world=world, shard_t3=shard, objective=args.objective)
     eng.set_stream(stream.cuda_stream)
     geno_d = torch.from_numpy(d.geno).to(f"cuda:{local}")
     phen_d = torch.from_numpy(d.phen).to(f"cuda:{local}")
@@ -240,7 +240,7 @@ def run_ours(args):
         "data": "synthetic (seeded HWE genotypes + planted 4-way interaction, SURVEY.md §8(d))",
         "config": {"workload": f"{args.config}: N={n} SNPs, M={m} samples ({d.n_controls} controls / "
                                f"{d.n_cases} cases), exhaustive C(N,4)={comb4(n)} quads, top_k={top_k}",
-                   "pipe": args.pipe, "parallelism": f"static LPT over (w-block, x) units x {world}" + (", T3 sharded + NCCL all_gather" if shard else ""),
+                   "pipe": args.pipe, "objective": args.objective, "parallelism": f"static LPT over (w-block, x) units x {world}" + (", T3 sharded + NCCL all_gather" if shard else ""),
                    "l2": "flushed (512 MiB write) before every timed step"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": int(n * m + m),
                 "d2h_bytes_per_step": int(top_k * 16 + 4)},
@@ -256,7 +256,8 @@ def run_ours(args):
         "quad_step_ms": [round(t, 3) for t in quad_ms], "load_merge_step_ms": other_ms,
         "useful_over_executed": (16.0 * st["quads"] * (d.n_controls + d.n_cases)) / max(st["executed_macs"], 1.0),
         "clocks": clk.summary(),
-        "best": {"quad": epi.unpack_index(res[0][0]), "k2": float(res[1][0])},
+        "best": {"quad": epi.unpack_index(res[0][0]), "key": float(res[1][0])}
+        if args.objective != "k2" else {"quad": epi.unpack_index(res[0][0]), "k2": float(res[1][0])},
     }
     if args.pipe == "tc":
         # second denominator: the microbenchmarked MMA rate at the clock logged during the timed region —
@@ -318,6 +319,8 @@ def main():
     ap.add_argument("--config", default="C2", choices=list(datagen.CONFIGS))
     ap.add_argument("--pipe", default="tc", choices=["tc", "lop3"])
     ap.add_argument("--top-k", type=int, default=16)
+    ap.add_argument("--objective", default="k2", choices=["k2", "mi", "chi2"],
+                    help="ranking objective (K2 is the paper's and the headline; MI / chi-square: SURVEY §8(f) NEXT-4)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--shard-t3", action="store_true", help="N > 1: build 1/world of the 3-way table per rank and "
                     "all-gather the shares (NCCL) instead of building it on every rank")
