@@ -88,3 +88,21 @@ def test_search3_objectives_match_oracle(objective, cfg, nsnp, k):
         idx, key = e.search3(k)
     np.testing.assert_array_equal(idx, want_idx)
     np.testing.assert_array_equal(key, want_key)
+
+
+def test_chi2_rejects_counts_whose_numerator_is_not_exact():
+    """EPI4_OBJ_CHI2 needs n0 n1 M < 2^53 (exact uint64 -> double numerators, include/epi4.h): at n0 = 4e6,
+    n1 = 1000 (packable: 22 + 10 bits) the product is 1.6e16, so the load fails for chi-square, not for K2."""
+    import paper_conf_icpp_nobreiss22_b200 as epi
+    n0, n1 = 4_000_000, 1000
+    rng = np.random.default_rng(5)
+    geno = rng.integers(0, 3, size=(4, n0 + n1), dtype=np.uint8)
+    phen = np.zeros(n0 + n1, dtype=np.uint8)
+    phen[:n1] = 1
+    with epi.Epi4(0, pipe="tc", objective="chi2") as e:
+        with pytest.raises(epi.Epi4Error):
+            e.load_genotypes(geno, phen)
+    with epi.Epi4(0, pipe="tc", objective="k2") as e:
+        e.load_genotypes(geno, phen)
+        idx, _ = e.search(1)
+        assert len(idx) == 1
