@@ -49,9 +49,10 @@ typedef struct {
     int32_t pipe;     /* EPI4_PIPE_*                                                               */
     int32_t rank;     /* this process' rank and the world size: epi4_search evaluates only the     */
     int32_t world;    /*   work units the static LPT plan assigns to `rank`       */
-    int32_t grid;     /* persistent-kernel CTAs (0 = 2 x number of SMs)                             */
-    int32_t debug;    /* diagnostics only, 0 in production (debug modes disable warp roles; results  */
-                      /*   invalid except bit 16 = exact K2 for every quad, no filter)               */
+    int32_t grid;     /* persistent-kernel CTAs (0 = number of SMs, rounded down to whole CTA pairs)  */
+    int32_t debug;    /* 0 in production.  Bit 16 = exact score for every quad (no fp32 filter; exact */
+                      /*   results).  Other bits disable warp roles (results invalid) and are only    */
+                      /*   accepted by a diagnostics build (EPI4_DEBUG_MODES), else EPI4_EINVAL.      */
     int32_t flags;    /* EPI4_FLAG_* bits                                                          */
     int32_t objective; /* EPI4_OBJ_K2 (default), EPI4_OBJ_MI or EPI4_OBJ_CHI2 (§8(f) NEXT-4) */
 } epi4_opts;

@@ -63,6 +63,8 @@ class Epi4:
 
     def load_genotypes(self, geno, phen):
         """Byte genotypes N x M (SNP-major, {0,1,2}) + phenotypes M; host (numpy) or device (torch)."""
+        if getattr(geno, "ndim", None) != 2:
+            raise ValueError("geno must be a 2-D N x M array")
         n, m = geno.shape
         binding.epi4_pack_genotypes(self.ctx, geno, phen, n, m)
 

@@ -121,6 +121,35 @@ def _kind(x):
     return EPI4_PTR_HOST
 
 
+def _dtype_name(x) -> str:
+    """'uint8', 'uint32', ... for a numpy array or a torch tensor (None for raw pointers)."""
+    if isinstance(x, np.ndarray):
+        return x.dtype.name
+    dt = getattr(x, "dtype", None)
+    return None if dt is None else str(dt).replace("torch.", "")
+
+
+def _require(x, name: str, dtype: str, shape: tuple):
+    """Argument check for array inputs (raw int pointers are passed through unchecked): the C ABI reads
+    `dtype` elements, so e.g. an int64 genotype array would be misread byte-wise."""
+    if x is None or isinstance(x, int):
+        return
+    if _dtype_name(x) != dtype:
+        raise TypeError(f"{name}: expected {dtype}, got {_dtype_name(x)}")
+    if tuple(x.shape) != tuple(shape):
+        raise ValueError(f"{name}: expected shape {tuple(shape)}, got {tuple(x.shape)}")
+    contig = x.flags["C_CONTIGUOUS"] if isinstance(x, np.ndarray) else x.is_contiguous()
+    if not contig:
+        raise ValueError(f"{name}: must be C-contiguous")
+
+
+def _same_kind(*xs) -> int:
+    kinds = {_kind(x) for x in xs if x is not None and not isinstance(x, int)}
+    if len(kinds) > 1:
+        raise ValueError("all arrays of one call must be on the same side (all host or all device)")
+    return kinds.pop() if kinds else EPI4_PTR_HOST
+
+
 def epi4_default_opts() -> epi4_opts:
     o = epi4_opts()
     _lib.epi4_default_opts(ctypes.byref(o))
@@ -142,13 +171,17 @@ def epi4_set_stream(ctx, stream) -> None:
 
 
 def epi4_load_bits(ctx, planes_ctrl, planes_case, n_snps, n_controls, n_cases, ptr_kind=None) -> None:
-    kind = _kind(planes_ctrl) if ptr_kind is None else ptr_kind
+    _require(planes_ctrl, "planes_ctrl", "uint32", (2 * int(n_snps), (int(n_controls) + 31) // 32))
+    _require(planes_case, "planes_case", "uint32", (2 * int(n_snps), (int(n_cases) + 31) // 32))
+    kind = _same_kind(planes_ctrl, planes_case) if ptr_kind is None else ptr_kind
     _check(_lib.epi4_load_bits(ctx, _ptr(planes_ctrl), _ptr(planes_case), int(n_snps), int(n_controls),
                                int(n_cases), kind))
 
 
 def epi4_pack_genotypes(ctx, geno, phen, n_snps, n_samples, ptr_kind=None) -> None:
-    kind = _kind(geno) if ptr_kind is None else ptr_kind
+    _require(geno, "geno", "uint8", (int(n_snps), int(n_samples)))
+    _require(phen, "phen", "uint8", (int(n_samples),))
+    kind = _same_kind(geno, phen) if ptr_kind is None else ptr_kind
     _check(_lib.epi4_pack_genotypes(ctx, _ptr(geno), _ptr(phen), int(n_snps), int(n_samples), kind))
 
 

@@ -14,6 +14,8 @@ FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std
          "-Xcompiler", "-fPIC", "-Xcompiler", "-O2", "--expt-relaxed-constexpr"]
 if os.environ.get("EPI4_PROF"):   # instrumented build: per-role cycle counters + debug-64 pipeline trace
     FLAGS.append("-DEPI4_PROF=1")
+if os.environ.get("EPI4_PROF") or os.environ.get("EPI4_DEBUG_MODES"):
+    FLAGS.append("-DEPI4_DEBUG_MODES=1")   # opts.debug bits that disable warp roles (diagnostics only)
 
 
 def sources():

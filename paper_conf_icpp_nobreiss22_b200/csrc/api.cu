@@ -464,6 +464,11 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
         return fail(EPI4_EINVAL, "objective=%d: EPI4_OBJ_K2, EPI4_OBJ_MI or EPI4_OBJ_CHI2", o.objective);
     if (o.pipe != EPI4_PIPE_TC && o.pipe != EPI4_PIPE_LOP3) return fail(EPI4_EINVAL, "unknown pipe %d", o.pipe);
     if (o.world < 1 || o.rank < 0 || o.rank >= o.world) return fail(EPI4_EINVAL, "bad rank/world %d/%d", o.rank, o.world);
+#ifndef EPI4_DEBUG_MODES
+    // diagnostic modes that disable warp roles (results invalid) exist only in a diagnostics build
+    // (build.py with EPI4_DEBUG_MODES=1); bit 16 (exact score for every quad, results exact) is always allowed
+    if (o.debug & ~16) return fail(EPI4_EINVAL, "debug=%d: only bit 16 is available in a production build", o.debug);
+#endif
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(EPI4_ENODEV, "no CUDA device");
     if (cuda_device < 0 || cuda_device >= ndev) return fail(EPI4_ENODEV, "device %d out of range", cuda_device);
@@ -524,6 +529,8 @@ int epi4_set_stream(epi4_ctx* c, void* s) {
 int epi4_load_bits(epi4_ctx* c, const uint32_t* pc, const uint32_t* pk, int32_t n_snps, int64_t n0, int64_t n1,
                    int32_t ptr_kind) {
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    c->loaded = false;                    // a rejected load never leaves the previous dataset searchable
+    c->t3_pending = false;
     if (!pc || !pk) return fail(EPI4_EINVAL, "planes pointer is NULL");
     if (int r = check_dims(n_snps, n0, n1)) return r;
     CU(cudaSetDevice(c->device));
@@ -557,6 +564,8 @@ int epi4_load_bits(epi4_ctx* c, const uint32_t* pc, const uint32_t* pk, int32_t 
 int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, int32_t n_snps, int64_t m,
                         int32_t ptr_kind) {
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    c->loaded = false;                    // a rejected load never leaves the previous dataset searchable
+    c->t3_pending = false;
     if (!geno || !phen) return fail(EPI4_EINVAL, "genotype pointer is NULL");
     if (n_snps < 4 || n_snps > 65536) return fail(EPI4_EINVAL, "n_snps=%d outside [4, 65536]", n_snps);
     if (m < 2 || m > ((int64_t)1 << 31) - 4) return fail(EPI4_EINVAL, "n_samples=%lld", (long long)m);

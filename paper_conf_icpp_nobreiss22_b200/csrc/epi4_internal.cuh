@@ -78,7 +78,7 @@ struct DevData {
     const double* xlx;           // X(k) = k ln k, M + 2 entries (EPI4_OBJ_MI)
     double mi_const;             // X(M) - X(n0) - X(n1)
     int32_t objective;           // EPI4_OBJ_*
-    const uint8_t* expl[2];      // {0,1}-byte expanded planes [chunk][snp][g][128 samples] (tcgen05 operands)
+    const uint8_t* expl[2];      // E2M1 {0, 1.0} nibble planes (tcgen05 operands; layout: expl_off below)
     double flt_off;              // fp32 K2 filter: exact-score a quad iff ln2 A + flt_off <= threshold (epilogue.cuh)
     float chi_a, chi_b;          // fp32 chi-square filter: M / n0, M / n1 (epilogue.cuh, cell_chi_acc)
     double chi_M;                // M

@@ -162,9 +162,7 @@ cudaError_t launch_untile(const uint32_t* planes, int32_t n, int64_t np, int32_t
     return cudaGetLastError();
 }
 
-// ---- {0,1}-byte expansion of the planes (operands of the i8 tensor-core pipe) ---------------------
-// expl[kc][r = 2 snp + g][128 B]: byte s of row r = bit s of plane (kc, snp, g); 16-byte piece c stored
-// at piece c ^ (r & 7) (UMMA SW128 pattern, rows are 128 B so the 8-row groups are 1 KiB aligned).
+// ---- E2M1 expansion of the planes (operands of the tensor-core pipe) ------------------------------
 // Tensor-core operand planes: E2M1 nibbles (1.0 = 0x2 for a set bit, 0 otherwise), two samples per byte
 // (sample 2j in the low nibble of byte j), 256 samples = one 128-byte K-major row per fp4 chunk C (the 128-sample
 // plane chunks 2C and 2C+1; a missing odd chunk reads as zeros).  Layout [C][row r = 2 snp + g][128 B] with
