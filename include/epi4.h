@@ -158,6 +158,22 @@ int epi4_t3_ready(epi4_ctx* ctx);
  * counts_dev = NULL disables.  Only for small N (the buffer has C(N,4)*162 entries). */
 int epi4_set_dump(epi4_ctx* ctx, uint32_t* counts_dev);
 
+/* Verification sample (parity at full size, SURVEY.md §8(c) tier 2): during every later epi4_search /
+ * epi4_search_units, record each evaluated quad whose packed index q satisfies
+ *     (mix64(q ^ seed) & (2^log2_rate - 1)) == 0,
+ *     mix64(x): x ^= x >> 30; x *= 0xBF58476D1CE4E5B9; x ^= x >> 27; x *= 0x94D049BB133111EB; x ^= x >> 31
+ * (splitmix64's finalizer, uint64 arithmetic), with its exact key (as in k2_out) and its 2 x 81 table, all
+ * computed from the contraction counts of the search kernel itself (the production path, not epi4_tables).
+ * Up to `capacity` quads are stored per search (later hits are counted only); capacity = 0 disables.
+ * log2_rate = 0 samples every quad.  Device memory is owned by the context. */
+int epi4_set_sample(epi4_ctx* ctx, int32_t log2_rate, uint64_t seed, int64_t capacity);
+/* Copy the last search's sample to HOST arrays of `capacity` entries (quads, keys; counts: capacity x 162,
+ * controls row first as in epi4_tables).  *n_out = number of sampled quads in that search (entries beyond the
+ * context's or this call's capacity are not written).  EPI4_ESTATE if no sample is configured.  The order of
+ * the entries is unspecified. */
+int epi4_get_sample(epi4_ctx* ctx, uint64_t* quads_out, double* keys_out, uint32_t* counts_out, int64_t capacity,
+                    int64_t* n_out);
+
 /* ---- plan --------------------------------------------------------------------
  * Work unit u = (w-range, x): all quads whose first SNP lies in [128*wr, 128*wr+128) and
  * whose second SNP is x.  The plan lists this rank's units (static LPT by modelled cost, identical

@@ -96,6 +96,15 @@ class Epi4:
         torch.cuda.current_stream().synchronize()
         binding.epi4_t3_ready(self.ctx)
 
+    def set_sample(self, log2_rate: int, seed: int = 0, capacity: int = 1 << 16):
+        """Verification sample of the next searches (epi4_set_sample); capacity 0 disables."""
+        binding.epi4_set_sample(self.ctx, log2_rate, seed, capacity)
+        self._samp_cap = int(capacity)
+
+    def get_sample(self):
+        """(packed quads, keys, counts [n, 2, 81], total hits) recorded by the last search."""
+        return binding.epi4_get_sample(self.ctx, getattr(self, "_samp_cap", 0))
+
     def tables(self, quads):
         return binding.epi4_tables(self.ctx, quads)
 

@@ -69,6 +69,8 @@ def _load():
         "epi4_search3": (ctypes.c_int, [P, I32, P, P, P]),
         "epi4_tables": (ctypes.c_int, [P, P, I64, P]),
         "epi4_set_dump": (ctypes.c_int, [P, P]),
+        "epi4_set_sample": (ctypes.c_int, [P, I32, ctypes.c_uint64, I64]),
+        "epi4_get_sample": (ctypes.c_int, [P, P, P, P, I64, ctypes.POINTER(I64)]),
         "epi4_t3_shard": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(I64), ctypes.POINTER(I64)]),
         "epi4_t3_ready": (ctypes.c_int, [P]),
         "epi4_plan_count": (I64, [I32, I32, I32]),
@@ -233,6 +235,21 @@ def epi4_t3_ready(ctx) -> None:
 
 def epi4_set_dump(ctx, counts_dev) -> None:
     _check(_lib.epi4_set_dump(ctx, _ptr(counts_dev)))
+
+
+def epi4_set_sample(ctx, log2_rate: int, seed: int, capacity: int) -> None:
+    _check(_lib.epi4_set_sample(ctx, int(log2_rate), ctypes.c_uint64(int(seed) & (2**64 - 1)), int(capacity)))
+
+
+def epi4_get_sample(ctx, capacity: int):
+    """(packed quads uint64[n], keys float64[n], counts uint32[n, 2, 81], total hits) of the last search."""
+    q = np.zeros(max(capacity, 1), dtype=np.uint64)
+    k = np.zeros(max(capacity, 1), dtype=np.float64)
+    c = np.zeros((max(capacity, 1), 2, 81), dtype=np.uint32)
+    n = ctypes.c_int64()
+    _check(_lib.epi4_get_sample(ctx, _ptr(q), _ptr(k), _ptr(c), int(capacity), ctypes.byref(n)))
+    m = min(int(n.value), int(capacity))
+    return q[:m], k[:m], c[:m], int(n.value)
 
 
 def epi4_plan_count(n_snps: int, rank: int = 0, world: int = 1) -> int:

@@ -103,6 +103,13 @@ struct epi4_ctx {
     int32_t* d_out_n = nullptr;
     unsigned int* d_status = nullptr;
     uint32_t* dump = nullptr;
+    // verification sample (epi4_set_sample)
+    int64_t samp_cap = 0;
+    uint64_t samp_seed = 0, samp_mask = 0;
+    unsigned long long* d_samp_n = nullptr;
+    uint64_t* d_samp_idx = nullptr;
+    double* d_samp_key = nullptr;
+    uint32_t* d_samp_counts = nullptr;
     cudaEvent_t ev[6] = {};
     epi4_stats stats{};
 };
@@ -514,6 +521,10 @@ void epi4_destroy(epi4_ctx* c) {
     dfree(c->d_out_idx);
     dfree(c->d_out_n);
     dfree(c->d_status);
+    dfree(c->d_samp_n);
+    dfree(c->d_samp_idx);
+    dfree(c->d_samp_key);
+    dfree(c->d_samp_counts);
     for (int i = 0; i < 6; ++i)
         if (c->ev[i]) cudaEventDestroy(c->ev[i]);
     if (c->own_stream) cudaStreamDestroy(c->own_stream);
@@ -640,6 +651,48 @@ int epi4_set_dump(epi4_ctx* c, uint32_t* counts_dev) {
     return 0;
 }
 
+int epi4_set_sample(epi4_ctx* c, int32_t log2_rate, uint64_t seed, int64_t capacity) {
+    if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
+    if (log2_rate < 0 || log2_rate > 63 || capacity < 0) return fail(EPI4_EINVAL, "bad sample arguments");
+    CU(cudaSetDevice(c->device));
+    dfree(c->d_samp_idx);
+    dfree(c->d_samp_key);
+    dfree(c->d_samp_counts);
+    c->samp_cap = 0;
+    if (capacity == 0) return 0;
+    if (!c->d_samp_n) CU(cudaMalloc(&c->d_samp_n, sizeof(unsigned long long)));
+    CU(cudaMalloc(&c->d_samp_idx, (size_t)capacity * sizeof(uint64_t)));
+    CU(cudaMalloc(&c->d_samp_key, (size_t)capacity * sizeof(double)));
+    CU(cudaMalloc(&c->d_samp_counts, (size_t)capacity * 162 * sizeof(uint32_t)));
+    CU(cudaMemset(c->d_samp_n, 0, sizeof(unsigned long long)));
+    c->samp_cap = capacity;
+    c->samp_seed = seed;
+    c->samp_mask = log2_rate == 0 ? 0 : (~0ull >> (64 - log2_rate));
+    return 0;
+}
+
+int epi4_get_sample(epi4_ctx* c, uint64_t* quads_out, double* keys_out, uint32_t* counts_out, int64_t capacity,
+                    int64_t* n_out) {
+    if (!c || !n_out) return fail(EPI4_EINVAL, "NULL argument");
+    if (!c->samp_cap) return fail(EPI4_ESTATE, "no verification sample configured (epi4_set_sample)");
+    if (capacity < 0 || (capacity > 0 && (!quads_out || !keys_out || !counts_out)))
+        return fail(EPI4_EINVAL, "bad output arguments");
+    CU(cudaSetDevice(c->device));
+    unsigned long long n = 0;
+    CU(cudaMemcpyAsync(&n, c->d_samp_n, sizeof n, cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaStreamSynchronize(c->stream));
+    const int64_t k = std::min<int64_t>(std::min<int64_t>((int64_t)n, capacity), c->samp_cap);
+    if (k > 0) {
+        CU(cudaMemcpyAsync(quads_out, c->d_samp_idx, (size_t)k * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
+        CU(cudaMemcpyAsync(keys_out, c->d_samp_key, (size_t)k * sizeof(double), cudaMemcpyDeviceToHost, c->stream));
+        CU(cudaMemcpyAsync(counts_out, c->d_samp_counts, (size_t)k * 162 * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                           c->stream));
+        CU(cudaStreamSynchronize(c->stream));
+    }
+    *n_out = (int64_t)n;
+    return 0;
+}
+
 int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world) {
     if (n_snps < 4 || n_snps > 65536 || world < 1 || rank < 0 || rank >= world) {
         fail(EPI4_EINVAL, "bad plan arguments");
@@ -728,6 +781,14 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     sp.list_idx = c->d_list_idx;
     sp.list_cnt = c->d_list_cnt;
     sp.dump = c->dump;
+    sp.samp_cap = c->samp_cap;
+    sp.samp_seed = c->samp_seed;
+    sp.samp_mask = c->samp_mask;
+    sp.samp_n = c->d_samp_n;
+    sp.samp_idx = c->d_samp_idx;
+    sp.samp_key = c->d_samp_key;
+    sp.samp_counts = c->d_samp_counts;
+    if (c->samp_cap) CU(cudaMemsetAsync(c->d_samp_n, 0, sizeof(unsigned long long), c->stream));
     sp.status = c->d_status;
     sp.quads_done = c->d_counters + 1;
     sp.prof = c->d_counters + 16;

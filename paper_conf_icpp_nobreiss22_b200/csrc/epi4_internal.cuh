@@ -162,7 +162,25 @@ struct SearchParams {
 
     int32_t debug;             // diagnostics only (results invalid): 1 skip producers, 2 skip scoring, 4 skip MMA,
                                // 128 no A copies (16: exact K2 for every quad, 64: trace)
+    // verification sample (epi4_set_sample): quads with (mix64(index ^ samp_seed) & samp_mask) == 0 are recorded
+    // with their exact key and 162 counts (the search kernel's own contraction + recovery); samp_cap = 0: off
+    int64_t samp_cap;
+    uint64_t samp_seed, samp_mask;
+    unsigned long long* samp_n;
+    uint64_t* samp_idx;
+    double* samp_key;
+    uint32_t* samp_counts;
 };
+
+// splitmix64 finalizer: the verification-sample hash (epi4.h epi4_set_sample)
+__host__ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
+    x ^= x >> 30;
+    x *= 0xBF58476D1CE4E5B9ull;
+    x ^= x >> 27;
+    x *= 0x94D049BB133111EBull;
+    x ^= x >> 31;
+    return x;
+}
 
 }  // namespace epi4
 

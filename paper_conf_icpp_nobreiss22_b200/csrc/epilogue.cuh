@@ -316,6 +316,33 @@ static __device__ __forceinline__ double score_quad_rare(const DevData& d, int w
     for (int k = 0; k < 16; ++k) t[k] = c16[k];
     return score_quad(d, w, x, y, z, t, dump_row);
 }
+// Verification sample (epi4_set_sample): is quad `idx` sampled?  Then record it: packed index, exact key of the
+// context's objective and its 2 x 81 counts, from the counts the search kernel itself produced.  Returns the
+// exact key through `key` (the quad is then offered to the top-k with it).  Slots beyond samp_cap are counted only.
+__device__ __forceinline__ bool sample_hit(const SearchParams& sp, uint64_t idx) {
+    return sp.samp_cap && (mix64(idx ^ sp.samp_seed) & sp.samp_mask) == 0;
+}
+static __device__ __noinline__ double sample_record(const SearchParams& sp, int w, int x, int y, int z,
+                                                    const uint32_t (&c16)[16]) {
+    const unsigned long long slot = atomicAdd(sp.samp_n, 1ull);
+    uint32_t scratch[162];
+    uint32_t* row = slot < (unsigned long long)sp.samp_cap ? sp.samp_counts + slot * 162 : scratch;
+    double key = score_quad(sp.d, w, x, y, z, c16, row);            // K2 + counts
+    if (sp.d.objective != EPI4_OBJ_K2) key = score_quad(sp.d, w, x, y, z, c16, nullptr);
+    if (slot < (unsigned long long)sp.samp_cap) {
+        sp.samp_idx[slot] = pack_quad(w, x, y, z);
+        sp.samp_key[slot] = key;
+    }
+    return key;
+}
+static __device__ __forceinline__ double sample_record_rare(const SearchParams& sp, int w, int x, int y, int z,
+                                                            const uint32_t (&c16)[16]) {
+    uint32_t t[16];
+#pragma unroll
+    for (int k = 0; k < 16; ++k) t[k] = c16[k];
+    return sample_record(sp, w, x, y, z, t);
+}
+
 // Third-order search: exact K2 of triple w < x < y from its 8 packed non-aa counts
 // c8[4a + 2b + c] (the 3-way-table mode's d = AA columns), the same recovery one order lower: generalized
 // cells S[9a + 3b + c] (digit 2 = '*') from c8, T2, T1 and n, aa recovered on the three axes,

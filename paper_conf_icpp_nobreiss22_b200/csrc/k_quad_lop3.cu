@@ -112,7 +112,12 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
                 uint32_t* dump = sp.dump ? sp.dump + rank4(w, x, y, z) * 162 : nullptr;
                 uint32_t c16[16];
                 pack16(d, c0, c1, c16);
-                key = score_quad(d, w, x, y, z, c16, dump);
+                if (!dump && sample_hit(sp, pack_quad(w, x, y, z))) {
+                    key = sample_record(sp, w, x, y, z, c16);
+                } else {
+                    key = score_quad(d, w, x, y, z, c16, dump);
+                    if (dump && d.objective != EPI4_OBJ_K2) key = score_quad(d, w, x, y, z, c16, nullptr);
+                }
                 idx = pack_quad(w, x, y, z);
                 ++my_quads;
             }

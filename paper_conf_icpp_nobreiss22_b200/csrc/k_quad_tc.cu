@@ -791,6 +791,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     offer = true;
                     if (dump) {
                         key = score_quad_rare(d, w, ti.x, y, ti.z, c16, dump);
+                        if (d.objective != EPI4_OBJ_K2) key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
+                    } else if (sample_hit(sp, pack_quad(w, ti.x, y, ti.z))) {
+                        key = sample_record_rare(sp, w, ti.x, y, ti.z, c16);
                     } else if (sp.use_filter) {
                         // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
                         // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2); FILT 2: MI

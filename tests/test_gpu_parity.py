@@ -23,7 +23,7 @@ def _epi():
     return epi
 
 
-def _engine(pipe="lop3", **kw):
+def _engine(pipe="tc", **kw):
     return _epi().Epi4(0, pipe=pipe, **kw)
 
 
@@ -200,7 +200,7 @@ def test_hand_example_on_gpu():
 
 # ---- configs C2..C5: sub-windows at full M and sampled quads at full N ---------------------------------
 
-WINDOWS = {"C2": 64, "C3": 48, "C4": 40, "C5": 56}
+WINDOWS = {"C2": 64, "C3": 64, "C4": 64, "C5": 64}
 
 
 @functools.lru_cache(maxsize=None)
