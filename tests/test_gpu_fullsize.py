@@ -106,7 +106,7 @@ def test_C4_windowed_slice_sampled_and_planted():
     lo, hi = max(0, u0 - 12), min(len(units), u0 + 12)
     sel = units[lo:hi]
     assert len(set(sel[:, 0].tolist())) >= 3 and (sel[:, 1] // wr_size == sel[:, 0]).any()
-    nq = int(sum(min(wr_size, x - wr * wr_size) * (n - x - 1) * (n - x - 2) // 2 for wr, x in sel))
+    nq = sum(min(wr_size, int(x) - int(wr) * wr_size) * (n - int(x) - 1) * (n - int(x) - 2) // 2 for wr, x in sel)
     r = rate_for(nq, 15000)
     with epi.Epi4(0, pipe="tc") as e:
         e.load_genotypes(d.geno, d.phen)
