@@ -14,7 +14,7 @@ import re
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libepi4.so")
+LIB_PATH = os.environ.get("EPI4_LIB") or os.path.join(HERE, "libepi4.so")   # EPI4_LIB: diagnostics builds only
 HEADER = os.path.join(os.path.dirname(HERE), "include", "epi4.h")
 
 EPI4_OK, EPI4_EINVAL, EPI4_ENOMEM, EPI4_ECUDA, EPI4_ESTATE, EPI4_ENODEV = 0, -1, -2, -3, -4, -5

@@ -8,7 +8,7 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libepi4.so")
+LIB = os.environ.get("EPI4_LIB_OUT") or os.path.join(HERE, "libepi4.so")   # EPI4_LIB_OUT: diagnostics builds
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-O2", "--expt-relaxed-constexpr"]
@@ -16,6 +16,7 @@ if os.environ.get("EPI4_PROF"):   # instrumented build: per-role cycle counters 
     FLAGS.append("-DEPI4_PROF=1")
 if os.environ.get("EPI4_PROF") or os.environ.get("EPI4_DEBUG_MODES"):
     FLAGS.append("-DEPI4_DEBUG_MODES=1")   # opts.debug bits that disable warp roles (diagnostics only)
+FLAGS += os.environ.get("EPI4_NVCC_EXTRA", "").split()   # diagnostics variants (e.g. -DEPI4_PROD_WARPS=8)
 
 
 def sources():
@@ -37,7 +38,7 @@ def needs_build() -> bool:
 def build(force: bool = False, verbose: bool = False, extra=()) -> str:
     if not force and not needs_build():
         return LIB
-    objdir = os.path.join(HERE, "build")
+    objdir = os.path.join(HERE, "build" + ("_" + os.path.basename(LIB) if os.environ.get("EPI4_LIB_OUT") else ""))
     os.makedirs(objdir, exist_ok=True)
     objs = []
     procs = []

@@ -65,7 +65,12 @@ constexpr int B_BYTES = CHUNKS * B_SUB;  // one TMA copy per stage (16 KiB)
 #ifndef EPI4_PROD_WARPS
 #define EPI4_PROD_WARPS 4
 #endif
-constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
+#ifndef EPI4_EPI_WARPS
+#define EPI4_EPI_WARPS 8
+#endif
+constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = EPI4_EPI_WARPS;
+static_assert(EPI_WARPS % 4 == 0 && PROD_WARPS % 4 == 0, "warpgroup-aligned roles (setmaxnreg, TMEM lane quadrants)");
+constexpr int EPI_NH = EPI_WARPS / 4;                     // epilogue warps per TMEM lane quadrant
 static_assert(PROD_WARPS % CHUNKS == 0, "producer warps come in groups of CHUNKS (one chunk of a step each)");
 constexpr int PROD_STRIDE = PROD_WARPS / CHUNKS;          // steps between two steps of one producer warp
 constexpr int MMA_ISSUERS = 2;           // leader CTA: two issuers alternate steps (one thread cannot hide
@@ -79,11 +84,13 @@ constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 512
 #define EPI4_REGS_CTL 32
 #endif
 #ifndef EPI4_REGS_PROD
-#define EPI4_REGS_PROD 128
+#define EPI4_REGS_PROD (PROD_WARPS == 4 ? 128 : 64)
 #endif
-constexpr bool REGSPLIT = PROD_WARPS == 4 && MMA_WARPS + TMA_WARPS == 4 && EPI_WARPS == 8;
+constexpr int NWARPS = EPI_WARP0 + EPI_WARPS;
+constexpr bool REGSPLIT = MMA_WARPS + TMA_WARPS == 4;
 constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
-constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176
+constexpr int REGS_EPI_RAW = (65536 / 32 - 4 * REGS_CTL - PROD_WARPS * REGS_PROD) / EPI_WARPS / 8 * 8;
+constexpr int REGS_EPI = REGS_EPI_RAW > 232 ? 232 : REGS_EPI_RAW;   // 176 with 4 producer / 8 epilogue warps
 constexpr int TMEM_COLS = 512;
 constexpr int REGIONS = 3;               // accumulator regions of N columns, rotated per tile (header comment)
 constexpr int ACC_COLS = REGIONS * N;
@@ -379,7 +386,7 @@ __device__ __forceinline__ void transpose8(uint32_t (&v)[16], int lane) {
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
 template <int SA, int SB, bool PK16, int FILT>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
-    static_assert(SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2,
+    static_assert(SA % 2 == 0 && SA % tc::PROD_STRIDE == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::TMA_WARPS == 2,
                   "ring sizes must be multiples of the alternating warps' stride (phase aliasing)");
     extern __shared__ unsigned char smem_raw[];
     // A ring (produced): afull (@leader: both CTAs' producers), aempty (MMA commit);
@@ -399,7 +406,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     // arbiter"), so the latency-critical roles (MMA / TMA issuers, producers) get the high physical warp ids
     // 8..15 and the throughput-bound epilogue the low ones; rw & 3 == warp & 3 (TMEM lane quadrant) and the
     // warpgroups stay aligned for setmaxnreg.
-    const int rw = (warp + 8) & 15;
+    const int rw = (warp + tc::NWARPS - tc::EPI_WARPS) % tc::NWARPS;
     const DevData& d = sp.d;
     const uint32_t rank = cluster_rank();
     const bool leader = rank == 0;
@@ -432,7 +439,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     if (rw >= tc::EPI_WARP0) {
         const int ew = rw - tc::EPI_WARP0, q = warp & 3, h = ew >> 2;
         const uint32_t tq = s_tmem + ((uint32_t)(q * 32) << 16);
-        for (int col = 16 * h; col < tc::ACC_COLS; col += 32) tmem_zero16(tq + (uint32_t)col);
+        for (int col = 16 * h; col < tc::ACC_COLS; col += 16 * tc::EPI_NH) tmem_zero16(tq + (uint32_t)col);
         if (h == 0)                      // E8M0 scale factors 2^0 for every MMA (any layout reads 0x7F)
             for (int col = tc::SF_COL; col < tc::TMEM_COLS; col += 16) tmem_fill16(tq + (uint32_t)col, 0x7F7F7F7Fu);
         tmem_wait_st();
@@ -453,7 +460,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 
     if (tc::REGSPLIT) {
         if (rw < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_CTL));
-        else if (rw < 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_PROD));
+        else if (rw < tc::EPI_WARP0) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_PROD));
         else asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(tc::REGS_EPI));
     }
     if (rw < tc::MMA_WARPS) {
@@ -610,18 +617,26 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 for (int k = 0; k < YK; ++k) ny[k] = ld_piece(E, C, ry + 4 * k);
             }
         };
-        load(pre);
-        pre.advance(sp, tc::PROD_STRIDE);
+        // register prefetch one own step ahead (4 producer warps), or (8 producer warps, half the registers) the
+        // step's own loads issued before the slot wait, latency hidden by the other warps' steps
+        constexpr bool PREFETCH = tc::PROD_WARPS == 4;
+        if (PREFETCH) {
+            load(pre);
+            pre.advance(sp, tc::PROD_STRIDE);
+        }
         for (int step = pstep0; st.valid(sp); step += tc::PROD_STRIDE) {
             const int sa = step % SA;
             if (lane == 0) TRACE(2, step);
             uint4 cx[4], cy[YK];
+            if (!PREFETCH) load(st);
 #pragma unroll
             for (int k = 0; k < 4; ++k) cx[k] = nx[k];
 #pragma unroll
             for (int k = 0; k < YK; ++k) cy[k] = ny[k];
-            load(pre);                                            // next own step's singles (in flight)
-            pre.advance(sp, tc::PROD_STRIDE);
+            if (PREFETCH) {
+                load(pre);                                        // next own step's singles (in flight)
+                pre.advance(sp, tc::PROD_STRIDE);
+            }
             const long long t0 = PCLK();
             mbar_wait(&aempty_bar[sa], (uint32_t)((step / SA) & 1) ^ 1u);   // A slot free (MMA of step - SA done)
             const long long t1 = PCLK();
@@ -660,7 +675,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         // with all 16 counts c16[8a + bcd'].
         const int ew = rw - tc::EPI_WARP0;             // 0..7
         const int q = warp & 3;                         // TMEM lane quadrant this warp may access
-        const int h = ew >> 2;                          // two warps per quadrant split the column groups
+        const int h = ew >> 2;                          // EPI_NH warps per quadrant split the column groups
         const int yl = 4 * q + (lane >> 3), L = lane & 7;
         unsigned long long my_quads = 0, n_exact = 0;
         long long t_wait = 0, t_busy = 0;
@@ -683,7 +698,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             // pass 1: pack each (control, case) count pair into one 32-bit word, in place in the case region,
             // and zero the control region, which the next tile's case accumulation reuses
 #pragma unroll 1
-            for (int g = h; g < tc::NG; g += 2) {
+            for (int g = h; g < tc::NG; g += tc::EPI_NH) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(R0 + 16 * g, v0);
                 tmem_ld16(R1 + 16 * g, v1);
@@ -706,12 +721,12 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             const bool yok = y < ti.z && !ti.skip;
             // pass 2: score the quads from the packed counts
 #pragma unroll 1
-            for (int g = h; g < tc::NG; g += 2) {
+            for (int g = h; g < tc::NG; g += tc::EPI_NH) {
                 uint32_t c16[16];
                 tmem_ld16(R1 + 16 * g, c16);
                 tmem_wait_ld();
                 tmem_zero16(R1 + 16 * g);                 // ready for a later tile's accumulation
-                if (g + 2 >= tc::NG) {
+                if (g + tc::EPI_NH >= tc::NG) {
                     tmem_wait_st();
                     tc_fence_before();
                     __syncwarp();
@@ -885,9 +900,11 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
                   : (pk16 ? launch_cfg<A_, B_, true, 0>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0>(sp, smem, grid, s))
     if (pick.sa == 4 && pick.sb == 6) EPI4_LAUNCH(4, 6);
     else if (pick.sa == 4 && pick.sb == 4) EPI4_LAUNCH(4, 4);
-    else if (pick.sa == 2 && pick.sb == 6) EPI4_LAUNCH(2, 6);
-    else if (pick.sa == 2 && pick.sb == 4) EPI4_LAUNCH(2, 4);
-    else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
+    else if constexpr (tc::PROD_STRIDE <= 2) {
+        if (pick.sa == 2 && pick.sb == 6) EPI4_LAUNCH(2, 6);
+        else if (pick.sa == 2 && pick.sb == 4) EPI4_LAUNCH(2, 4);
+        else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
+    }
 #undef EPI4_LAUNCH
     if (launches) ++*launches;
     return e;

@@ -17,8 +17,9 @@ ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--debug", type=int, default=0)
 ap.add_argument("--grid", type=int, default=0)
 ap.add_argument("--objective", default="k2", choices=["k2", "mi", "chi2"])
+ap.add_argument("--n-snps", type=int, default=None, help="first N SNPs of the config's dataset (all M samples)")
 a = ap.parse_args()
-d = datagen.make_config(a.config)
+d = datagen.make_config(a.config, n_snps=a.n_snps)
 with epi.Epi4(0, pipe=a.pipe, debug=a.debug, grid=a.grid, objective=a.objective) as e:
     e.load_genotypes(d.geno, d.phen)
     for _ in range(a.repeat):
