@@ -59,21 +59,6 @@ cudaError_t grow(T*& p, size_t& cap, size_t bytes) {
 }
 }  // namespace
 
-// The work plan of a search, cached across searches of the same shape (a bench step re-plans nothing and copies
-// no plan data to the device): this rank's units [ub, ue) of the static LPT plan, grouped by (T3 slab R, X) when
-// the 3-way table is windowed, with their group-relative inclusive prefix of tiles / pair tiles.
-struct SearchPlan {
-    struct Group { int64_t b, e; int32_t wr, xr; };
-    bool valid = false;
-    int32_t n = 0, rank = 0, world = 0, pipe = -1;
-    int64_t ub = 0, ue = 0;
-    bool windowed = false;
-    std::vector<Unit> units;
-    std::vector<int64_t> prefix_host;   // group-relative inclusive prefix
-    std::vector<Group> groups;
-    bool table_cached = false;          // d_tiles holds the whole (single-group, single-chunk) tile table
-};
-
 struct epi4_ctx {
     int device = 0;
     epi4_opts opts{};
@@ -103,15 +88,10 @@ struct epi4_ctx {
     size_t cap_scratch = 0;
     // search workspace
     Unit* d_units = nullptr;
+    int64_t* d_prefix = nullptr;
     size_t units_cap = 0;
-    uint64_t* d_tiles = nullptr;   // tensor-core pipe: pair-tile table of the search (k_tile_table), 16 B per pair
+    uint64_t* d_tiles = nullptr;   // tensor-core pipe: decoded tile table (k_tile_table), 8 B per tile
     size_t cap_tiles = 0;
-    uint64_t* d_tiles3 = nullptr;  // host-built pair tiles of the 3-way-table mode / third-order search
-    size_t cap_tiles3 = 0;
-    int64_t* d_gprefix = nullptr;  // group-relative inclusive tile / pair-tile prefix per unit
-    int64_t tile_chunk = (int64_t)1 << 24;   // pair tiles per search launch (bounds the tile table: 256 MiB)
-    SearchPlan plan;               // cached work plan of the last search (epi4_search_units)
-    unsigned char* h_out = nullptr;   // pinned: out count, status, counters
     unsigned long long* d_counters = nullptr;   // [0] tile counter, [1] quads done
     double* d_list_k2 = nullptr;
     uint64_t* d_list_idx = nullptr;
@@ -166,7 +146,7 @@ DevData devdata(const epi4_ctx* c) {
     d.nchunks4[1] = (c->nchunks[1] + 1) / 2;
     d.nsteps[0] = (d.nchunks4[0] + 1) / 2;
     d.nsteps[1] = (d.nchunks4[1] + 1) / 2;
-    d.nrb = c->npad / 32;
+    d.nrb = c->npad / 64;
     // c0 <= n0 < 2^pk_shift; 16 whenever both counts fit 16 bits (the epilogue then unpacks each half into a
     // float with one byte permute, epilogue.cuh cell_T_acc<true>)
     d.pk_shift = 1;
@@ -231,9 +211,9 @@ struct PlanEntry {
 
 std::vector<PlanEntry> all_units(int32_t n) {
     std::vector<PlanEntry> v;
-    const int32_t nr = (n + EPI4_WU - 1) / EPI4_WU;
+    const int32_t nr = (n + EPI4_WP - 1) / EPI4_WP;
     for (int32_t wr = 0; wr < nr; ++wr)
-        for (int32_t x = wr * EPI4_WU + 1; x <= n - 3; ++x) {
+        for (int32_t x = wr * EPI4_WP + 1; x <= n - 3; ++x) {
             const double cost = (double)unit_tiles(n, x);
             if (cost > 0) v.push_back({{wr, x}, cost});
         }
@@ -278,79 +258,6 @@ int ensure_lists(epi4_ctx* c, int32_t slots, int32_t cap) {
     return 0;
 }
 
-// The search's work plan (cached, SearchPlan): units of this rank's plan slice [ub, ue), grouped for the
-// windowed 3-way table, the group-relative prefix, uploaded once; the tile table is rebuilt only when needed.
-int prepare_units(epi4_ctx* c, int64_t ub, int64_t ue) {
-    SearchPlan& pl = c->plan;
-    const bool tcp = c->opts.pipe != EPI4_PIPE_LOP3;
-    if (pl.valid && pl.n == c->n && pl.rank == c->opts.rank && pl.world == c->opts.world && pl.pipe == c->opts.pipe &&
-        pl.windowed == c->t3_windowed && pl.ub == ub && pl.ue == ue)
-        return 0;
-    pl.valid = false;
-    pl.table_cached = false;
-    std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
-    const int64_t nall = (int64_t)plan.size();
-    int64_t b = ub < 0 ? 0 : ub, e = (ue < 0 || ue > nall) ? nall : ue;
-    if (b > e) b = e;
-    const int64_t nu = e - b;
-    pl.units.assign((size_t)nu, Unit{0, 0});
-    for (int64_t i = 0; i < nu; ++i) pl.units[(size_t)i] = plan[(size_t)(b + i)].u;
-    // Windowed T3: the units are taken grouped by (slab R = 128-SNP range of w, 128-SNP x-range X) so that each
-    // launch reads only the slabs FIRST(R) and FIRST(X) (rebuilt on the tensor cores when R or X changes); the
-    // result does not depend on the order (top-k by (K2, index)).  Resident T3: one group, the plan order.
-    pl.groups.clear();
-    if (c->t3_windowed && nu > 0) {
-        std::stable_sort(pl.units.begin(), pl.units.end(), [](const Unit& p, const Unit& q) {
-            const int32_t rp = p.wr * EPI4_WU / EPI4_WP, rq = q.wr * EPI4_WU / EPI4_WP;
-            if (rp != rq) return rp < rq;
-            if (p.x / EPI4_WP != q.x / EPI4_WP) return p.x / EPI4_WP < q.x / EPI4_WP;
-            return p.wr != q.wr ? p.wr < q.wr : p.x < q.x;
-        });
-        for (int64_t i = 0; i < nu; ++i) {
-            const int32_t r = pl.units[(size_t)i].wr * EPI4_WU / EPI4_WP, xr = pl.units[(size_t)i].x / EPI4_WP;
-            if (pl.groups.empty() || pl.groups.back().wr != r || pl.groups.back().xr != xr)
-                pl.groups.push_back(SearchPlan::Group{i, i, r, xr});
-            pl.groups.back().e = i + 1;
-        }
-    } else if (nu > 0) {
-        pl.groups.push_back(SearchPlan::Group{0, nu, -1, -1});
-    }
-    pl.prefix_host.assign((size_t)nu, 0);
-    int64_t maxg = 0;
-    for (const SearchPlan::Group& g : pl.groups) {
-        int64_t acc = 0;
-        for (int64_t i = g.b; i < g.e; ++i) {
-            const int32_t x = pl.units[(size_t)i].x;
-            acc += tcp ? unit_pairs(c->n, x) : unit_tiles(c->n, x);
-            pl.prefix_host[(size_t)i] = acc;
-        }
-        maxg = std::max(maxg, acc);
-    }
-    if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
-        dfree(c->d_units);
-        dfree(c->d_gprefix);
-        c->units_cap = (size_t)std::max<int64_t>(nu, 1);
-        CU(cudaMalloc(&c->d_units, c->units_cap * sizeof(Unit)));
-        CU(cudaMalloc(&c->d_gprefix, c->units_cap * sizeof(int64_t)));
-    }
-    if (nu > 0) {
-        CU(cudaMemcpyAsync(c->d_units, pl.units.data(), (size_t)nu * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
-        CU(cudaMemcpyAsync(c->d_gprefix, pl.prefix_host.data(), (size_t)nu * sizeof(int64_t), cudaMemcpyHostToDevice,
-                           c->stream));
-        CU(cudaStreamSynchronize(c->stream));   // pageable sources
-    }
-    if (tcp) CU(grow(c->d_tiles, c->cap_tiles, (size_t)std::max<int64_t>(1, std::min(maxg, c->tile_chunk)) * 16));
-    pl.n = c->n;
-    pl.rank = c->opts.rank;
-    pl.world = c->opts.world;
-    pl.pipe = c->opts.pipe;
-    pl.windowed = c->t3_windowed;
-    pl.ub = ub;
-    pl.ue = ue;
-    pl.valid = true;
-    return 0;
-}
-
 // bytes of one windowed-T3 slab: 128 first SNPs x C(n, 2) pairs x 8 packed cells
 size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * sizeof(uint32_t); }
 
@@ -358,40 +265,26 @@ size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * s
 // tensorOp_3way): tiles (w-range wp, x, y-range y0, z = n) cover every w < x < y < n exactly
 // once.  slab_w0 < 0: all w-ranges, resident colex layout; else only the w-range starting at slab_w0, written
 // as the slab FIRST([slab_w0, slab_w0 + 128)) (DevData t3_win).
-// the pair tiles of unit (wr, x) against z = n (the all-ones SNP): y-ranges y0 = x + 1 + 16 k <= n - 1, two per
-// pair, an odd last one paired with a skipped copy (tile_entry)
-void append_pairs_z1(std::vector<uint64_t>& out, int32_t n, int32_t wr, int32_t x) {
-    int32_t pend = -1;
-    for (int32_t y0 = x + 1; y0 <= n - 1; y0 += EPI4_YR) {
-        if (pend < 0) { pend = y0; continue; }
-        out.push_back(tile_entry(wr, x, pend, n, false));
-        out.push_back(tile_entry(wr, x, y0, n, false));
-        pend = -1;
-    }
-    if (pend >= 0) {
-        out.push_back(tile_entry(wr, x, pend, n, false));
-        out.push_back(tile_entry(wr, x, pend, n, true));
-    }
-}
-
 int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) {
     const int32_t n = c->n;
     std::vector<uint64_t>& tiles = c->host_tiles;
     tiles.clear();
     for (int32_t x = 1; x <= n - 2; ++x)
-        for (int32_t wr = 0; wr * EPI4_WU < x; ++wr) {
-            if (slab_w0 >= 0 && (wr * EPI4_WU < slab_w0 || wr * EPI4_WU >= slab_w0 + EPI4_WP)) continue;
-            append_pairs_z1(tiles, n, wr, x);
+        for (int32_t wp = 0; wp * EPI4_WP < x; ++wp) {
+            if (slab_w0 >= 0 && wp * EPI4_WP != slab_w0) continue;
+            for (int32_t y0 = x + 1; y0 <= n - 1; y0 += EPI4_YR_TC)
+                tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
+                                ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
         }
     if (tiles.empty()) return 0;
-    CU(grow(c->d_tiles3, c->cap_tiles3, tiles.size() * sizeof(uint64_t)));
-    CU(cudaMemcpyAsync(c->d_tiles3, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice, c->stream));
+    CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
+    CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice, c->stream));
     const int32_t grid = std::max(2, (c->opts.grid > 0 ? c->opts.grid : c->sm_count) / 2 * 2);
     if (int r = ensure_lists(c, grid, 1)) return r;
     SearchParams sp{};
     sp.d = devdata(c);
-    sp.tile_info = c->d_tiles3;
-    sp.ntiles = (int64_t)tiles.size() / 2;
+    sp.tile_info = c->d_tiles;
+    sp.ntiles = (int64_t)tiles.size();
     sp.t3_out = out;
     sp.t3_slab_w0 = slab_w0;
     sp.topk = 1;
@@ -525,7 +418,7 @@ namespace {
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
     c->loaded = false;
     c->n = n;
-    c->npad = (n + 16 + 63) / 64 * 64;   // rows past n read as zero planes (y up to n + 13, the all-ones row n, w < 64 ceil(n / 64))
+    c->npad = (n + EPI4_YR + EPI4_WP - 1) / EPI4_WP * EPI4_WP;   // rows past n read as zero planes
     c->np[0] = n0;
     c->np[1] = n1;
     for (int p = 0; p < 2; ++p) {
@@ -603,7 +496,6 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_idx, EPI4_MAX_TOPK * sizeof(uint64_t));
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_n, sizeof(int32_t));
     for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&c->ev[i]);
-    if (e == cudaSuccess) e = cudaMallocHost(&c->h_out, 512);
     if (e != cudaSuccess) {
         epi4_destroy(c);
         return fail(EPI4_ECUDA, "create: %s", cudaGetErrorString(e));
@@ -619,10 +511,8 @@ void epi4_destroy(epi4_ctx* c) {
     if (c->stream) cudaStreamSynchronize(c->stream);
     release_data(c);
     dfree(c->d_units);
+    dfree(c->d_prefix);
     dfree(c->d_tiles);
-    dfree(c->d_tiles3);
-    dfree(c->d_gprefix);
-    if (c->h_out) cudaFreeHost(c->h_out);
     dfree(c->d_counters);
     dfree(c->d_list_k2);
     dfree(c->d_list_idx);
@@ -831,12 +721,43 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!quads_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
     CU(cudaSetDevice(c->device));
-    const bool tcp = c->opts.pipe != EPI4_PIPE_LOP3;
-    if (tcp && std::max(c->np[0], c->np[1]) > ((int64_t)1 << 24))
+    std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
+    const int64_t nall = (int64_t)plan.size();
+    if (ue < 0 || ue > nall) ue = nall;
+    if (ub < 0) ub = 0;
+    if (ub > ue) ub = ue;
+    const int64_t nu = ue - ub;
+    if (c->opts.pipe != EPI4_PIPE_LOP3 && std::max(c->np[0], c->np[1]) > ((int64_t)1 << 24))
         return fail(EPI4_EINVAL, "tensor-core pipe: fp32 accumulators are exact up to 2^24 samples per phenotype "
                                  "(%lld, %lld); use EPI4_PIPE_LOP3", (long long)c->np[0], (long long)c->np[1]);
-    if (int r = prepare_units(c, ub, ue)) return r;
-    const SearchPlan& pl = c->plan;
+    const int32_t G = quad_split(c->opts.pipe), YR = quad_yr(c->opts.pipe);
+    std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
+    for (int64_t i = 0; i < nu; ++i) units[(size_t)i] = plan[(size_t)(ub + i)].u;
+    // Windowed T3: the units are taken grouped by (w-range R, 128-SNP x-range X) so that each launch reads
+    // only the slabs FIRST(R) and FIRST(X) (rebuilt on the tensor cores when R or X changes); the result does
+    // not depend on the order (top-k by (K2, index)).  Resident T3: one group, the plan order.
+    struct Group { int64_t b, e; int32_t wr, xr; };
+    std::vector<Group> groups;
+    if (c->t3_windowed && nu > 0) {
+        std::stable_sort(units.begin(), units.begin() + nu, [](const Unit& p, const Unit& q) {
+            return p.wr != q.wr ? p.wr < q.wr : p.x < q.x;
+        });
+        for (int64_t i = 0; i < nu; ++i) {
+            const int32_t xr = units[(size_t)i].x / EPI4_WP;
+            if (groups.empty() || groups.back().wr != units[(size_t)i].wr || groups.back().xr != xr)
+                groups.push_back(Group{i, i, units[(size_t)i].wr, xr});
+            groups.back().e = i + 1;
+        }
+    } else if (nu > 0) {
+        groups.push_back(Group{0, nu, -1, -1});
+    }
+    if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
+        dfree(c->d_units);
+        dfree(c->d_prefix);
+        c->units_cap = (size_t)std::max<int64_t>(nu, 1);
+        CU(cudaMalloc(&c->d_units, c->units_cap * sizeof(Unit)));
+        CU(cudaMalloc(&c->d_prefix, c->units_cap * sizeof(int64_t)));
+    }
     int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
     grid = std::max(2, grid / 2 * 2);                 // whole CTA pairs
     if (int r = ensure_lists(c, grid, top_k)) return r;
@@ -844,9 +765,16 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaMemsetAsync(c->d_counters, 0, 32 * sizeof(unsigned long long), c->stream));
     CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
 
-    SearchParams sp{};
+    SearchParams sp;
     sp.d = devdata(c);
+    sp.units = c->d_units;
+    sp.prefix = c->d_prefix;
+    sp.tile_info = nullptr;
+    sp.t3_out = nullptr;
     sp.t3_slab_w0 = -1;
+    sp.search3 = 0;
+    sp.nunits = 0;
+    sp.ntiles = 0;
     sp.tile_counter = c->d_counters;
     sp.topk = top_k;
     sp.list_k2 = c->d_list_k2;
@@ -876,9 +804,16 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaEventRecord(c->ev[2], c->stream));
     int64_t acc = 0;
     int32_t slab_r = -1, slab_x = -1;
-    for (const SearchPlan::Group& gr : pl.groups) {
-        const int64_t gn = gr.e - gr.b, gtiles = pl.prefix_host[(size_t)gr.e - 1];
-        if (gtiles == 0) continue;
+    std::vector<int64_t> prefix;
+    for (const Group& gr : groups) {
+        const int64_t gn = gr.e - gr.b;
+        prefix.assign((size_t)gn, 0);
+        int64_t gacc = 0;
+        for (int64_t i = 0; i < gn; ++i) {
+            gacc += unit_tiles(c->n, units[(size_t)(gr.b + i)].x, YR) * G;
+            prefix[(size_t)i] = gacc;
+        }
+        if (gacc == 0) continue;
         if (c->t3_windowed) {
             if (gr.wr != slab_r) {            // FIRST(R) into T3
                 if (int r = build_t3_tc(c, c->T3, gr.wr * EPI4_WP, &c->stats.launches)) return r;
@@ -895,39 +830,30 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
             sp.d.T3 = c->T3;
             sp.d.T3x = gr.xr == gr.wr ? c->T3 : c->T3x;
         }
-        // this group's units and their inclusive tile (CUDA core) / pair-tile (tensor core) prefix, on the device
-        sp.units = c->d_units + gr.b;
-        sp.prefix = c->d_gprefix + gr.b;
+        // pageable host source: the copy has completed when cudaMemcpyAsync returns, so `prefix` may be reused
+        CU(cudaMemcpyAsync(c->d_units, units.data() + gr.b, gn * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
+        CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), gn * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
         sp.nunits = gn;
-        if (!tcp) {
-            sp.ntiles = gtiles;
-            CU(launch_quad_lop3(sp, grid, c->stream, &c->stats.launches));
-        } else {
-            // pair tiles in chunks of at most tile_chunk (bounded tile-table memory; one persistent launch each)
-            for (int64_t t0 = 0; t0 < gtiles; t0 += c->tile_chunk) {
-                const int64_t t1 = std::min(gtiles, t0 + c->tile_chunk);
-                const bool cached = pl.table_cached && pl.groups.size() == 1 && t0 == 0 && t1 == gtiles;
-                if (!cached) {
-                    CU(launch_tile_table(sp, t0, t1, c->d_tiles, c->stream, &c->stats.launches));
-                    if (pl.groups.size() == 1 && t0 == 0 && t1 == gtiles) c->plan.table_cached = true;
-                }
-                sp.tile_info = c->d_tiles;
-                sp.ntiles = t1 - t0;
-                CU(launch_quad_tc(sp, grid, c->stream, &c->stats.launches));
-            }
+        sp.ntiles = gacc;
+        sp.tile_info = nullptr;
+        if (c->opts.pipe != EPI4_PIPE_LOP3) {
+            CU(grow(c->d_tiles, c->cap_tiles, (size_t)gacc * sizeof(uint64_t)));
+            sp.tile_info = c->d_tiles;
+            CU(launch_tile_table(sp, c->d_tiles, c->stream, &c->stats.launches));
         }
-        acc += gtiles;
+        cudaError_t e = c->opts.pipe == EPI4_PIPE_LOP3 ? launch_quad_lop3(sp, grid, c->stream, &c->stats.launches)
+                                                       : launch_quad_tc(sp, grid, c->stream, &c->stats.launches);
+        CU(e);
+        acc += gacc;
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(launch_merge(sp, grid, c->d_out_k2, c->d_out_idx, c->d_out_n, c->stream, &c->stats.launches));
-    int32_t* h_n = reinterpret_cast<int32_t*>(c->h_out);
-    unsigned long long* h_ctr = reinterpret_cast<unsigned long long*>(c->h_out + 16);
-    unsigned int* h_st = reinterpret_cast<unsigned int*>(c->h_out + 8);
-    CU(cudaMemcpyAsync(h_n, c->d_out_n, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
-    CU(cudaMemcpyAsync(h_st, c->d_status, sizeof(unsigned int), cudaMemcpyDeviceToHost, c->stream));
+    int32_t nout = 0;
+    unsigned long long ctr[32] = {0};
+    CU(cudaMemcpyAsync(&nout, c->d_out_n, sizeof nout, cudaMemcpyDeviceToHost, c->stream));
     CU(cudaMemcpyAsync(quads_out, c->d_out_idx, (size_t)top_k * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
     CU(cudaMemcpyAsync(k2_out, c->d_out_k2, (size_t)top_k * sizeof(double), cudaMemcpyDeviceToHost, c->stream));
-    CU(cudaMemcpyAsync(h_ctr, c->d_counters, 32 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaMemcpyAsync(ctr, c->d_counters, sizeof ctr, cudaMemcpyDeviceToHost, c->stream));
     CU(cudaEventRecord(c->ev[4], c->stream));
     CU(cudaStreamSynchronize(c->stream));
     float ms = 0;
@@ -935,16 +861,17 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     c->stats.ms_quad = ms;
     CU(cudaEventElapsedTime(&ms, c->ev[3], c->ev[4]));
     c->stats.ms_merge = ms;
-    c->stats.quads = (int64_t)h_ctr[1];
-    for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)h_ctr[16 + i];
-    c->stats.tiles = acc;
-    // MACs the contraction executes: per tile 64 w x 16 y x 16 (b, c, d, a) per sample, the tensor-core operands
-    // over whole 512-sample steps (two fp4 chunks, zero-padded) and both tiles of every pair (incl. a skipped
-    // one), the CUDA-core kernel over 128-sample chunks
-    const double ksamples = tcp ? (double)(sp.d.nsteps[0] + sp.d.nsteps[1]) * 512.0
-                                : (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES;
-    c->stats.executed_macs = (double)acc * (tcp ? 2.0 : 1.0) * EPI4_WU * EPI4_YR * 16.0 * ksamples;
-    *n_out = *h_n;
+    c->stats.quads = (int64_t)ctr[1];
+    for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)ctr[16 + i];
+    c->stats.tiles = acc / G;
+    // MACs the contraction executes: 256 (w, a) rows (a 128-SNP w-range) x 8 YR columns per unit tile and
+    // sample; the tensor-core operands run over whole 512-sample steps (two fp4 chunks, zero-padded), the
+    // CUDA-core kernel over 128-sample chunks
+    const double ksamples = c->opts.pipe == EPI4_PIPE_LOP3
+                                ? (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES
+                                : (double)(sp.d.nsteps[0] + sp.d.nsteps[1]) * 512.0;
+    c->stats.executed_macs = (double)(acc / G) * 256.0 * 8.0 * YR * ksamples;
+    *n_out = nout;
     return 0;
 }
 
@@ -961,10 +888,15 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
     std::vector<uint64_t>& tiles = c->host_tiles;
     tiles.clear();
-    for (const PlanEntry& pe : plan) append_pairs_z1(tiles, c->n, pe.u.wr, pe.u.x);
+    auto add = [&](int32_t wr, int32_t x) {
+        for (int32_t y0 = x + 1; y0 <= c->n - 1; y0 += EPI4_YR_TC)
+            tiles.push_back((uint64_t)(uint16_t)wr | ((uint64_t)(uint16_t)x << 16) | ((uint64_t)(uint16_t)y0 << 32) |
+                            ((uint64_t)(uint16_t)c->n << 48));
+    };
+    for (const PlanEntry& pe : plan) add(pe.u.wr, pe.u.x);
     // the 4-way plan has no units with x = n - 2 (no room for z); their triples (w, n - 2, n - 1) go to rank 0
     if (c->opts.rank == 0)
-        for (int32_t wr = 0; wr * EPI4_WU < c->n - 2; ++wr) append_pairs_z1(tiles, c->n, wr, c->n - 2);
+        for (int32_t wr = 0; wr * EPI4_WP < c->n - 2; ++wr) add(wr, c->n - 2);
     int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
     grid = std::max(2, grid / 2 * 2);
     if (int r = ensure_lists(c, grid, top_k)) return r;
@@ -984,11 +916,11 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     c->stats.launches = 0;
     CU(cudaEventRecord(c->ev[2], c->stream));
     if (!tiles.empty()) {
-        CU(grow(c->d_tiles3, c->cap_tiles3, tiles.size() * sizeof(uint64_t)));
-        CU(cudaMemcpyAsync(c->d_tiles3, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice,
+        CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
+        CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice,
                            c->stream));
-        sp.tile_info = c->d_tiles3;
-        sp.ntiles = (int64_t)tiles.size() / 2;
+        sp.tile_info = c->d_tiles;
+        sp.ntiles = (int64_t)tiles.size();
         CU(launch_quad_tc(sp, grid, c->stream, &c->stats.launches));
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
@@ -1004,7 +936,7 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     CU(cudaEventElapsedTime(&ms, c->ev[2], c->ev[3]));
     c->stats.ms_quad = ms;
     c->stats.quads = (int64_t)ctr[1];
-    c->stats.tiles = (int64_t)tiles.size() / 2;
+    c->stats.tiles = (int64_t)tiles.size();
     *n_out = nout;
     return 0;
 }

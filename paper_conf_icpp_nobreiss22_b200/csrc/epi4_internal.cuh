@@ -22,11 +22,12 @@
 #include "../../include/epi4.h"
 
 #define EPI4_B 32             // SNP block size accepted in epi4_opts (32-SNP blocks)
-#define EPI4_WU 64            // w-range of a work unit: 64 first SNPs (the N = 128 = 64 x {AA, Aa} columns of the
-                              // tensor-core tile, the 64 threads of a CUDA-core tile)
-#define EPI4_WP 128           // first-SNP range of one windowed-T3 slab
-#define EPI4_YR 16            // y-range of a tile: 16 consecutive SNPs after x (both pipes)
-#define EPI4_YR_TC EPI4_YR
+#define EPI4_WR 64            // w-range of one CTA / rows of its A operand: 64 SNPs x {AA, Aa}
+#define EPI4_WP 128           // w-range of a work unit (a CTA pair: two 64-SNP halves)
+#define EPI4_YR 16            // y-range of a CUDA-core (LOP3) tile: 16 consecutive SNPs after x
+#ifndef EPI4_YR_TC
+#define EPI4_YR_TC 16         // y-range of a tensor-core tile (N = 128 = 16 x 8 columns; measured best, k_quad_tc.cu)
+#endif
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
 
@@ -58,7 +59,7 @@ struct DevData {
     int32_t nchunks[2];          // 128-sample chunks per phenotype
     int32_t nchunks4[2];         // 256-sample fp4 chunks per phenotype (rows of expl)
     int32_t nsteps[2];           // tensor-core pipeline steps per phenotype: pairs of fp4 chunks (512 samples)
-    int32_t nrb;                 // 64-row blocks of expl per chunk (= npad / 32)
+    int32_t nrb;                 // 128-row blocks of expl per chunk (= npad / 64)
     int32_t pk_shift;            // (control, case) counts packed as c0 | c1 << pk_shift everywhere (bits(n0))
     int32_t n;                   // SNPs
     int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
@@ -84,11 +85,11 @@ struct DevData {
     double mi_E;                 // fp32 MI filter: rounding bound (bits) on V = sum_c [X2(r0) + X2(r1) - X2(r_c)]
 };
 
-// byte offset of (fp4 chunk C, row r = 2 snp + g) in expl: blocked [chunk pair][64-row block][C & 1][row][128 B]
-// so that the 2 chunks x 64 rows (32 SNPs x {AA, Aa}) of one CTA's B operand are one contiguous 16 KiB bulk copy;
-// nrb = 64-row blocks per chunk (= npad / 32)
+// byte offset of (fp4 chunk C, row r = 2 snp + g) in expl: blocked [chunk pair][128-row block][C & 1][row][128 B]
+// so that the 2 chunks x 128 rows of one A tile are one contiguous 32 KiB bulk copy (a 16 KiB copy is processed
+// at ~42 B/clk/SM, a 32 KiB copy at ~75: tools/probe_tma3.cu)
 __host__ __device__ __forceinline__ int64_t expl_off(int64_t C, int64_t r, int32_t nrb) {
-    return ((((C >> 1) * nrb + (r >> 6)) * 2 + (C & 1)) * 64 + (r & 63)) * 128;
+    return ((((C >> 1) * nrb + (r >> 7)) * 2 + (C & 1)) * 128 + (r & 127)) * 128;
 }
 
 // offset (in uint32 words) of (chunk kc, snp, g, word w) in a chunked plane array
@@ -96,12 +97,13 @@ __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, 
     return ((kc * npad + snp) * 2 + g) * EPI4_CHUNK_WORDS + w;
 }
 
-// A work unit (wr, x): the quads (w, x, y, z) with w in the 64-SNP range [64 wr, 64 wr + 64), w < x, second SNP
-// x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + 16) with y0 = x + 1 + 16 k, and z in (y0, n);
-// a tile holds 64 x 16 (w, y) combinations.  The tensor-core kernel runs the tiles of a unit in pairs (one per
-// CTA of a cluster, sharing the unit's w operand); an odd last tile is paired with a skipped copy of itself.
+// A work unit (wp, x): the quads (w, x, y, z) with w in the 128-SNP range [128 wp, 128 wp + 128), w < x,
+// second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + yr) with y0 = x + 1 + yr k,
+// and z in (y0, n); a tile holds 128 x yr (w, y) combinations (yr = EPI4_YR_TC tensor core, EPI4_YR CUDA core), split into
+// the two 64-SNP halves of the w-range (the two CTAs of a tensor-core cluster, or two tiles of the CUDA-core
+// kernel).
 struct Unit {
-    int32_t wr, x;   // wr = 64-SNP w-range index
+    int32_t wr, x;   // wr = 128-SNP w-range index
 };
 
 __host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x, int32_t yr = EPI4_YR) {
@@ -109,7 +111,6 @@ __host__ __device__ __forceinline__ int64_t unit_tiles(int32_t n, int32_t x, int
     for (int32_t y0 = x + 1; y0 <= n - 2; y0 += yr) t += n - y0 - 1;
     return t;
 }
-__host__ __device__ __forceinline__ int64_t unit_pairs(int32_t n, int32_t x) { return (unit_tiles(n, x) + 1) / 2; }
 
 // decode tile t of unit (x) -> (y0, z), y-range yr
 __device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t, int32_t& y0, int32_t& z,
@@ -123,12 +124,6 @@ __device__ __forceinline__ void unit_tile_decode(int32_t n, int32_t x, int64_t t
         t -= cnt;
     }
     z = n;  // unreachable for valid t
-}
-
-// tensor-core tile table entry (one per CTA of a pair tile): wr | skip << 15 | x << 16 | y0 << 32 | z << 48
-__host__ __device__ __forceinline__ uint64_t tile_entry(int32_t wr, int32_t x, int32_t y0, int32_t z, bool skip) {
-    return (uint64_t)(wr & 0x7FFF) | ((uint64_t)(skip ? 1 : 0) << 15) | ((uint64_t)(uint16_t)x << 16) |
-           ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)z << 48);
 }
 
 // find the unit of a flat tile index by binary search on the inclusive prefix of tile counts
@@ -145,13 +140,13 @@ __device__ __forceinline__ int64_t find_unit(const int64_t* prefix, int64_t nuni
 struct SearchParams {
     DevData d;
     const Unit* units;
-    const int64_t* prefix;     // inclusive prefix of tiles (CUDA-core pipe) / pair tiles (tensor-core pipe) per unit
-    const uint64_t* tile_info; // (tensor-core pipe) 2 entries per pair tile, tile_entry() (k_tile_table)
+    const int64_t* prefix;     // inclusive prefix of tiles per unit
+    const uint64_t* tile_info; // (tensor-core pipe) decoded tiles: wp | x << 16 | y0 << 32 | z << 48 (k_tile_table)
     uint32_t* t3_out;          // non-NULL: 3-way-table mode of k_quad_tc (z = the all-ones SNP n, writes T3)
     int32_t t3_slab_w0;        // 3-way-table mode: < 0 resident colex layout, else the slab FIRST([w0, w0+128))
     int32_t search3;           // third-order search mode (z = the all-ones SNP n, epi4_search3)
     int64_t nunits;
-    int64_t ntiles;            // tiles (CUDA-core pipe) / pair tiles (tensor-core pipe)
+    int64_t ntiles;
     unsigned long long* tile_counter;   // dynamic scheduler
     int32_t topk;              // list capacity used (<= EPI4_MAX_TOPK)
     double* list_k2;           // per-CTA lists [grid][topk]
@@ -207,8 +202,9 @@ cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T
                        cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
-cudaError_t launch_tile_table(const SearchParams& sp, int64_t t0, int64_t t1, uint64_t* out, cudaStream_t s,
-                              int64_t* launches);
+cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches);
+int32_t quad_split(int32_t pipe);   // tiles per unit tile (CUDA-core kernel: the two 64-SNP halves)
+int32_t quad_yr(int32_t pipe);      // y-range of a tile
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,
                          int32_t* out_n, cudaStream_t s, int64_t* launches);
 cudaError_t launch_tables(const DevData& d, const uint64_t* quads, int64_t n, uint32_t* out, unsigned int* status,

@@ -189,7 +189,7 @@ __global__ void __launch_bounds__(256) k_expand(const uint32_t* __restrict__ pla
         o[k] = v;
     }
     const int sw = cc ^ (int)(r & 7);
-    reinterpret_cast<uint4*>(expl + expl_off(C, r, npad / 32))[sw] = make_uint4(o[0], o[1], o[2], o[3]);
+    reinterpret_cast<uint4*>(expl + expl_off(C, r, npad / 64))[sw] = make_uint4(o[0], o[1], o[2], o[3]);
 }
 
 cudaError_t launch_expand(const uint32_t* planes, int32_t npad, int32_t nchunks, uint8_t* expl, cudaStream_t s,

@@ -1,6 +1,6 @@
 // k_quad_lop3.cu — CUDA-core contraction (EPI4_PIPE_LOP3): AND + POPC on bit planes.
 //
-// The cross-check pipe of SURVEY.md §8(a) a5: for each tile (the unit's 64-SNP w-range wr, x,
+// The cross-check pipe of SURVEY.md §8(a) a5: for each tile (64-SNP half wr of a unit's w-range, x,
 // y-range y0, z) the 64 x 16
 // (w, y) combinations are counted directly: for each 32-sample word, the pair rows
 // (w,x,a,b) = P_a(w) & P_b(x) ("combine") are ANDed with the pair columns
@@ -36,12 +36,12 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
         __syncthreads();
         if (tile >= sp.ntiles) break;
         const int64_t u = find_unit(sp.prefix, sp.nunits, tile);
-        const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);
-        const int32_t wr = sp.units[u].wr, x = sp.units[u].x;
+        const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);   // = 2 * unit tile + half
+        const int32_t wr = sp.units[u].wr * 2 + (int32_t)(t & 1), x = sp.units[u].x;
         int32_t y0, z;
-        unit_tile_decode(d.n, x, t, y0, z, EPI4_YR);
+        unit_tile_decode(d.n, x, t >> 1, y0, z, EPI4_YR);
         const int i = tid & 63, jg = tid >> 6;
-        const int w = wr * EPI4_WU + i;
+        const int w = wr * EPI4_WR + i;
 
         uint32_t cnt[2][LOP3_Q][16];
 #pragma unroll

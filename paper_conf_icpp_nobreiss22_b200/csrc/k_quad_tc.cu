@@ -2,48 +2,49 @@
 // (tcgen05.mma.cta_group::2.kind::mxf4, E2M1 {0, 1.0} operands, fp32 accumulators in TMEM) with the fused
 // epilogue.
 //
-// What it computes: for a tile (64-SNP w-range wr, x, y-range y0, z) and each
-// phenotype p the 128 x 128 matrix
-//     C_p[(y, b, c, d)][(w, a)] = sum over samples s of phenotype p of P_b(x)[s] P_c(y)[s] P_d(z)[s] P_a(w)[s]
-// for the 16 SNPs y = y0..y0+15 and the 64 SNPs w of the range: the 16 non-aa genotype counts of the 64 x 16
-// quads (w, x, y, z) ("a matrix with 16 values per each quad").
+// What it computes: for a tile (w-range pair wp, x, y-range y0, z) and each
+// phenotype p the 256 x N matrix (N = 8 YR, YR = EPI4_YR_TC = 16 y per tile, N = 128)
+//     C_p[(w, a)][(y, b, c, d)] = sum over samples s of phenotype p of P_a(w)[s] P_b(x)[s] P_c(y)[s] P_d(z)[s]
+// for the 128 SNPs w of the range pair and the YR SNPs y = y0..y0+YR-1: the 16 non-aa genotype counts of the
+// 128 x YR quads (w, x, y, z) ("a matrix with 16 values per each quad").
 // Factorisation: the paper ANDs SNP pairs into both operands (combine);
-// here the A operand (M side) holds TRIPLE products P_b(x) & P_c(y) & P_d(z), built on chip from a few single-SNP
-// planes, and the B operand (N side) the raw single-SNP planes (w, a), copied from L2 by the TMA engine.
-// Why this way round (round 2; tools/probe_smem_bw.cu, profiles/r02_*): the operand streamed from L2 is the one
-// whose rows each carry only one SNP.  With the singles on the M side (round 1) every 128 x 128 x 512-sample step
-// streamed 32 KiB of A per CTA from L2 (64 B/clk/SM at the full MMA rate) — above the ~41 B/clk/SM the L2 delivers
-// to every SM at once, so the tensor pipe idled ~half the time; now a step streams the 16 KiB of w singles plus
-// ~4.5 KiB of x/y/z singles for the producers.  The w range per tile also shrinks from 128 to 64 SNPs, which halves
-// the diagonal waste (rows w >= x of the units whose x lies inside their own w-range).
+// here the A operand is the raw single-SNP planes (w, a), copied from HBM by the TMA engine, and x is folded
+// into the B operand, whose columns are triple products P_b(x) & P_c(y) & P_d(z) built on chip.
 // Why block-scaled FP4: sm_100a has no native binary tensor op (ptxas emulates mma.sync ...b1.and.popc with
 // legacy IMMA).  A set bit is the E2M1 value 1.0 (nibble 0x2), so AND of packed nibbles
 // is the product, and with all E8M0 block scales = 1 the MMA sums exact small integers: the fp32 accumulator
 // is exact up to 2^24 per phenotype (host check; tools/probe_mxf4.cu: 0 mismatches, counts to 76800).
-// kind::mxf4 runs M=256 K=64 in N/2 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the operand bytes.
+// kind::mxf4 runs M=256 K=64 in N/2 cycles: twice the {0,1}-MACs of kind::i8 (K=32) at half the operand
+// bytes (2 samples per byte).
 // Why 2-CTA: a 1-CTA M=128 MMA issues every ~97 cycles whatever N; cta_group::2 reaches the full rate.
+// Why N = 128: the A operand is streamed from L2 once per (tile, sample chunk), 128 B per row and 256 samples
+// for every N columns (N = 128 needs 64 B/clk/SM of A at the full MMA rate, below the ~75 B/clk/SM an SM
+// ingests with 32 KiB copies, tools/probe_tma3.cu); N = 160 (20 y) and 96 (12 y) were measured 3 % and 9 %
+// slower at C2 and equal at C5.  TMEM holds three regions of N fp32 columns plus the scale
+// factors; tile t accumulates its controls in region (-t) mod 3 and its cases in the next one.  When the tile
+// is done the epilogue first packs every (control, case) pair into one 32-bit word in the case region and
+// zeroes the control region (pass 1, a few hundred cycles), which the case accumulation of tile t+1 reuses;
+// it then scores the quads from the packed region (pass 2), which the control accumulation of tile t+2
+// reuses (two buffers of 2 x N columns would not fit in 512 at N = 160).
 //
-// CTA pair (cluster of 2) = one PAIR TILE: two tiles of the same unit (wr, x), one per CTA.  CTA r holds the A rows
-// of its own tile (16 y x 8 (b, c, d) = 128 rows) and the B rows of w = 64 wr + 32 r .. + 31 (64 rows: the pair's
-// N = 128 columns are split between the CTAs); the leader (r = 0) issues the MMAs for both, and each CTA's TMEM
-// receives its 128 rows x all 128 columns: lane 8 y_l + 4b + 2c + d, column 2 w_l + a.  TMEM holds three regions
-// of 128 fp32 columns plus the scale factors; tile t accumulates its controls in region (-t) mod 3 and its cases
-// in the next one.  When the tile is done the epilogue first packs every (control, case) pair into one 32-bit
-// word in the case region and zeroes the control region (pass 1), which the case accumulation of tile t+1 reuses;
-// it then scores the quads from the packed region (pass 2), which the control accumulation of tile t+2 reuses.
+// CTA pair (cluster of 2): CTA r holds the A rows of w-range 2wp + r (64 SNPs x {AA, Aa}) and builds the
+// B columns of y = y0 + r YR/2 .. y0 + (r + 1) YR/2 - 1; the leader (r = 0) issues the MMAs for both; each
+// CTA's TMEM receives its 128 rows x all N columns and its epilogue scores its 64 x YR quads.
 // Warp roles (each CTA: 16 warps = 4 warpgroups with setmaxnreg budgets, 1 CTA per SM, persistent, static
-// pair-tile stride over clusters):
+// tile stride over clusters):
 //   warps 0..1  : leader — MMA issuers (alternating steps, one elected lane each); follower — warp 0 relays
-//                 "B landed" to the leader's barrier; warp 0 also allocates TMEM (cta_group::2)
-//   warps 2..3  : TMA issuers (alternating steps): the CTA's 64 B rows, one 16 KiB bulk copy per step,
-//                 pre-swizzled in HBM
-//   warps 4..7  : producers (one chunk of every 2nd step each) — the CTA's A, x_b & y_c & z_d per 16-byte piece,
-//                 K-major SW128, from singles loaded into registers one step ahead; then an arrival on the
-//                 leader's barrier
-//   warps 8..15 : epilogue — pass 1 (pack, arrive `pk`), pass 2: tcgen05.ld of the packed counts, an 8 x 8
-//                 transpose across the 8 (b, c, d) lanes of each y so that one thread holds one quad's 16 packed
-//                 counts, re-zeroing, the shared per-quad evaluation (epilogue.cuh); an arrival on `ep`
-// One step = two 256-sample fp4 chunks of one phenotype = 8 MMAs (M=256, N=128, K=64).
+//                 "A landed" to the leader's `full` barrier; warp 0 also allocates TMEM (cta_group::2)
+//   warps 2..3  : TMA issuers (alternating steps): the CTA's A, one 32 KiB bulk copy per step, pre-swizzled in HBM
+//   warps 4..7  : producers (one chunk of every 2nd step each) — the CTA's half of B, x_b & y_c & z_d per
+//                 16-byte piece, K-major SW128, from singles loaded into registers one step ahead; then an
+//                 arrival on the leader's `full`
+//   warps 8..15 : epilogue — pass 1 (pack, arrive `pk`), pass 2: tcgen05.ld of the packed counts, lane-pair
+//                 exchange so one thread holds one quad's 2 x 16 counts, re-zeroing, the shared per-quad
+//                 evaluation (epilogue.cuh); an arrival on the leader's `ep` barrier
+// Pipelines: STAGES x {A, B half} per CTA (sfull: own TMA landed; full @leader: both B halves built and the
+// follower's A landed; empty: the issuer's MMA commit, multicast to both CTAs); TMEM: the region rotation
+// above (tfull -> epilogue; pk, ep -> MMA issuers).  One step = two 256-sample fp4 chunks of one phenotype =
+// 8 MMAs.
 #include <cstdio>
 #include <cstdlib>
 #include <type_traits>
@@ -52,51 +53,62 @@
 namespace epi4 {
 
 namespace tc {
-constexpr int M = 256, N = 2 * EPI4_WU;  // UMMA shape (cta_group::2), K = 64 fp4 = 32 bytes per instruction
-constexpr int YT = EPI4_YR;              // y per tile (per CTA)
+constexpr int M = 256, N = 8 * EPI4_YR_TC;   // UMMA shape (cta_group::2), K = 64 fp4 = 32 bytes per instruction
 constexpr int ROWB = 128;                // bytes of one K-major operand row per fp4 chunk (256 samples)
-constexpr int CHUNKS = 2;                // fp4 chunks per pipeline stage (512 samples)
-constexpr int A_ROWS = 8 * YT;           // this CTA's A rows: (y, b, c, d) (128)
-constexpr int A_SUB = A_ROWS * ROWB;     // one chunk of A (16 KiB)
-constexpr int A_BYTES = CHUNKS * A_SUB;  // produced per stage (32 KiB)
-constexpr int B_ROWS = N / 2;            // this CTA's B rows (64 = 32 w x {AA, Aa})
-constexpr int B_SUB = B_ROWS * ROWB;     // 8 KiB
-constexpr int B_BYTES = CHUNKS * B_SUB;  // one TMA copy per stage (16 KiB)
+constexpr int CHUNKS = 2;                // fp4 chunks per pipeline stage (512 samples): one 32 KiB A copy
+constexpr int A_SUB = 128 * ROWB;        // this CTA's 128 A rows of one chunk (16 KiB)
+constexpr int A_BYTES = CHUNKS * A_SUB;
+constexpr int B_ROWS = N / 2;            // this CTA's B columns (64)
+constexpr int B_SUB = (B_ROWS + 7) / 8 * 1024;
+constexpr int B_BYTES = CHUNKS * B_SUB;
+constexpr int YH = EPI4_YR_TC / 2;       // y SNPs per CTA (8)
+constexpr int TX_BYTES = A_BYTES;                          // bytes this CTA's TMA brings per A stage
+#ifndef EPI4_A_SPLIT
+#define EPI4_A_SPLIT 1
+#endif
+constexpr int A_SPLIT = EPI4_A_SPLIT;    // lanes issuing one A stage's bulk copy in pieces (tools/probe_tma.cu: several
+                                         // concurrently issued copies ingest faster than one)
 #ifndef EPI4_PROD_WARPS
 #define EPI4_PROD_WARPS 4
 #endif
-#ifndef EPI4_EPI_WARPS
-#define EPI4_EPI_WARPS 8
-#endif
-constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = EPI4_EPI_WARPS;
-static_assert(EPI_WARPS % 4 == 0 && PROD_WARPS % 4 == 0, "warpgroup-aligned roles (setmaxnreg, TMEM lane quadrants)");
-constexpr int EPI_NH = EPI_WARPS / 4;                     // epilogue warps per TMEM lane quadrant
+constexpr int PROD_WARPS = EPI4_PROD_WARPS, EPI_WARPS = 8;
 static_assert(PROD_WARPS % CHUNKS == 0, "producer warps come in groups of CHUNKS (one chunk of a step each)");
 constexpr int PROD_STRIDE = PROD_WARPS / CHUNKS;          // steps between two steps of one producer warp
-constexpr int MMA_ISSUERS = 2;           // leader CTA: two issuers alternate steps (one thread cannot hide
+#ifndef EPI4_MMA_ISSUERS
+#define EPI4_MMA_ISSUERS 2
+#endif
+constexpr int MMA_ISSUERS = EPI4_MMA_ISSUERS;   // 1: one issuer, MMAs complete in step order (any ring sizes)
+constexpr int MMA_WARPS = 2;             // leader CTA: two issuers alternate steps (one thread cannot hide
                                          // its own wait/bookkeeping latency behind the blocking MMA issue)
-constexpr int MMA_WARPS = 2;
 constexpr int TMA_WARPS = 2;             // a bulk-copy issue blocks its thread ~150-200 cycles: two warps alternate
 constexpr int TMA_WARP0 = MMA_WARPS, PROD_WARP0 = TMA_WARP0 + TMA_WARPS, EPI_WARP0 = PROD_WARP0 + PROD_WARPS;
-constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 512
-// register split across the 4 warpgroups (MMA+TMA | producers | 2 x epilogue), setmaxnreg
+constexpr int THREADS = 32 * (EPI_WARP0 + EPI_WARPS);         // 512 with 4 producer warps (128 registers each before setmaxnreg)
+// register split across the 4 warpgroups (needs the 16-warp layout: MMA+TMA | producers | 2 x epilogue)
+#ifndef EPI4_REGSPLIT
+#define EPI4_REGSPLIT 1
+#endif
+#ifndef EPI4_EPI_LOW
+#define EPI4_EPI_LOW 1
+#endif
+constexpr bool REGSPLIT = EPI4_REGSPLIT && PROD_WARPS == 4 && MMA_WARPS + TMA_WARPS == 4 && EPI_WARPS == 8;
 #ifndef EPI4_REGS_CTL
-#define EPI4_REGS_CTL 32
+#define EPI4_REGS_CTL 40
 #endif
 #ifndef EPI4_REGS_PROD
-#define EPI4_REGS_PROD (PROD_WARPS == 4 ? 128 : 64)
+#define EPI4_REGS_PROD 120
 #endif
-constexpr int NWARPS = EPI_WARP0 + EPI_WARPS;
-constexpr bool REGSPLIT = MMA_WARPS + TMA_WARPS == 4;
 constexpr int REGS_CTL = EPI4_REGS_CTL, REGS_PROD = EPI4_REGS_PROD;
-constexpr int REGS_EPI_RAW = (65536 / 32 - 4 * REGS_CTL - PROD_WARPS * REGS_PROD) / EPI_WARPS / 8 * 8;
-constexpr int REGS_EPI = REGS_EPI_RAW > 232 ? 232 : REGS_EPI_RAW;   // 176 with 4 producer / 8 epilogue warps
+constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;   // 176 with 40 / 120
+// measured (C2 kernel, same box): control/producers 56/104 520 ms, 48/112 503, 40/120 499, 32/128 504; the
+// epilogue needs >= 176 (48/120 -> 168: 561 ms); control 24 does not fit its code (illegal instruction)
+constexpr int gcd_c(int a, int b) { return b ? gcd_c(b, a % b) : a; }
+constexpr int lcm_c(int a, int b) { return a / gcd_c(a, b) * b; }
 constexpr int TMEM_COLS = 512;
 constexpr int REGIONS = 3;               // accumulator regions of N columns, rotated per tile (header comment)
 constexpr int ACC_COLS = REGIONS * N;
 constexpr int SF_COL = 480;              // scale factors (all E8M0 0x7F = 1.0): columns 480..511, every lane
 static_assert(ACC_COLS <= SF_COL, "TMEM: accumulators overlap the scale factors");
-constexpr int NG = N / 16;               // 16-column groups of an accumulator (8 w each)
+constexpr int NG = N / 16;               // 16-column groups of an accumulator (8)
 constexpr int CLUSTER = 2;
 // block-scaled instruction descriptor: A/B E2M1 (format 1 at bits 7 and 10), K-major, N>>3 at bit 17,
 // scale format E8M0 (bit 23), M>>4 at bit 24, scale-factor ids 0, K = 64 (bit 31 = 0)
@@ -263,65 +275,61 @@ __device__ __forceinline__ void cluster_sync_all() {
 }
 
 struct TileInfo {
-    int32_t wr, x, y0, z;
-    bool skip;
+    int32_t wp, x, y0, z;
 };
-__device__ __forceinline__ TileInfo unpack_tile(uint64_t v) {
+__device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t tile) {
+    const int64_t u = find_unit(sp.prefix, sp.nunits, tile);
+    const int64_t t = tile - (u ? sp.prefix[u - 1] : 0);
     TileInfo ti;
-    ti.wr = (int32_t)(v & 0x7FFF);
-    ti.skip = (v >> 15) & 1;
+    ti.wp = sp.units[u].wr;
+    ti.x = sp.units[u].x;
+    unit_tile_decode(sp.d.n, ti.x, t, ti.y0, ti.z, EPI4_YR_TC);
+    return ti;
+}
+
+// The tile table (one uint64 per tile, filled by k_tile_table before the search): a tile change in the hot
+// kernel costs one load instead of decode_tile's binary search over the unit prefix (~log2(units) dependent
+// global loads) and the y-range loop, which stalled the TMA / producer / epilogue warps at every tile change.
+__global__ void __launch_bounds__(256) k_tile_table(SearchParams sp, uint64_t* __restrict__ out) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= sp.ntiles) return;
+    const TileInfo ti = decode_tile(sp, t);
+    out[t] = (uint64_t)(uint16_t)ti.wp | ((uint64_t)(uint16_t)ti.x << 16) | ((uint64_t)(uint16_t)ti.y0 << 32) |
+             ((uint64_t)(uint16_t)ti.z << 48);
+}
+cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches) {
+    if (sp.ntiles <= 0) return cudaSuccess;
+    k_tile_table<<<(unsigned)((sp.ntiles + 255) / 256), 256, 0, s>>>(sp, out);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+__device__ __forceinline__ TileInfo load_tile(const SearchParams& sp, int64_t tile) {
+    const uint64_t v = __ldg(sp.tile_info + tile);
+    TileInfo ti;
+    ti.wp = (int32_t)(v & 0xFFFF);
     ti.x = (int32_t)((v >> 16) & 0xFFFF);
     ti.y0 = (int32_t)((v >> 32) & 0xFFFF);
     ti.z = (int32_t)(v >> 48);
     return ti;
 }
 
-// The tile table: pair tiles [t0, t1) of the units (2 entries each: the tiles 2p, 2p+1 of the unit, the second a
-// skipped copy of the first when the unit has an odd number of tiles), filled before each search launch so a tile
-// change in the hot kernel costs one load instead of a binary search over the unit prefix (round 1: -3 %).
-__global__ void __launch_bounds__(256) k_tile_table(SearchParams sp, int64_t t0, int64_t t1, uint64_t* __restrict__ out) {
-    const int64_t t = t0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= t1) return;
-    const int64_t u = find_unit(sp.prefix, sp.nunits, t);
-    const int64_t p = t - (u ? sp.prefix[u - 1] : 0);
-    const int32_t wr = sp.units[u].wr, x = sp.units[u].x;
-    int32_t y0a, za, y0b, zb;
-    unit_tile_decode(sp.d.n, x, 2 * p, y0a, za);
-    const bool skipb = 2 * p + 1 >= unit_tiles(sp.d.n, x);
-    if (skipb) { y0b = y0a; zb = za; }
-    else unit_tile_decode(sp.d.n, x, 2 * p + 1, y0b, zb);
-    out[2 * (t - t0)] = tile_entry(wr, x, y0a, za, false);
-    out[2 * (t - t0) + 1] = tile_entry(wr, x, y0b, zb, skipb);
-}
-cudaError_t launch_tile_table(const SearchParams& sp, int64_t t0, int64_t t1, uint64_t* out, cudaStream_t s,
-                              int64_t* launches) {
-    if (t1 <= t0) return cudaSuccess;
-    k_tile_table<<<(unsigned)((t1 - t0 + 255) / 256), 256, 0, s>>>(sp, t0, t1, out);
-    if (launches) ++*launches;
-    return cudaGetLastError();
-}
-__device__ __forceinline__ TileInfo load_tile(const SearchParams& sp, int64_t tile, uint32_t rank) {
-    return unpack_tile(__ldg(sp.tile_info + 2 * tile + rank));
-}
-
-// iterator over the (pair tile, phenotype, chunk) steps of this cluster; advance(k) moves k steps ahead.
+// iterator over the (tile, phenotype, chunk) steps of this cluster; advance(k) moves k steps ahead.
 // Chunk counts live in registers (runtime indexing of kernel-parameter arrays spills the parameter block).
 struct StepIt {
     int64_t tile;
     TileInfo ti;
     int p, kc;
     int nch0, nch1;
-    uint32_t rank;
-    __device__ __forceinline__ void init(const SearchParams& sp, uint32_t r) {
+    __device__ __forceinline__ void init(const SearchParams& sp) {
         tile = cluster_id_x();
         p = 0;
         kc = 0;
-        rank = r;
         nch0 = sp.d.nsteps[0];
         nch1 = sp.d.nsteps[1];
-        if (tile < sp.ntiles) ti = load_tile(sp, tile, rank);
+        if (tile < sp.ntiles) ti = load_tile(sp, tile);
     }
     __device__ __forceinline__ bool valid(const SearchParams& sp) const { return tile < sp.ntiles; }
+    // physical chunk of this step (a tile-dependent rotation of the K loop was measured slower: r01 notes)
     __device__ __forceinline__ int chunk() const { return kc; }
     __device__ __forceinline__ void advance(const SearchParams& sp, int k) {
         kc += k;
@@ -334,7 +342,7 @@ struct StepIt {
                 tile += nclusters_x();
             }
         }
-        if (tile != t0 && tile < sp.ntiles) ti = load_tile(sp, tile, rank);
+        if (tile != t0 && tile < sp.ntiles) ti = load_tile(sp, tile);
     }
 };
 
@@ -356,49 +364,26 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 #define PCLK() 0LL
 #endif
 
-// 8 x 8 transpose of 2-word elements across the 8 lanes L = lane & 7 of each y (butterfly over lane bits 4, 2, 1):
-// lane L enters with E_i = (v[2i], v[2i+1]) for i = 0..7 (its own (b, c, d) row, w_l = 8g + i, a = 0/1) and leaves
-// with slot s holding E_L of source lane s, i.e. v[2s + a] = count (a, bcd = s) of quad w_l = 8g + L.
-// Stage m: for every slot pair (i0, i1 = i0 | m) (bit m of i0 clear) the lane whose bit m is clear keeps slot i0
-// and replaces slot i1 with the partner's slot i0; the other keeps i1 and replaces i0 with the partner's i1.
-__device__ __forceinline__ void transpose8(uint32_t (&v)[16], int lane) {
-#pragma unroll
-    for (int m = 4; m >= 1; m >>= 1) {
-        const bool hi = (lane & m) != 0;
-#pragma unroll
-        for (int i0 = 0; i0 < 8; ++i0) {
-            if (i0 & m) continue;
-            const int i1 = i0 | m;
-#pragma unroll
-            for (int a = 0; a < 2; ++a) {
-                const uint32_t send = hi ? v[2 * i0 + a] : v[2 * i1 + a];
-                const uint32_t recv = __shfl_xor_sync(0xffffffffu, send, m);
-                if (hi) v[2 * i0 + a] = recv;
-                else v[2 * i1 + a] = recv;
-            }
-        }
-    }
-}
-
-// Global step s of a cluster uses produced-A stage s % SA (phase (s / SA) & 1) and TMA-B stage s % SB.  The two
-// MMA issuers may issue (and complete) the steps of the other parity out of order, so a waiter is only protected
+// Global step s of a cluster uses A stage s % SA (phase (s / SA) & 1) and B stage s % SB.  The two MMA
+// issuers may issue (and complete) the steps of the other parity out of order, so a waiter is only protected
 // from phase aliasing if its previous wait on a ring was on the same issuer's steps: both ring sizes must be
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
 template <int SA, int SB, bool PK16, int FILT>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
-    static_assert(SA % 2 == 0 && SA % tc::PROD_STRIDE == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::TMA_WARPS == 2,
+    static_assert(tc::MMA_ISSUERS == 1 ||
+                  (SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2),
                   "ring sizes must be multiples of the alternating warps' stride (phase aliasing)");
     extern __shared__ unsigned char smem_raw[];
-    // A ring (produced): afull (@leader: both CTAs' producers), aempty (MMA commit);
-    // B ring (TMA): bfull (own TMA landed), bpeer (@leader: the follower's B landed, relayed), bempty (MMA commit)
-    __shared__ __align__(8) uint64_t afull_bar[SA], aempty_bar[SA], bfull_bar[SB], bpeer_bar[SB], bempty_bar[SB];
+    // A ring: afull (own TMA landed), apeer (@leader: the follower's A landed, relayed), aempty (MMA commit);
+    // B ring: bfull (@leader: both CTAs' producers), bempty (MMA commit)
+    __shared__ __align__(8) uint64_t afull_bar[SA], apeer_bar[SA], aempty_bar[SA], bfull_bar[SB], bempty_bar[SB];
     __shared__ __align__(8) uint64_t tfull_bar[2], pk_bar, ep_bar[2];
     __shared__ uint32_t s_tmem;
     // 1024-aligned A ring, then the B ring, then the top-k state
     // (same offsets in both CTAs of the pair: the MMA addresses the peer's operands at the same offsets)
     const uint32_t raw = smem_u32(smem_raw);
-    unsigned char* aring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-    unsigned char* bring = aring + SA * tc::A_BYTES;
+    unsigned char* ring = smem_raw + (((raw + 1023u) & ~1023u) - raw);
+    unsigned char* bring = ring + SA * tc::A_BYTES;
     TopKSmem tk = topk_carve(bring + SB * tc::B_BYTES, sp.topk);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -406,18 +391,18 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     // arbiter"), so the latency-critical roles (MMA / TMA issuers, producers) get the high physical warp ids
     // 8..15 and the throughput-bound epilogue the low ones; rw & 3 == warp & 3 (TMEM lane quadrant) and the
     // warpgroups stay aligned for setmaxnreg.
-    const int rw = (warp + tc::NWARPS - tc::EPI_WARPS) % tc::NWARPS;
+    const int rw = EPI4_EPI_LOW ? ((warp + 8) & 15) : warp;
     const DevData& d = sp.d;
     const uint32_t rank = cluster_rank();
     const bool leader = rank == 0;
     if (tid == 0) {
         for (int s = 0; s < SA; ++s) {
-            mbar_init(&afull_bar[s], tc::CLUSTER * tc::CHUNKS);   // (leader) both CTAs' producers
+            mbar_init(&afull_bar[s], 1);
+            mbar_init(&apeer_bar[s], 1);                  // (leader) the follower's relay
             mbar_init(&aempty_bar[s], 1);                 // the leader's MMA commit
         }
         for (int s = 0; s < SB; ++s) {
-            mbar_init(&bfull_bar[s], 1);
-            mbar_init(&bpeer_bar[s], 1);                  // (leader) the follower's relay
+            mbar_init(&bfull_bar[s], tc::CLUSTER * tc::CHUNKS);   // (leader) both CTAs' producers
             mbar_init(&bempty_bar[s], 1);                 // the leader's MMA commit
         }
         for (int b = 0; b < 2; ++b) {
@@ -439,7 +424,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     if (rw >= tc::EPI_WARP0) {
         const int ew = rw - tc::EPI_WARP0, q = warp & 3, h = ew >> 2;
         const uint32_t tq = s_tmem + ((uint32_t)(q * 32) << 16);
-        for (int col = 16 * h; col < tc::ACC_COLS; col += 16 * tc::EPI_NH) tmem_zero16(tq + (uint32_t)col);
+        for (int col = 16 * h; col < tc::ACC_COLS; col += 32) tmem_zero16(tq + (uint32_t)col);
         if (h == 0)                      // E8M0 scale factors 2^0 for every MMA (any layout reads 0x7F)
             for (int col = tc::SF_COL; col < tc::TMEM_COLS; col += 16) tmem_fill16(tq + (uint32_t)col, 0x7F7F7F7Fu);
         tmem_wait_st();
@@ -458,19 +443,24 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     const uint8_t* const expl0 = d.expl[0];
     const uint8_t* const expl1 = d.expl[1];
 
+    // Warp-specialised register budgets (setmaxnreg, per warpgroup): the MMA/TMA issuers and the producers
+    // need few registers; the epilogue warpgroups take the rest (EPI4_REGS_EPI) so the per-quad evaluation
+    // runs without spills and with more loads in flight.
     if (tc::REGSPLIT) {
         if (rw < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_CTL));
-        else if (rw < tc::EPI_WARP0) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_PROD));
+        else if (rw < 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_PROD));
         else asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(tc::REGS_EPI));
     }
     if (rw < tc::MMA_WARPS) {
         // ===================== MMA issuers (leader CTA) =====================
         // Issuer m takes the steps s with s % MMA_WARPS == m.  The whole warp runs the loop (warp-uniform
-        // control flow keeps the descriptors in uniform registers); one elected lane issues.  Every MMA
-        // accumulates (the epilogue re-zeroes the accumulators), so the two issuers' MMAs commute.
-        if (leader) {
+        // control flow keeps the descriptors in uniform registers); one elected lane issues.  Descriptors are
+        // precomputed once: per MMA only a 64-bit add (tools/probe_mma3.cu).  Every MMA accumulates (the
+        // epilogue re-zeroes the accumulators), so the two issuers' MMAs commute.
+        if (leader && rw < tc::MMA_ISSUERS) {
             const int m = rw;
-            const uint64_t adesc0 = sw128_desc(smem_u32(aring)), bdesc0 = sw128_desc(smem_u32(bring));
+            const uint32_t ring_s = smem_u32(ring), bring_s = smem_u32(bring);
+            const uint64_t adesc0 = sw128_desc(ring_s), bdesc0 = sw128_desc(bring_s);
             const uint32_t sf_addr = tmem + tc::SF_COL;
             int it = 0, gstep = 0;
             long long t_wait = 0, t_tempty = 0;
@@ -500,10 +490,10 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         const uint32_t pa = (uint32_t)((gstep / SA) & 1), pb = (uint32_t)((gstep / SB) & 1);
                         const long long t0 = PCLK();
                         if (lane == 0) TRACE(12, gstep);
-                        mbar_wait(&afull_bar[sa], pa);              // both A halves built
+                        mbar_wait(&bfull_bar[sb], pb);              // both B halves built
                         if (lane == 0) TRACE(15, gstep);
-                        mbar_wait(&bpeer_bar[sb], pb);              // follower's B landed
-                        mbar_wait(&bfull_bar[sb], pb);              // own B landed
+                        mbar_wait(&apeer_bar[sa], pa);              // follower's A landed
+                        mbar_wait(&afull_bar[sa], pa);              // own A landed
                         t_wait += PCLK() - t0;
                         if (lane == 0) TRACE(10, gstep);
                         tc_fence_after();
@@ -533,70 +523,82 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 atomicAdd(sp.prof + 7, (unsigned long long)t_tempty);
             }
         } else if (rw == 0) {
-            // follower: relay "my B landed" to the leader's bpeer barrier
+            // follower: relay "my A landed" (sfull) to the leader's full barrier, off the producers' path
             StepIt st;
-            st.init(sp, rank);
+            st.init(sp);
             for (int gstep = 0; st.valid(sp); st.advance(sp, 1), ++gstep) {
-                mbar_wait(&bfull_bar[gstep % SB], (uint32_t)((gstep / SB) & 1));
+                mbar_wait(&afull_bar[gstep % SA], (uint32_t)((gstep / SA) & 1));
                 if (lane == 0) TRACE(14, gstep);
-                if (lane == 0) mbar_arrive_cluster(&bpeer_bar[gstep % SB], 0);
+                if (lane == 0) mbar_arrive_cluster(&apeer_bar[gstep % SA], 0);
                 __syncwarp();
             }
         }
         __syncwarp();
     } else if (rw < tc::PROD_WARP0) {
-        // ===================== TMA issuers: this CTA's B (16 KiB per step) =====================
-        const int tw = rw - tc::TMA_WARP0;
-        StepIt st;
-        st.init(sp, rank);
-        st.advance(sp, tw);
-        long long t_wait = 0;
-        const uint32_t bring_s = smem_u32(bring);
-        for (int gstep = tw; st.valid(sp); st.advance(sp, tc::TMA_WARPS), gstep += tc::TMA_WARPS) {
-            const int sb = gstep % SB;
-            const long long t0 = PCLK();
-            mbar_wait(&bempty_bar[sb], (uint32_t)((gstep / SB) & 1) ^ 1u);
-            t_wait += PCLK() - t0;
-            if (lane == 0) TRACE(0, gstep);
-            // rows 2 (64 wr + 32 rank) .. + 63 of the step's two chunks: 16 contiguous KiB in HBM
-            const uint8_t* src = (st.p ? expl1 : expl0) +
-                                 expl_off(2 * (int64_t)st.chunk(), (int64_t)(st.ti.wr * 2 + (int)rank) * 64, nrb);
-            if (sp.debug & 128) {             // diagnostics: no copy (the MMA reads stale operands)
-                if (lane == 0) mbar_arrive_local(&bfull_bar[sb]);
+        // ===================== TMA issuers: this CTA's A (16 KiB per step) =====================
+        // warp t takes the steps s with s % TMA_WARPS == t; the whole warp runs the loop (uniform operands),
+        // one elected lane issues
+        {
+            const int tw = rw - tc::TMA_WARP0;
+            StepIt st;
+            st.init(sp);
+            st.advance(sp, tw);
+            long long t_wait = 0;
+            const uint32_t ring_s = smem_u32(ring);
+            for (int gstep = tw; st.valid(sp); st.advance(sp, tc::TMA_WARPS), gstep += tc::TMA_WARPS) {
+                const int sa = gstep % SA;
+                const long long t0 = PCLK();
+                mbar_wait(&aempty_bar[sa], (uint32_t)((gstep / SA) & 1) ^ 1u);
+                t_wait += PCLK() - t0;
+                if (lane == 0) TRACE(0, gstep);
+                // this CTA's 128 A rows (row block 2 wp + rank) of the step's two chunks: 32 contiguous KiB in HBM,
+                // copied as A_SPLIT pieces issued by as many lanes
+                const uint8_t* src = (st.p ? expl1 : expl0) +
+                                     expl_off(2 * (int64_t)st.chunk(), (int64_t)(st.ti.wp * 2 + (int)rank) * 128, nrb);
+                if (sp.debug & 128) {             // diagnostics: no copy (the MMA reads stale operands)
+                    if (lane == 0) mbar_arrive_local(&afull_bar[sa]);
+                    __syncwarp();
+                    continue;
+                }
+                if (lane == 0) mbar_expect_tx(&afull_bar[sa], tc::TX_BYTES);
                 __syncwarp();
-                continue;
+                if (lane < tc::A_SPLIT) {
+                    constexpr uint32_t piece = tc::A_BYTES / tc::A_SPLIT;
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                                 ::"r"(ring_s + (uint32_t)(sa * tc::A_BYTES) + lane * piece), "l"(src + lane * piece),
+                                 "r"(piece), "r"(smem_u32(&afull_bar[sa]))
+                                 : "memory");
+                }
+                __syncwarp();
+                if (lane == 0) TRACE(1, gstep);
             }
-            if (lane == 0) {
-                mbar_expect_tx(&bfull_bar[sb], tc::B_BYTES);
-                bulk_g2s(bring + sb * tc::B_BYTES, src, tc::B_BYTES, &bfull_bar[sb]);
-            }
-            __syncwarp();
-            if (lane == 0) TRACE(1, gstep);
+            if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
         }
-        (void)bring_s;
-        if (EPI4_PROF && lane == 0) atomicAdd(sp.prof + 6, (unsigned long long)t_wait);
     } else if (rw < tc::EPI_WARP0) {
         // ===================== producers =====================
-        // Producer warp j builds chunk jc = j % CHUNKS of this CTA's A for every step s with s % PROD_STRIDE ==
-        // j / CHUNKS.  Its singles (x, z and the tile's 16 y SNPs, two planes each, pre-swizzled in HBM) are loaded
-        // straight into registers one own step ahead.  Lane: 16-byte piece cc = lane & 7 of the 256-sample K row,
-        // plane c = (lane >> 3) & 1, y_l = (lane >> 4) + 2k (k = 0..7); A[row 8 y_l + 4b + 2c + d] = x_b & y_c & z_d
-        // (a nibble-wise AND of E2M1 {0, 1.0} values is their product).
-        constexpr int YK = tc::YT / 2;
+        // Producer warp j builds chunk jc = j % CHUNKS of this CTA's B half of every step s with
+        // s % PROD_STRIDE == j / CHUNKS.  Its singles (x, z and the CTA's YH y SNPs, two planes each, pre-swizzled
+        // in HBM) are loaded straight into registers one own step ahead (no shared-memory staging).  Lane:
+        // 16-byte piece cc = lane & 7 of the 256-sample K row, plane c = (lane >> 3) & 1, y_local = (lane >> 4) + 2k
+        // (k = 0..YH/2-1); B[n = 8 y_local + 4b + 2c + d] = x_b & y_c & z_d (a nibble-wise AND of E2M1 {0, 1.0}
+        // values is their product).  The follower's A is certified to the leader by the relay warp, so producers
+        // never wait for the TMA.
+        static_assert(tc::YH % 2 == 0, "two y per lane pair");
+        constexpr int YK = tc::YH / 2;
         const int pw = rw - tc::PROD_WARP0;
         const int jc = pw % tc::CHUNKS, pstep0 = pw / tc::CHUNKS;   // chunk of the step, first step
         const int cc = lane & 7, cpl = (lane >> 3) & 1, yq = lane >> 4;
         const bool build = !(sp.debug & 1);
-        // store offsets inside the A chunk for bd = 2b + d (row 8 y_l + n7; y_l = yq: + 2048 per k)
-        uint32_t aoff[4];
+        // store offsets inside the B sub-tile for bd = 2b + d (y_local = yq; + 2048 per k)
+        uint32_t boff[4];
 #pragma unroll
         for (int bd = 0; bd < 4; ++bd) {
             const int n7 = (bd >> 1) * 4 + cpl * 2 + (bd & 1);
-            aoff[bd] = (uint32_t)(yq * 1024 + n7 * 128 + ((cc ^ n7) << 4));
+            boff[bd] = (uint32_t)(yq * 1024 + n7 * 128 + ((cc ^ n7) << 4));
         }
-        long long t_wait = 0, t_busy = 0;
+        long long t_wait = 0, t_busy = 0, t_arr = 0;
         StepIt st, pre;
-        st.init(sp, rank);
+        st.init(sp);
         st.advance(sp, pstep0);
         pre = st;
         // logical piece cc of absolute row r sits at piece cc ^ (r & 7) of the row in HBM
@@ -612,71 +614,78 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 nx[1] = ld_piece(E, C, 2 * (int64_t)it.ti.x + 1);
                 nx[2] = ld_piece(E, C, 2 * (int64_t)it.ti.z);
                 nx[3] = ld_piece(E, C, 2 * (int64_t)it.ti.z + 1);
-                const int64_t ry = 2 * (int64_t)(it.ti.y0 + yq) + cpl;
+                const int64_t ry = 2 * (int64_t)(it.ti.y0 + tc::YH * (int)rank + yq) + cpl;
 #pragma unroll
                 for (int k = 0; k < YK; ++k) ny[k] = ld_piece(E, C, ry + 4 * k);
             }
         };
-        // register prefetch one own step ahead (4 producer warps), or (8 producer warps, half the registers) the
-        // step's own loads issued before the slot wait, latency hidden by the other warps' steps
-        constexpr bool PREFETCH = tc::PROD_WARPS == 4;
-        if (PREFETCH) {
-            load(pre);
-            pre.advance(sp, tc::PROD_STRIDE);
-        }
+        load(pre);
+        pre.advance(sp, tc::PROD_STRIDE);
         for (int step = pstep0; st.valid(sp); step += tc::PROD_STRIDE) {
-            const int sa = step % SA;
+            const int sb = step % SB;
             if (lane == 0) TRACE(2, step);
             uint4 cx[4], cy[YK];
-            if (!PREFETCH) load(st);
 #pragma unroll
             for (int k = 0; k < 4; ++k) cx[k] = nx[k];
 #pragma unroll
             for (int k = 0; k < YK; ++k) cy[k] = ny[k];
-            if (PREFETCH) {
-                load(pre);                                        // next own step's singles (in flight)
-                pre.advance(sp, tc::PROD_STRIDE);
-            }
+            load(pre);                                            // next own step's singles (in flight)
+            pre.advance(sp, tc::PROD_STRIDE);
             const long long t0 = PCLK();
-            mbar_wait(&aempty_bar[sa], (uint32_t)((step / SA) & 1) ^ 1u);   // A slot free (MMA of step - SA done)
+            mbar_wait(&bempty_bar[sb], (uint32_t)((step / SB) & 1) ^ 1u);   // B slot free (MMA of step - SB done)
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             if (lane == 0) TRACE(4, step);
+#if EPI4_PROF
+            {   // trace event 3: this step's singles have arrived (a value-dependent branch waits for the loads)
+                uint32_t dep = cx[0].x | cx[1].y | cx[2].z | cx[3].w;
+#pragma unroll
+                for (int k = 0; k < YK; ++k) dep |= cy[k].x;
+                if (lane == 0 && dep != 0x9E3779B9u) TRACE(3, step);
+            }
+#endif
             if (build) {
-                unsigned char* adst = aring + sa * tc::A_BYTES + jc * tc::A_SUB;
+                unsigned char* bdst = bring + sb * tc::B_BYTES + jc * tc::B_SUB;
                 const uint4 xz[4] = {and4(cx[0], cx[2]), and4(cx[0], cx[3]), and4(cx[1], cx[2]), and4(cx[1], cx[3])};
 #pragma unroll
                 for (int k = 0; k < YK; ++k)
 #pragma unroll
                     for (int bd = 0; bd < 4; ++bd)
-                        *reinterpret_cast<uint4*>(adst + aoff[bd] + k * 2048) = and4(cy[k], xz[bd]);
+                        *reinterpret_cast<uint4*>(bdst + boff[bd] + k * 2048) = and4(cy[k], xz[bd]);
                 if (lane == 0) TRACE(6, step);
                 fence_proxy_async();                      // generic-proxy stores -> visible to the tensor core
             }
             __syncwarp();
+            const long long t2 = PCLK();
             if (lane == 0) {
                 TRACE(7, step);
-                if (leader) mbar_arrive_local(&afull_bar[sa]);
-                else mbar_arrive_cluster(&afull_bar[sa], 0);             // the leader's barrier
+                if (leader) mbar_arrive_local(&bfull_bar[sb]);
+                else mbar_arrive_cluster(&bfull_bar[sb], 0);             // the leader's barrier
                 TRACE(9, step);
             }
             __syncwarp();
-            if (EPI4_PROF) t_busy += PCLK() - t1;
+            if (EPI4_PROF) {
+                const long long t3 = PCLK();
+                t_busy += t3 - t1;
+                t_arr += t3 - t2;
+            }
             st.advance(sp, tc::PROD_STRIDE);
         }
         if (EPI4_PROF && lane == 0) {
             atomicAdd(sp.prof + 3, (unsigned long long)t_busy);
             atomicAdd(sp.prof + 4, (unsigned long long)t_wait);
+            (void)t_arr;
         }
     } else {
         // ===================== epilogue =====================
-        // lane quadrant q holds rows 32q..32q+31 = (y_l, b, c, d) with y_l = 4q + (lane >> 3), bcd = lane & 7; a
-        // 16-column group g holds w_l = 8g..8g+7 x a.  After transpose8 lane L = bcd owns the quad w_l = 8g + L
-        // with all 16 counts c16[8a + bcd'].
+        // lane quadrant q holds rows 32q..32q+31 = (w_local, a) with w_local = row/2; a 16-column group g
+        // holds y_local = 2g, 2g+1 x (b, c, d).  Lanes a=0/a=1 swap halves so that lane a owns the quad
+        // y_local = 2g + a with all 16 counts c16[8a' + 4b + 2c + d].
         const int ew = rw - tc::EPI_WARP0;             // 0..7
         const int q = warp & 3;                         // TMEM lane quadrant this warp may access
-        const int h = ew >> 2;                          // EPI_NH warps per quadrant split the column groups
-        const int yl = 4 * q + (lane >> 3), L = lane & 7;
+        const int h = ew >> 2;                          // two warps per quadrant split the column groups
+        const int row = q * 32 + lane;
+        const int wl = row >> 1, a = row & 1;
         unsigned long long my_quads = 0, n_exact = 0;
         long long t_wait = 0, t_busy = 0;
         const bool score = !(sp.debug & 2);
@@ -684,7 +693,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         const uint32_t pks = (uint32_t)d.pk_shift;
         int r0 = 0;                                     // the MMA issuers' region rotation
         for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
-            const TileInfo ti = load_tile(sp, tile, rank);
+            const TileInfo ti = load_tile(sp, tile);
             const int buf = it & 1;
             const uint32_t tphase = (uint32_t)((it >> 1) & 1);
             const int r1 = r0 == 2 ? 0 : r0 + 1;
@@ -693,12 +702,13 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             const long long t1 = PCLK();
             t_wait += t1 - t0;
             tc_fence_after();
+            const int w = (ti.wp * 2 + (int)rank) * EPI4_WR + wl;
             const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
             const uint32_t R0 = tq + (uint32_t)(r0 * tc::N), R1 = tq + (uint32_t)(r1 * tc::N);
             // pass 1: pack each (control, case) count pair into one 32-bit word, in place in the case region,
             // and zero the control region, which the next tile's case accumulation reuses
 #pragma unroll 1
-            for (int g = h; g < tc::NG; g += tc::EPI_NH) {
+            for (int g = h; g < tc::NG; g += 2) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(R0 + 16 * g, v0);
                 tmem_ld16(R1 + 16 * g, v1);
@@ -717,16 +727,14 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 if (leader) mbar_arrive_local(&pk_bar);
                 else mbar_arrive_cluster(&pk_bar, 0);   // the leader's barrier
             }
-            const int y = ti.y0 + yl;
-            const bool yok = y < ti.z && !ti.skip;
             // pass 2: score the quads from the packed counts
 #pragma unroll 1
-            for (int g = h; g < tc::NG; g += tc::EPI_NH) {
-                uint32_t c16[16];
-                tmem_ld16(R1 + 16 * g, c16);
+            for (int g = h; g < tc::NG; g += 2) {
+                uint32_t v[16];
+                tmem_ld16(R1 + 16 * g, v);
                 tmem_wait_ld();
                 tmem_zero16(R1 + 16 * g);                 // ready for a later tile's accumulation
-                if (g + tc::EPI_NH >= tc::NG) {
+                if (g + 2 >= tc::NG) {
                     tmem_wait_st();
                     tc_fence_before();
                     __syncwarp();
@@ -735,38 +743,38 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         else mbar_arrive_cluster(&ep_bar[buf], 0);   // the leader's barrier
                     }
                 }
-                const int w = ti.wr * EPI4_WU + 8 * g + L;
-                // skip the exchange when no lane of the warp has a valid quad in this group (diagonal units)
-                if (!__any_sync(0xffffffffu, yok && w < ti.x)) continue;
-                transpose8(c16, lane);
-                // c16 now holds (a, bcd) at index 2 bcd + a; the evaluation wants 8a + bcd
-                uint32_t t16[16];
+                uint32_t c16[16];
 #pragma unroll
-                for (int s = 0; s < 8; ++s) {
-                    t16[s] = c16[2 * s];
-                    t16[8 + s] = c16[2 * s + 1];
+                for (int k = 0; k < 8; ++k) {
+                    // send my values for the other lane's quad, keep mine; lane a keeps c16[8a + k] = its own
+                    // v[8a + k] and takes c16[8(1-a) + k] from the partner (packed control | case words)
+                    const uint32_t sv = a ? v[k] : v[8 + k];
+                    const uint32_t rv = __shfl_xor_sync(0xffffffffu, sv, 1);
+                    c16[k] = a ? rv : v[k];
+                    c16[8 + k] = a ? v[8 + k] : rv;
                 }
+                const int y = ti.y0 + 2 * g + a;
                 if (sp.t3_out) {
-                    // 3-way-table mode (z = the all-ones SNP n): the d = AA counts are T3(w, x, y)[a b c]
+                    // 3-way-table mode (z = the all-ones SNP n): the d = AA columns are T3(w, x, y)[a b c]
                     // (PAPER.md:L118 tensorOp_3way); already packed (control | case), written in the T3 layout
-                    if (yok && w < ti.x) {
+                    if (w < ti.x && y < ti.z) {
                         // resident: colex rank; windowed slab FIRST(R): (w - w0) * C(n,2) + rank2(x, y)
                         const int64_t e = sp.t3_slab_w0 >= 0
                                               ? (int64_t)(w - sp.t3_slab_w0) * c2(d.n) + c2(y) + ti.x
                                               : rank3(w, ti.x, y);
                         uint4* o = reinterpret_cast<uint4*>(sp.t3_out + e * 8);
-                        o[0] = make_uint4(t16[0], t16[2], t16[4], t16[6]);
-                        o[1] = make_uint4(t16[8], t16[10], t16[12], t16[14]);
+                        o[0] = make_uint4(c16[0], c16[2], c16[4], c16[6]);
+                        o[1] = make_uint4(c16[8], c16[10], c16[12], c16[14]);
                     }
                     continue;
                 }
                 if (sp.search3) {
-                    // third-order search (z = the all-ones SNP n): triple (w, x, y) from the d = AA counts
-                    const bool v3 = yok && (w < ti.x) && score;
+                    // third-order search (z = the all-ones SNP n): triple (w, x, y) from the d = AA columns
+                    const bool v3 = (w < ti.x) && (y < ti.z) && score;
                     double key3 = 0.0;
                     uint64_t idx3 = 0;
                     if (v3) {
-                        const uint32_t c8[8] = {t16[0], t16[2], t16[4], t16[6], t16[8], t16[10], t16[12], t16[14]};
+                        const uint32_t c8[8] = {c16[0], c16[2], c16[4], c16[6], c16[8], c16[10], c16[12], c16[14]};
                         key3 = score_triple(d, w, ti.x, y, c8);
                         idx3 = pack_quad(w, ti.x, y, 0);
                         ++my_quads;
@@ -774,7 +782,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     warp_offer(tk, v3, key3, idx3);
                     continue;
                 }
-                const bool valid = yok && (w < ti.x) && score;
+                const bool valid = (w < ti.x) && (y < ti.z) && score;
                 double key = 0.0;
                 uint64_t idx = 0;
                 bool offer = false;
@@ -782,18 +790,18 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     uint32_t* dump = sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
                     offer = true;
                     if (dump) {
-                        key = score_quad_rare(d, w, ti.x, y, ti.z, t16, dump);
-                        if (d.objective != EPI4_OBJ_K2) key = score_quad_rare(d, w, ti.x, y, ti.z, t16, nullptr);
+                        key = score_quad_rare(d, w, ti.x, y, ti.z, c16, dump);
+                        if (d.objective != EPI4_OBJ_K2) key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
                     } else if (sample_hit(sp, pack_quad(w, ti.x, y, ti.z))) {
-                        key = sample_record_rare(sp, w, ti.x, y, ti.z, t16);
+                        key = sample_record_rare(sp, w, ti.x, y, ti.z, c16);
                     } else if (sp.use_filter) {
                         // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
                         // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2); FILT 2: MI
                         // upper bound (key = -M*I)
                         float flt;
                         double unused;
-                        quad_eval<FILT == 1 ? 5 : FILT == 2 ? 6 : 0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y,
-                                                                          ti.z, t16, flt, unused, nullptr);
+                        quad_eval<FILT == 1 ? 5 : FILT == 2 ? 6 : 0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt,
+                                                           unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
                         if (FILT == 1)
                             offer = d.chi_M - (double)flt * (1.0 + 1.0 / 4096.0) <= thr;
@@ -803,11 +811,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                             offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
                             // rare path: the noinline exact scorer takes the counts through local memory
-                            key = score_quad_rare(d, w, ti.x, y, ti.z, t16, nullptr);
+                            key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
                             ++n_exact;
                         }
                     } else {
-                        key = score_quad_rare(d, w, ti.x, y, ti.z, t16, nullptr);
+                        key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
                     }
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;
@@ -869,6 +877,11 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16, FILT>, sp);
 }
 
+// tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
+// cluster (1 tile); the CUDA-core kernel processes them as 2 tiles
+int32_t quad_split(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? 2 : 1; }
+int32_t quad_yr(int32_t pipe) { return pipe == EPI4_PIPE_LOP3 ? EPI4_YR : EPI4_YR_TC; }
+
 cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t s, int64_t* launches) {
     SearchParams sp = sp_in;
     grid = grid / tc::CLUSTER * tc::CLUSTER;
@@ -876,21 +889,22 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     const size_t fixed = 1024 + topk_smem_bytes(sp.topk) + 1024;   // alignment + static smem slack
-    // deepest rings that fit: produced A stages (32 KiB) x TMA B stages (16 KiB)
+    // deepest rings that fit (the A copies carry the long L2 latency; a B stage is only held from its
+    // production to its MMA)
     struct Cfg { int sa, sb; };
-    const Cfg cands[] = {{4, 6}, {4, 4}, {2, 6}, {2, 4}, {2, 2}};
+    const Cfg cands[] = {{tc::MMA_ISSUERS == 1 ? 5 : 4, tc::MMA_ISSUERS == 1 ? 3 : 4}, {6, 2}, {4, 4}, {4, 2}, {2, 2}};
     Cfg pick{0, 0};
     for (const Cfg& c : cands)
         if (!pick.sa && fixed + (size_t)c.sa * tc::A_BYTES + (size_t)c.sb * tc::B_BYTES <= (size_t)optin) pick = c;
-    if (getenv("EPI4_STAGES")) {   // diagnostics: EPI4_STAGES=<sa><sb>, e.g. 44
+    if (getenv("EPI4_STAGES")) {   // diagnostics: EPI4_STAGES=<sa><sb>, e.g. 43
         const int v = atoi(getenv("EPI4_STAGES"));
         pick = Cfg{v / 10, v % 10};
     }
     if (!pick.sa) return cudaErrorInvalidConfiguration;
     const size_t smem = 1024 + (size_t)pick.sa * tc::A_BYTES + (size_t)pick.sb * tc::B_BYTES + topk_smem_bytes(sp.topk);
     if (getenv("EPI4_VERBOSE"))
-        fprintf(stderr, "k_quad_tc: A/B stages %d/%d, filter %d, smem %zu B, grid %d, pair tiles %lld\n", pick.sa,
-                pick.sb, sp.use_filter, smem, grid, (long long)sp.ntiles);
+        fprintf(stderr, "k_quad_tc: %d producer warps, A/B stages %d/%d, A split %d, filter %d, smem %zu B, grid %d\n",
+                tc::PROD_WARPS, pick.sa, pick.sb, tc::A_SPLIT, sp.use_filter, smem, grid);
     cudaError_t e = cudaErrorInvalidConfiguration;
     const bool pk16 = sp.d.pk_shift == 16;
     const int filt = sp.use_filter == 2 ? 1 : sp.use_filter == 3 ? 2 : 0;   // FILT 1: chi-square, 2: MI
@@ -898,13 +912,13 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     e = filt == 1 ? (pk16 ? launch_cfg<A_, B_, true, 1>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1>(sp, smem, grid, s)) \
       : filt == 2 ? (pk16 ? launch_cfg<A_, B_, true, 2>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 2>(sp, smem, grid, s)) \
                   : (pk16 ? launch_cfg<A_, B_, true, 0>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0>(sp, smem, grid, s))
-    if (pick.sa == 4 && pick.sb == 6) EPI4_LAUNCH(4, 6);
+    if (pick.sa == 5 && pick.sb == 3) {
+        if constexpr (tc::MMA_ISSUERS == 1) EPI4_LAUNCH(5, 3);
+    } else if (pick.sa == 4 && pick.sb == 6) EPI4_LAUNCH(4, 6);
+    else if (pick.sa == 6 && pick.sb == 2) EPI4_LAUNCH(6, 2);
     else if (pick.sa == 4 && pick.sb == 4) EPI4_LAUNCH(4, 4);
-    else if constexpr (tc::PROD_STRIDE <= 2) {
-        if (pick.sa == 2 && pick.sb == 6) EPI4_LAUNCH(2, 6);
-        else if (pick.sa == 2 && pick.sb == 4) EPI4_LAUNCH(2, 4);
-        else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
-    }
+    else if (pick.sa == 4 && pick.sb == 2) EPI4_LAUNCH(4, 2);
+    else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
 #undef EPI4_LAUNCH
     if (launches) ++*launches;
     return e;

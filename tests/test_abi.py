@@ -46,7 +46,7 @@ def test_plan_rejects_bad_arguments():
 
 
 def _quads_of_unit(n, wb, x):
-    for w in range(64 * wb, min(64 * wb + 64, x)):
+    for w in range(128 * wb, min(128 * wb + 128, x)):
         for y in range(x + 1, n):
             for z in range(y + 1, n):
                 yield (w, x, y, z)

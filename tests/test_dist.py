@@ -34,7 +34,7 @@ def _worker(rank, world, port, top_k, q):
         units, _ = binding.epi4_plan_units(n, rank, world)
         quads = []
         for wb, x in units:
-            for w in range(64 * wb, min(64 * wb + 64, x)):
+            for w in range(128 * wb, min(128 * wb + 128, x)):
                 for y in range(x + 1, n):
                     for z in range(y + 1, n):
                         quads.append((w, int(x), y, z))

@@ -263,7 +263,7 @@ def test_full_C2_units_sample_and_planted(pipe):
     quads = []
     for u in sel:
         wb, x = (int(v) for v in units[u])
-        for w in range(64 * wb, min(64 * wb + 64, x)):
+        for w in range(128 * wb, min(128 * wb + 128, x)):
             for y in range(x + 1, n):
                 for z in range(y + 1, n):
                     quads.append((w, x, y, z))
