@@ -148,5 +148,16 @@ int main() {
     run<3, 0, 65536>(src, bytes / 65536, cyc, nsm);
     run<4, 1, 32768>(src, bytes / 32768, cyc, nsm);
     run<4, 2, 32768>(src, bytes / 32768, cyc, nsm);
+    run<6, 1, 32768>(src, bytes / 32768, cyc, nsm);
+    run<6, 2, 32768>(src, bytes / 32768, cyc, nsm);
+    // a 64 MB source (less reuse across SMs)
+    uint8_t* big;
+    const size_t bbytes = (size_t)64 << 20;
+    cudaMalloc(&big, bbytes);
+    cudaMemset(big, 1, bbytes);
+    run<4, 0, 32768>(big, bbytes / 32768, cyc, nsm);
+    run<6, 0, 32768>(big, bbytes / 32768, cyc, nsm);
+    run<4, 1, 32768>(big, bbytes / 32768, cyc, nsm);
+    run<4, 2, 32768>(big, bbytes / 32768, cyc, nsm);
     return 0;
 }
