@@ -2,7 +2,7 @@
 """Benchmark of the exhaustive fourth-order K2 search (BASELINE.json metric: tera quads/s scaled to
 sample size, C(N,4)*M / t).
 
-  python bench.py --gpus N --steps K --warmup W [--config C2] [--pipe tc] [--impl ours|reference]
+  python bench.py --gpus N --steps K --warmup W [--config C5] [--also C2] [--pipe tc] [--impl ours|reference]
 
 A step = one pass of the whole hot path over the config's synthetic dataset:
 pack the byte genotypes into bit planes (a1), T1/T2/T3 (a2, a4), the 4-way contraction with the fused
@@ -12,6 +12,11 @@ pinned HOST buffers (H2D of the genotypes and D2H of the result inside the timed
 For N > 1 (torchrun) the quad space of the same dataset is split across ranks by the static LPT plan:
 total work is fixed -> "scaling": "strong" (the paper's Fig. 3 experiment).
 `--impl reference` times the CPU oracle (the only reference this tier has) on a bounded sample.
+
+The default workload is C5 (N=1024, M=100003, 30/70): the largest BASELINE.json config one B200 runs within the
+driver's step protocol (C3 takes ~165 s per step, C4 is 8-GPU work).  The same run also times C2 (the config
+BASELINE.json lists as "single B200") with the same steps / warm-up and reports it under "also" in the same
+JSON line (--also none to skip).  `--gpus N` without torchrun relaunches itself under torch.distributed.run.
 """
 from __future__ import annotations
 
@@ -101,6 +106,16 @@ class ClockSampler:
                 "samples": len(self.samples)}
 
 
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
 def cpu_oracle_sample(d, target_s=12.0, max_w=None):
     """Time the oracle (as it stands) on the first W SNPs at full M; W picked so it runs ~target_s."""
     import oracle
@@ -116,27 +131,21 @@ def cpu_oracle_sample(d, target_s=12.0, max_w=None):
     t0 = time.perf_counter()
     oracle.search(d.geno, d.phen, top_k=1, n_snps=w)
     t = time.perf_counter() - t0
-    return {"value": comb4(w) * d.n_samples / t / 1e12, "unit": UNIT, "cores": cores, "kind": "oracle",
+    rate = comb4(w) * d.n_samples / t
+    full_h = comb4(d.n_snps) * d.n_samples / rate / 3600.0
+    return {"value": rate / 1e12, "unit": UNIT, "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
             "sample": f"exhaustive search over the first {w} SNPs ({comb4(w)} quads) x all M={d.n_samples} "
-                      f"samples of {d.name}; {t:.2f} s on {cores} host threads"}
+                      f"samples of {d.name}; {t:.2f} s on {cores} host threads",
+            "extrapolated_full_run_hours": full_h}
 
 
 def flush_l2(torch, buf):
     buf.zero_()   # 512 MiB write > 126 MB L2, outside the timed region
 
 
-def run_ours(args):
-    import torch
-    import torch.distributed as dist
-    import paper_conf_icpp_nobreiss22_b200 as epi
-
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    d = datagen.make_config(args.config)
+def measure(cfg, args, world, rank, local, torch, dist, epi):
+    """W warm-up steps and K timed steps of the whole hot path on config `cfg`; returns the JSON fields."""
+    d = datagen.make_config(cfg)
     n, m = d.n_snps, d.n_samples
     stream = torch.cuda.Stream()
     # N > 1: every rank builds the 3-way table on its tensor cores (~3 ms at C2, tiny next to the search);
@@ -230,7 +239,7 @@ def run_ours(args):
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(f"{args.config}:{args.pipe}")
+            traffic = json.load(open(tf)).get(f"{cfg}:{args.pipe}")
         except Exception:
             traffic = None
     out = {
@@ -238,9 +247,11 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": t_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "e2m1 (mxf4, f32 accum)" if args.pipe == "tc" else "u32",
         "data": "synthetic (seeded HWE genotypes + planted 4-way interaction, SURVEY.md §8(d))",
-        "config": {"workload": f"{args.config}: N={n} SNPs, M={m} samples ({d.n_controls} controls / "
+        "config": {"workload": f"{cfg}: N={n} SNPs, M={m} samples ({d.n_controls} controls / "
                                f"{d.n_cases} cases), exhaustive C(N,4)={comb4(n)} quads, top_k={top_k}",
-                   "pipe": args.pipe, "objective": args.objective, "parallelism": f"static LPT over (w-block, x) units x {world}" + (", T3 sharded + NCCL all_gather" if shard else ""),
+                   "pipe": args.pipe, "objective": args.objective,
+                   "parallelism": f"static LPT over (w-block, x) units x {world} ranks (NCCL world {world})" +
+                                  (", T3 sharded + NCCL all_gather" if shard else ""),
                    "l2": "flushed (512 MiB write) before every timed step"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": int(n * m + m),
                 "d2h_bytes_per_step": int(top_k * 16 + 4)},
@@ -271,11 +282,50 @@ def run_ours(args):
                                                 f"{mhz:.0f} MHz median SM clock of the timed region")
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_oracle_sample(d)
+    eng.close()
+    del geno_d, phen_d, flush
+    torch.cuda.empty_cache()
+    return out
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_nobreiss22_b200 as epi
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+        sys.exit(2)
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        assert dist.get_world_size() == world
+    out = measure(args.config, args, world, rank, local, torch, dist, epi)
+    if args.also not in ("none", "", args.config):
+        sec = measure(args.also, args, world, rank, local, torch, dist, epi)
+        out["also"] = {k: sec[k] for k in ("config", "value", "unit", "ms_per_step", "e2e", "roofline", "step_ms",
+                                           "quad_step_ms", "useful_over_executed", "clocks", "best",
+                                           "breakdown_ms", "gpu_launches") if k in sec}
+        if "cpu_baseline" in sec:
+            out["also"]["cpu_baseline"] = sec["cpu_baseline"]
     if rank == 0:
         print(json.dumps(out), flush=True)
-    eng.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def relaunch(args):
+    """`--gpus N` without torchrun: run N ranks under torch.distributed.run on this node (127.0.0.1)."""
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
 
 
 def run_reference(args):
@@ -305,7 +355,9 @@ def run_reference(args):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": f"{args.config}: N={d.n_snps}, M={d.n_samples}; CPU oracle on a bounded sample"},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+                         "cpu_model": cpu_model(),
+                         "extrapolated_full_run_hours": comb4(d.n_snps) * d.n_samples / (value * 1e12) / 3600.0},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -316,7 +368,9 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2", choices=list(datagen.CONFIGS))
+    ap.add_argument("--config", default="C5", choices=list(datagen.CONFIGS))
+    ap.add_argument("--also", default="C2", help="second config timed in the same run, reported under 'also' "
+                    "(none to skip)")
     ap.add_argument("--pipe", default="tc", choices=["tc", "lop3"])
     ap.add_argument("--top-k", type=int, default=16)
     ap.add_argument("--objective", default="k2", choices=["k2", "mi", "chi2"],
@@ -327,6 +381,8 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch(args)
     (run_reference if args.impl == "reference" else run_ours)(args)
 
 

@@ -181,6 +181,12 @@ int epi4_get_sample(epi4_ctx* ctx, uint64_t* quads_out, double* keys_out, uint32
 int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world);
 int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* wb_x_out /* 2 x count */,
                     double* cost_out /* count, may be NULL */);
+/* The same with opts.flags: with EPI4_FLAG_T3_WINDOWED the plan a windowed-T3 context uses (whole slab groups
+ * (128-SNP range of w, 128-SNP range of x) dealt longest first, groups above 1/(4 world) of the work split by x),
+ * so that each rank rebuilds only its own groups' slabs. */
+int64_t epi4_plan_count_ex(int32_t n_snps, int32_t rank, int32_t world, int32_t flags);
+int epi4_plan_units_ex(int32_t n_snps, int32_t rank, int32_t world, int32_t flags, int32_t* wb_x_out,
+                       double* cost_out);
 
 /* ---- measurement ---------------------------------------------------------------------------- */
 typedef struct {

@@ -75,6 +75,8 @@ def _load():
         "epi4_t3_ready": (ctypes.c_int, [P]),
         "epi4_plan_count": (I64, [I32, I32, I32]),
         "epi4_plan_units": (ctypes.c_int, [I32, I32, I32, P, P]),
+        "epi4_plan_count_ex": (I64, [I32, I32, I32, I32]),
+        "epi4_plan_units_ex": (ctypes.c_int, [I32, I32, I32, I32, P, P]),
         "epi4_get_stats": (ctypes.c_int, [P, ctypes.POINTER(epi4_stats)]),
         "epi4_last_error": (ctypes.c_char_p, []),
         "epi4_version": (ctypes.c_char_p, []),
@@ -261,6 +263,14 @@ def epi4_plan_units(n_snps: int, rank: int = 0, world: int = 1):
     u = np.zeros((max(cnt, 1), 2), dtype=np.int32)
     c = np.zeros(max(cnt, 1), dtype=np.float64)
     _check(_lib.epi4_plan_units(int(n_snps), int(rank), int(world), _ptr(u), _ptr(c)))
+    return u[:cnt], c[:cnt]
+
+
+def epi4_plan_units_ex(n_snps: int, rank: int = 0, world: int = 1, flags: int = 0):
+    cnt = _check(int(_lib.epi4_plan_count_ex(int(n_snps), int(rank), int(world), int(flags))))
+    u = np.zeros((max(cnt, 1), 2), dtype=np.int32)
+    c = np.zeros(max(cnt, 1), dtype=np.float64)
+    _check(_lib.epi4_plan_units_ex(int(n_snps), int(rank), int(world), int(flags), _ptr(u), _ptr(c)))
     return u[:cnt], c[:cnt]
 
 

@@ -59,6 +59,22 @@ cudaError_t grow(T*& p, size_t& cap, size_t bytes) {
 }
 }  // namespace
 
+// The work plan of a search, cached across searches of the same shape: a bench step re-plans nothing and copies
+// no plan data to the device.  This rank's units [ub, ue) of the static LPT plan, grouped by slab (R, X) when the
+// 3-way table is windowed, with their group-relative inclusive prefix of tiles; the tile table of a one-group,
+// one-chunk plan stays on the device.
+struct SearchPlan {
+    struct Group { int64_t b, e; int32_t wr, xr; };
+    bool valid = false;
+    int32_t n = 0, rank = 0, world = 0, pipe = -1;
+    int64_t ub = 0, ue = 0;
+    bool windowed = false;
+    std::vector<Unit> units;
+    std::vector<int64_t> prefix;        // group-relative inclusive prefix of tiles per unit
+    std::vector<Group> groups;
+    bool table_cached = false;
+};
+
 struct epi4_ctx {
     int device = 0;
     epi4_opts opts{};
@@ -84,12 +100,19 @@ struct epi4_ctx {
     size_t cap_planes[2] = {0, 0}, cap_T1 = 0, cap_T2 = 0, cap_T3 = 0, cap_lgam = 0, cap_expl[2] = {0, 0};
     unsigned char* scratch = nullptr;     // H2D staging / pack indices
     std::vector<double> host_L;           // lgamma(n + 1), grown on demand
-    std::vector<uint64_t> host_tiles;     // 3-way-table mode tile list (build_t3_tc)
+    std::vector<uint64_t> host_tiles;     // 3-way-table mode / third-order search tile lists
+    uint64_t* d_tiles3 = nullptr;         // device copy of a host-built tile list
+    size_t cap_tiles3 = 0;
+    int64_t t3_tiles_key = -1;            // d_tiles3 holds the resident-T3 tiles of this N (no rebuild per load)
+    int64_t t3_tiles_n = 0;
+    int64_t lgam_m = -1, xlx_m = -1;      // M of the tables currently on the device (uploaded once per M)
     size_t cap_scratch = 0;
     // search workspace
     Unit* d_units = nullptr;
     int64_t* d_prefix = nullptr;
     size_t units_cap = 0;
+    SearchPlan plan;
+    int64_t tile_chunk = (int64_t)1 << 25;   // tiles per search launch (bounds the tile table: 256 MiB)
     uint64_t* d_tiles = nullptr;   // tensor-core pipe: decoded tile table (k_tile_table), 8 B per tile
     size_t cap_tiles = 0;
     unsigned long long* d_counters = nullptr;   // [0] tile counter, [1] quads done
@@ -103,6 +126,7 @@ struct epi4_ctx {
     int32_t* d_out_n = nullptr;
     unsigned int* d_status = nullptr;
     uint32_t* dump = nullptr;
+    unsigned char* h_out = nullptr;       // pinned: small device -> host results (counts, status, counters)
     // verification sample (epi4_set_sample)
     int64_t samp_cap = 0;
     uint64_t samp_seed = 0, samp_mask = 0;
@@ -220,7 +244,15 @@ std::vector<PlanEntry> all_units(int32_t n) {
     return v;
 }
 
-std::vector<PlanEntry> plan_rank(int32_t n, int32_t rank, int32_t world) {
+// Slab group of a unit for the windowed 3-way table: (128-SNP range of w, 128-SNP range of x) — a launch over one
+// group reads only the slabs FIRST(R) and FIRST(X).
+inline int64_t slab_group(const Unit& u) { return (int64_t)u.wr * 65536 + u.x / EPI4_WP; }
+
+// Static LPT plan of this rank, identical on every rank.  grouped = false: units dealt longest
+// first onto the least-loaded rank.  grouped = true (windowed T3): whole slab groups (R, X) are dealt longest
+// first, so a rank rebuilds only the slabs of its own groups (~groups / world of them instead of all); a group
+// larger than 1/(4 world) of the total is split into x sub-ranges first so that the partition stays balanced.
+std::vector<PlanEntry> plan_rank(int32_t n, int32_t rank, int32_t world, bool grouped = false) {
     std::vector<PlanEntry> v = all_units(n);
     // longest processing time first; ties broken by (wb, x) so every rank computes the same plan
     std::stable_sort(v.begin(), v.end(), [](const PlanEntry& a, const PlanEntry& b) {
@@ -231,12 +263,43 @@ std::vector<PlanEntry> plan_rank(int32_t n, int32_t rank, int32_t world) {
     if (world <= 1) return v;
     std::vector<double> load(world, 0.0);
     std::vector<PlanEntry> mine;
-    for (const PlanEntry& e : v) {
+    if (!grouped) {
+        for (const PlanEntry& e : v) {
+            int best = 0;
+            for (int r = 1; r < world; ++r)
+                if (load[r] < load[best]) best = r;
+            load[best] += e.cost;
+            if (best == rank) mine.push_back(e);
+        }
+        return mine;
+    }
+    // groups of units in (R, X) order, big groups split into consecutive-x pieces of <= cap cost
+    std::stable_sort(v.begin(), v.end(), [](const PlanEntry& a, const PlanEntry& b) {
+        const int64_t ga = slab_group(a.u), gb = slab_group(b.u);
+        if (ga != gb) return ga < gb;
+        return a.u.x < b.u.x;
+    });
+    double total = 0.0;
+    for (const PlanEntry& e : v) total += e.cost;
+    const double cap = total / (4.0 * world);
+    struct Piece { size_t b, e; double cost; };
+    std::vector<Piece> pieces;
+    for (size_t i = 0; i < v.size(); ++i) {
+        const bool same = !pieces.empty() && slab_group(v[pieces.back().b].u) == slab_group(v[i].u);
+        if (!same || pieces.back().cost + v[i].cost > cap) pieces.push_back(Piece{i, i, 0.0});
+        pieces.back().e = i + 1;
+        pieces.back().cost += v[i].cost;
+    }
+    std::vector<size_t> order(pieces.size());
+    for (size_t i = 0; i < order.size(); ++i) order[i] = i;
+    std::stable_sort(order.begin(), order.end(), [&](size_t a, size_t b) { return pieces[a].cost > pieces[b].cost; });
+    for (size_t k : order) {
         int best = 0;
         for (int r = 1; r < world; ++r)
             if (load[r] < load[best]) best = r;
-        load[best] += e.cost;
-        if (best == rank) mine.push_back(e);
+        load[best] += pieces[k].cost;
+        if (best == rank)
+            for (size_t i = pieces[k].b; i < pieces[k].e; ++i) mine.push_back(v[i]);
     }
     return mine;
 }
@@ -258,6 +321,72 @@ int ensure_lists(epi4_ctx* c, int32_t slots, int32_t cap) {
     return 0;
 }
 
+int prepare_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t G, int32_t YR) {
+    SearchPlan& pl = c->plan;
+    if (pl.valid && pl.n == c->n && pl.rank == c->opts.rank && pl.world == c->opts.world && pl.pipe == c->opts.pipe &&
+        pl.windowed == c->t3_windowed && pl.ub == ub && pl.ue == ue)
+        return 0;
+    pl.valid = false;
+    pl.table_cached = false;
+    std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world, c->t3_windowed);
+    const int64_t nall = (int64_t)plan.size();
+    int64_t b = ub < 0 ? 0 : ub, e = (ue < 0 || ue > nall) ? nall : ue;
+    if (b > e) b = e;
+    const int64_t nu = e - b;
+    pl.units.assign((size_t)nu, Unit{0, 0});
+    for (int64_t i = 0; i < nu; ++i) pl.units[(size_t)i] = plan[(size_t)(b + i)].u;
+    // Windowed T3: the units are taken grouped by slab (R, X) so that each launch reads only the slabs FIRST(R)
+    // and FIRST(X) (rebuilt on the tensor cores when R or X changes); the result does not depend on the order
+    // (top-k by (K2, index)).  Resident T3: one group, the plan order.
+    pl.groups.clear();
+    if (c->t3_windowed && nu > 0) {
+        std::stable_sort(pl.units.begin(), pl.units.end(), [](const Unit& p, const Unit& q) {
+            const int64_t gp = slab_group(p), gq = slab_group(q);
+            return gp != gq ? gp < gq : p.x < q.x;
+        });
+        for (int64_t i = 0; i < nu; ++i) {
+            const Unit& u = pl.units[(size_t)i];
+            if (pl.groups.empty() || pl.groups.back().wr != u.wr || pl.groups.back().xr != u.x / EPI4_WP)
+                pl.groups.push_back(SearchPlan::Group{i, i, u.wr, u.x / EPI4_WP});
+            pl.groups.back().e = i + 1;
+        }
+    } else if (nu > 0) {
+        pl.groups.push_back(SearchPlan::Group{0, nu, -1, -1});
+    }
+    pl.prefix.assign((size_t)nu, 0);
+    int64_t maxg = 0;
+    for (const SearchPlan::Group& g : pl.groups) {
+        int64_t acc = 0;
+        for (int64_t i = g.b; i < g.e; ++i) {
+            acc += unit_tiles(c->n, pl.units[(size_t)i].x, YR) * G;
+            pl.prefix[(size_t)i] = acc;
+        }
+        maxg = std::max(maxg, acc);
+    }
+    if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
+        dfree(c->d_units);
+        dfree(c->d_prefix);
+        c->units_cap = (size_t)std::max<int64_t>(nu, 1);
+        CU(cudaMalloc(&c->d_units, c->units_cap * sizeof(Unit)));
+        CU(cudaMalloc(&c->d_prefix, c->units_cap * sizeof(int64_t)));
+    }
+    if (nu > 0) {   // pageable sources: complete when cudaMemcpy returns
+        CU(cudaMemcpy(c->d_units, pl.units.data(), (size_t)nu * sizeof(Unit), cudaMemcpyHostToDevice));
+        CU(cudaMemcpy(c->d_prefix, pl.prefix.data(), (size_t)nu * sizeof(int64_t), cudaMemcpyHostToDevice));
+    }
+    if (c->opts.pipe != EPI4_PIPE_LOP3)
+        CU(grow(c->d_tiles, c->cap_tiles, (size_t)std::max<int64_t>(1, std::min(maxg, c->tile_chunk)) * sizeof(uint64_t)));
+    pl.n = c->n;
+    pl.rank = c->opts.rank;
+    pl.world = c->opts.world;
+    pl.pipe = c->opts.pipe;
+    pl.windowed = c->t3_windowed;
+    pl.ub = ub;
+    pl.ue = ue;
+    pl.valid = true;
+    return 0;
+}
+
 // bytes of one windowed-T3 slab: 128 first SNPs x C(n, 2) pairs x 8 packed cells
 size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * sizeof(uint32_t); }
 
@@ -267,24 +396,33 @@ size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * s
 // as the slab FIRST([slab_w0, slab_w0 + 128)) (DevData t3_win).
 int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) {
     const int32_t n = c->n;
-    std::vector<uint64_t>& tiles = c->host_tiles;
-    tiles.clear();
-    for (int32_t x = 1; x <= n - 2; ++x)
-        for (int32_t wp = 0; wp * EPI4_WP < x; ++wp) {
-            if (slab_w0 >= 0 && wp * EPI4_WP != slab_w0) continue;
-            for (int32_t y0 = x + 1; y0 <= n - 1; y0 += EPI4_YR_TC)
-                tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
-                                ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
-        }
-    if (tiles.empty()) return 0;
-    CU(grow(c->d_tiles, c->cap_tiles, tiles.size() * sizeof(uint64_t)));
-    CU(cudaMemcpyAsync(c->d_tiles, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice, c->stream));
+    // the tile list depends only on (N, slab): the resident list is kept on the device across loads of the same N
+    const int64_t key = (int64_t)n * 2 + (slab_w0 >= 0 ? 1 : 0);
+    if (slab_w0 >= 0 || c->t3_tiles_key != key) {
+        std::vector<uint64_t>& tiles = c->host_tiles;
+        tiles.clear();
+        for (int32_t x = 1; x <= n - 2; ++x)
+            for (int32_t wp = 0; wp * EPI4_WP < x; ++wp) {
+                if (slab_w0 >= 0 && wp * EPI4_WP != slab_w0) continue;
+                for (int32_t y0 = x + 1; y0 <= n - 1; y0 += EPI4_YR_TC)
+                    tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
+                                    ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
+            }
+        c->t3_tiles_key = -1;
+        c->t3_tiles_n = (int64_t)tiles.size();
+        if (tiles.empty()) return 0;
+        CU(grow(c->d_tiles3, c->cap_tiles3, tiles.size() * sizeof(uint64_t)));
+        // pageable source: the copy is complete when cudaMemcpy returns
+        CU(cudaMemcpy(c->d_tiles3, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice));
+        if (slab_w0 < 0) c->t3_tiles_key = key;
+    }
+    if (c->t3_tiles_n == 0) return 0;
     const int32_t grid = std::max(2, (c->opts.grid > 0 ? c->opts.grid : c->sm_count) / 2 * 2);
     if (int r = ensure_lists(c, grid, 1)) return r;
     SearchParams sp{};
     sp.d = devdata(c);
-    sp.tile_info = c->d_tiles;
-    sp.ntiles = (int64_t)tiles.size();
+    sp.tile_info = c->d_tiles3;
+    sp.ntiles = c->t3_tiles_n;
     sp.t3_out = out;
     sp.t3_slab_w0 = slab_w0;
     sp.topk = 1;
@@ -295,19 +433,14 @@ int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) 
     sp.quads_done = c->d_counters + 2;
     sp.prof = c->d_counters + 24;
     CU(launch_quad_tc(sp, grid, c->stream, launches));
-    CU(cudaStreamSynchronize(c->stream));   // the host tile list must outlive the async copy
     return 0;
 }
 
+// The rest of a load, enqueued behind the pack / retile kernels without waiting for them: tables, expansion,
+// T1/T2/T3.  The only host synchronisation of a load is the one at its end, which also reads the status word the
+// pack / retile kernels set (invalid genotype codes, pad bits, AA & Aa), so a bad dataset is still rejected by
+// the load call itself.
 int finish_load(epi4_ctx* c) {
-    // status of the pack / retile kernels
-    unsigned int st = 0;
-    CU(cudaMemcpyAsync(&st, c->d_status, sizeof st, cudaMemcpyDeviceToHost, c->stream));
-    CU(cudaStreamSynchronize(c->stream));
-    if (st & EPI4_ST_BAD_GENO) return fail(EPI4_EINVAL, "genotype code > 2");
-    if (st & EPI4_ST_BAD_PHEN) return fail(EPI4_EINVAL, "phenotype value > 1");
-    if (st & EPI4_ST_PAD_BITS) return fail(EPI4_EINVAL, "pad bits beyond the sample count are set");
-    if (st & EPI4_ST_AA_AND_Aa) return fail(EPI4_EINVAL, "a sample has both AA and Aa bits set");
     // lower-order tables: packed (control | case << pk_shift) words, epilogue.cuh
     {
         const DevData dd = devdata(c);
@@ -328,7 +461,7 @@ int finish_load(epi4_ctx* c) {
     c->t3_shard = shard ? (c3(n) + c->opts.world - 1) / c->opts.world : c3(n);
     const size_t t3b = (size_t)c->t3_shard * (shard ? c->opts.world : 1) * 8 * sizeof(uint32_t);
     size_t freeb = 0, totb = 0;
-    CU(cudaMemGetInfo(&freeb, &totb));
+    if (t3b > c->cap_T3 || (c->opts.flags & EPI4_FLAG_T3_WINDOWED)) CU(cudaMemGetInfo(&freeb, &totb));   // only when growing
     // windowed T3 (tensor-core pipe): when the resident table does not fit, or on request
     c->t3_windowed = c->opts.pipe == EPI4_PIPE_TC && !shard && n >= 3 &&
                      ((c->opts.flags & EPI4_FLAG_T3_WINDOWED) ||
@@ -350,8 +483,11 @@ int finish_load(epi4_ctx* c) {
         L.resize((size_t)m + 2);
         for (size_t k = have; k < L.size(); ++k) L[k] = std::lgamma((double)k + 1.0);
     }
-    CU(grow(c->lgam, c->cap_lgam, ((size_t)m + 2) * sizeof(double)));
-    CU(cudaMemcpyAsync(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+    if (c->lgam_m != m) {   // uploaded once per sample count (pageable: complete when cudaMemcpy returns)
+        CU(grow(c->lgam, c->cap_lgam, ((size_t)m + 2) * sizeof(double)));
+        CU(cudaMemcpy(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice));
+        c->lgam_m = m;
+    }
     if (c->opts.objective == EPI4_OBJ_MI) {   // X(k) = k ln k, X(0) = 0
         std::vector<double>& X = c->host_X;
         const size_t hx = X.size();
@@ -359,10 +495,12 @@ int finish_load(epi4_ctx* c) {
             X.resize((size_t)m + 2);
             for (size_t k = hx; k < X.size(); ++k) X[k] = k ? (double)k * std::log((double)k) : 0.0;
         }
-        CU(grow(c->xlx, c->cap_xlx, ((size_t)m + 2) * sizeof(double)));
-        CU(cudaMemcpyAsync(c->xlx, X.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
+        if (c->xlx_m != m) {
+            CU(grow(c->xlx, c->cap_xlx, ((size_t)m + 2) * sizeof(double)));
+            CU(cudaMemcpy(c->xlx, X.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice));
+            c->xlx_m = m;
+        }
     }
-    CU(cudaStreamSynchronize(c->stream));   // the host table must outlive the async copy
     CU(cudaEventRecord(c->ev[2], c->stream));
     // the tensor-core pipe builds T3 on the tensor cores (k_quad_tc's 3-way-table mode, the paper's
     // tensorOp_3way) against the all-ones SNP n; the CUDA-core pipe and the sharded
@@ -384,7 +522,14 @@ int finish_load(epi4_ctx* c) {
         if (int r = build_t3_tc(c, c->T3, -1, &c->stats.launches_load)) return r;
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
-    CU(cudaStreamSynchronize(c->stream));
+    unsigned int* st_h = reinterpret_cast<unsigned int*>(c->h_out + 8);
+    CU(cudaMemcpyAsync(st_h, c->d_status, sizeof(unsigned int), cudaMemcpyDeviceToHost, c->stream));
+    CU(cudaStreamSynchronize(c->stream));   // the load's one host synchronisation
+    const unsigned int st = *st_h;
+    if (st & EPI4_ST_BAD_GENO) return fail(EPI4_EINVAL, "genotype code > 2");
+    if (st & EPI4_ST_BAD_PHEN) return fail(EPI4_EINVAL, "phenotype value > 1");
+    if (st & EPI4_ST_PAD_BITS) return fail(EPI4_EINVAL, "pad bits beyond the sample count are set");
+    if (st & EPI4_ST_AA_AND_Aa) return fail(EPI4_EINVAL, "a sample has both AA and Aa bits set");
     float ms = 0;
     CU(cudaEventElapsedTime(&ms, c->ev[2], c->ev[3]));
     c->stats.ms_pop = ms;
@@ -496,6 +641,7 @@ int epi4_create(epi4_ctx** out, int32_t cuda_device, const epi4_opts* opts) {
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_idx, EPI4_MAX_TOPK * sizeof(uint64_t));
     if (e == cudaSuccess) e = cudaMalloc(&c->d_out_n, sizeof(int32_t));
     for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = cudaEventCreate(&c->ev[i]);
+    if (e == cudaSuccess) e = cudaMallocHost(&c->h_out, 512);
     if (e != cudaSuccess) {
         epi4_destroy(c);
         return fail(EPI4_ECUDA, "create: %s", cudaGetErrorString(e));
@@ -513,6 +659,7 @@ void epi4_destroy(epi4_ctx* c) {
     dfree(c->d_units);
     dfree(c->d_prefix);
     dfree(c->d_tiles);
+    dfree(c->d_tiles3);
     dfree(c->d_counters);
     dfree(c->d_list_k2);
     dfree(c->d_list_idx);
@@ -521,6 +668,7 @@ void epi4_destroy(epi4_ctx* c) {
     dfree(c->d_out_idx);
     dfree(c->d_out_n);
     dfree(c->d_status);
+    if (c->h_out) cudaFreeHost(c->h_out);
     dfree(c->d_samp_n);
     dfree(c->d_samp_idx);
     dfree(c->d_samp_key);
@@ -584,6 +732,15 @@ int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, i
     CU(cudaSetDevice(c->device));
     c->stats.launches_load = 0;
     const uint8_t *dg = geno, *dp = phen;
+    // class sizes: counted here for host phenotypes (no device round trip), by the split kernel for device ones
+    int32_t cnt[2] = {0, 0};
+    if (ptr_kind == EPI4_PTR_HOST) {
+        for (int64_t s = 0; s < m; ++s) {
+            if (phen[s] > 1) return fail(EPI4_EINVAL, "phenotype value > 1");
+            ++cnt[phen[s]];
+        }
+        if (int r = check_dims(n_snps, cnt[0], cnt[1])) return r;
+    }
     // scratch: [pack indices (2m+2) int32][genotypes n*m][phenotypes m] (the last two only for host input)
     const size_t idx_bytes = ((size_t)(2 * m + 2) * sizeof(int32_t) + 255) & ~(size_t)255;
     const size_t gbytes = ptr_kind == EPI4_PTR_HOST ? (((size_t)n_snps * m + 255) & ~(size_t)255) + (size_t)m : 0;
@@ -601,26 +758,24 @@ int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, i
     CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
     // pass 1: split by phenotype (idx0 at [0, m), idx1 at [m, 2m), counts at [2m, 2m+2))
     CU(launch_split_phen(dp, m, idx, idx + m, idx + 2 * m, c->d_status, c->stream, &c->stats.launches_load));
-    int32_t cnt[2] = {0, 0};
-    unsigned int st = 0;
-    CU(cudaMemcpyAsync(cnt, idx + 2 * m, sizeof cnt, cudaMemcpyDeviceToHost, c->stream));
-    CU(cudaMemcpyAsync(&st, c->d_status, sizeof st, cudaMemcpyDeviceToHost, c->stream));
-    CU(cudaStreamSynchronize(c->stream));
-    int r = 0;
-    if (st & EPI4_ST_BAD_PHEN) r = fail(EPI4_EINVAL, "phenotype value > 1");
-    else r = check_dims(n_snps, cnt[0], cnt[1]);
-    if (!r) r = alloc_planes(c, n_snps, cnt[0], cnt[1]);
-    if (!r) {
-        for (int p = 0; p < 2 && !r; ++p) {
-            cudaError_t e = launch_pack(dg, n_snps, m, idx + (p ? m : 0), c->np[p], c->npad, c->nchunks[p],
-                                        c->planes[p], c->d_status, c->stream, &c->stats.launches_load);
-            if (e != cudaSuccess) r = fail(EPI4_ECUDA, "pack: %s", cudaGetErrorString(e));
-        }
+    if (ptr_kind == EPI4_PTR_DEVICE) {   // the sizes decide allocations and launch shapes: one small round trip
+        int32_t* h = reinterpret_cast<int32_t*>(c->h_out);
+        CU(cudaMemcpyAsync(h, idx + 2 * m, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
+        CU(cudaMemcpyAsync(h + 2, c->d_status, sizeof(unsigned int), cudaMemcpyDeviceToHost, c->stream));
+        CU(cudaStreamSynchronize(c->stream));
+        if ((uint32_t)h[2] & EPI4_ST_BAD_PHEN) return fail(EPI4_EINVAL, "phenotype value > 1");
+        cnt[0] = h[0];
+        cnt[1] = h[1];
+        if (int r = check_dims(n_snps, cnt[0], cnt[1])) return r;
     }
-    cudaEventRecord(c->ev[1], c->stream);
-    cudaStreamSynchronize(c->stream);
-    if (r) return r;
-    r = finish_load(c);
+    if (int r = alloc_planes(c, n_snps, cnt[0], cnt[1])) return r;
+    for (int p = 0; p < 2; ++p) {
+        cudaError_t e = launch_pack(dg, n_snps, m, idx + (p ? m : 0), c->np[p], c->npad, c->nchunks[p], c->planes[p],
+                                    c->d_status, c->stream, &c->stats.launches_load);
+        if (e != cudaSuccess) return fail(EPI4_ECUDA, "pack: %s", cudaGetErrorString(e));
+    }
+    CU(cudaEventRecord(c->ev[1], c->stream));
+    const int r = finish_load(c);   // no synchronisation before it: the pack status is read at its end
     float ms = 0;
     cudaEventElapsedTime(&ms, c->ev[0], c->ev[1]);
     c->stats.ms_pack = ms;
@@ -693,24 +848,29 @@ int epi4_get_sample(epi4_ctx* c, uint64_t* quads_out, double* keys_out, uint32_t
     return 0;
 }
 
-int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world) {
+int64_t epi4_plan_count_ex(int32_t n_snps, int32_t rank, int32_t world, int32_t flags) {
     if (n_snps < 4 || n_snps > 65536 || world < 1 || rank < 0 || rank >= world) {
         fail(EPI4_EINVAL, "bad plan arguments");
         return EPI4_EINVAL;
     }
-    return (int64_t)plan_rank(n_snps, rank, world).size();
+    return (int64_t)plan_rank(n_snps, rank, world, (flags & EPI4_FLAG_T3_WINDOWED) != 0).size();
 }
 
-int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* out, double* cost_out) {
+int epi4_plan_units_ex(int32_t n_snps, int32_t rank, int32_t world, int32_t flags, int32_t* out, double* cost_out) {
     if (n_snps < 4 || n_snps > 65536 || world < 1 || rank < 0 || rank >= world || !out)
         return fail(EPI4_EINVAL, "bad plan arguments");
-    std::vector<PlanEntry> v = plan_rank(n_snps, rank, world);
+    std::vector<PlanEntry> v = plan_rank(n_snps, rank, world, (flags & EPI4_FLAG_T3_WINDOWED) != 0);
     for (size_t i = 0; i < v.size(); ++i) {
         out[2 * i] = v[i].u.wr;
         out[2 * i + 1] = v[i].u.x;
         if (cost_out) cost_out[i] = v[i].cost;
     }
     return 0;
+}
+
+int64_t epi4_plan_count(int32_t n_snps, int32_t rank, int32_t world) { return epi4_plan_count_ex(n_snps, rank, world, 0); }
+int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* out, double* cost_out) {
+    return epi4_plan_units_ex(n_snps, rank, world, 0, out, cost_out);
 }
 
 int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64_t* quads_out, double* k2_out,
@@ -721,43 +881,12 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (top_k < 1 || top_k > EPI4_MAX_TOPK) return fail(EPI4_EINVAL, "top_k=%d outside [1, %d]", top_k, EPI4_MAX_TOPK);
     if (!quads_out || !k2_out || !n_out) return fail(EPI4_EINVAL, "NULL output pointer");
     CU(cudaSetDevice(c->device));
-    std::vector<PlanEntry> plan = plan_rank(c->n, c->opts.rank, c->opts.world);
-    const int64_t nall = (int64_t)plan.size();
-    if (ue < 0 || ue > nall) ue = nall;
-    if (ub < 0) ub = 0;
-    if (ub > ue) ub = ue;
-    const int64_t nu = ue - ub;
     if (c->opts.pipe != EPI4_PIPE_LOP3 && std::max(c->np[0], c->np[1]) > ((int64_t)1 << 24))
         return fail(EPI4_EINVAL, "tensor-core pipe: fp32 accumulators are exact up to 2^24 samples per phenotype "
                                  "(%lld, %lld); use EPI4_PIPE_LOP3", (long long)c->np[0], (long long)c->np[1]);
     const int32_t G = quad_split(c->opts.pipe), YR = quad_yr(c->opts.pipe);
-    std::vector<Unit> units((size_t)std::max<int64_t>(nu, 1));
-    for (int64_t i = 0; i < nu; ++i) units[(size_t)i] = plan[(size_t)(ub + i)].u;
-    // Windowed T3: the units are taken grouped by (w-range R, 128-SNP x-range X) so that each launch reads
-    // only the slabs FIRST(R) and FIRST(X) (rebuilt on the tensor cores when R or X changes); the result does
-    // not depend on the order (top-k by (K2, index)).  Resident T3: one group, the plan order.
-    struct Group { int64_t b, e; int32_t wr, xr; };
-    std::vector<Group> groups;
-    if (c->t3_windowed && nu > 0) {
-        std::stable_sort(units.begin(), units.begin() + nu, [](const Unit& p, const Unit& q) {
-            return p.wr != q.wr ? p.wr < q.wr : p.x < q.x;
-        });
-        for (int64_t i = 0; i < nu; ++i) {
-            const int32_t xr = units[(size_t)i].x / EPI4_WP;
-            if (groups.empty() || groups.back().wr != units[(size_t)i].wr || groups.back().xr != xr)
-                groups.push_back(Group{i, i, units[(size_t)i].wr, xr});
-            groups.back().e = i + 1;
-        }
-    } else if (nu > 0) {
-        groups.push_back(Group{0, nu, -1, -1});
-    }
-    if ((size_t)std::max<int64_t>(nu, 1) > c->units_cap) {
-        dfree(c->d_units);
-        dfree(c->d_prefix);
-        c->units_cap = (size_t)std::max<int64_t>(nu, 1);
-        CU(cudaMalloc(&c->d_units, c->units_cap * sizeof(Unit)));
-        CU(cudaMalloc(&c->d_prefix, c->units_cap * sizeof(int64_t)));
-    }
+    if (int r = prepare_units(c, ub, ue, G, YR)) return r;
+    const SearchPlan& pl = c->plan;
     int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
     grid = std::max(2, grid / 2 * 2);                 // whole CTA pairs
     if (int r = ensure_lists(c, grid, top_k)) return r;
@@ -765,16 +894,9 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaMemsetAsync(c->d_counters, 0, 32 * sizeof(unsigned long long), c->stream));
     CU(cudaMemsetAsync(c->d_status, 0, sizeof(unsigned int), c->stream));
 
-    SearchParams sp;
+    SearchParams sp{};
     sp.d = devdata(c);
-    sp.units = c->d_units;
-    sp.prefix = c->d_prefix;
-    sp.tile_info = nullptr;
-    sp.t3_out = nullptr;
     sp.t3_slab_w0 = -1;
-    sp.search3 = 0;
-    sp.nunits = 0;
-    sp.ntiles = 0;
     sp.tile_counter = c->d_counters;
     sp.topk = top_k;
     sp.list_k2 = c->d_list_k2;
@@ -804,16 +926,9 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     CU(cudaEventRecord(c->ev[2], c->stream));
     int64_t acc = 0;
     int32_t slab_r = -1, slab_x = -1;
-    std::vector<int64_t> prefix;
-    for (const Group& gr : groups) {
-        const int64_t gn = gr.e - gr.b;
-        prefix.assign((size_t)gn, 0);
-        int64_t gacc = 0;
-        for (int64_t i = 0; i < gn; ++i) {
-            gacc += unit_tiles(c->n, units[(size_t)(gr.b + i)].x, YR) * G;
-            prefix[(size_t)i] = gacc;
-        }
-        if (gacc == 0) continue;
+    for (const SearchPlan::Group& gr : pl.groups) {
+        const int64_t gn = gr.e - gr.b, gtiles = pl.prefix[(size_t)gr.e - 1];
+        if (gtiles == 0) continue;
         if (c->t3_windowed) {
             if (gr.wr != slab_r) {            // FIRST(R) into T3
                 if (int r = build_t3_tc(c, c->T3, gr.wr * EPI4_WP, &c->stats.launches)) return r;
@@ -830,21 +945,28 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
             sp.d.T3 = c->T3;
             sp.d.T3x = gr.xr == gr.wr ? c->T3 : c->T3x;
         }
-        // pageable host source: the copy has completed when cudaMemcpyAsync returns, so `prefix` may be reused
-        CU(cudaMemcpyAsync(c->d_units, units.data() + gr.b, gn * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
-        CU(cudaMemcpyAsync(c->d_prefix, prefix.data(), gn * sizeof(int64_t), cudaMemcpyHostToDevice, c->stream));
+        sp.units = c->d_units + gr.b;
+        sp.prefix = c->d_prefix + gr.b;
         sp.nunits = gn;
-        sp.ntiles = gacc;
-        sp.tile_info = nullptr;
-        if (c->opts.pipe != EPI4_PIPE_LOP3) {
-            CU(grow(c->d_tiles, c->cap_tiles, (size_t)gacc * sizeof(uint64_t)));
-            sp.tile_info = c->d_tiles;
-            CU(launch_tile_table(sp, c->d_tiles, c->stream, &c->stats.launches));
+        if (c->opts.pipe == EPI4_PIPE_LOP3) {
+            sp.ntiles = gtiles;
+            sp.tile_info = nullptr;
+            CU(launch_quad_lop3(sp, grid, c->stream, &c->stats.launches));
+        } else {
+            // tiles in chunks of at most tile_chunk (bounded tile-table memory), one persistent launch each
+            for (int64_t t0 = 0; t0 < gtiles; t0 += c->tile_chunk) {
+                const int64_t t1 = std::min(gtiles, t0 + c->tile_chunk);
+                const bool whole = pl.groups.size() == 1 && t0 == 0 && t1 == gtiles;
+                if (!(whole && pl.table_cached)) {
+                    CU(launch_tile_table(sp, t0, t1, c->d_tiles, c->stream, &c->stats.launches));
+                    c->plan.table_cached = whole;
+                }
+                sp.tile_info = c->d_tiles;
+                sp.ntiles = t1 - t0;
+                CU(launch_quad_tc(sp, grid, c->stream, &c->stats.launches));
+            }
         }
-        cudaError_t e = c->opts.pipe == EPI4_PIPE_LOP3 ? launch_quad_lop3(sp, grid, c->stream, &c->stats.launches)
-                                                       : launch_quad_tc(sp, grid, c->stream, &c->stats.launches);
-        CU(e);
-        acc += gacc;
+        acc += gtiles;
     }
     CU(cudaEventRecord(c->ev[3], c->stream));
     CU(launch_merge(sp, grid, c->d_out_k2, c->d_out_idx, c->d_out_n, c->stream, &c->stats.launches));
@@ -907,6 +1029,7 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     sp.t3_slab_w0 = -1;
     sp.search3 = 1;
     sp.topk = top_k;
+    c->plan.table_cached = false;             // d_tiles is reused below
     sp.list_k2 = c->d_list_k2;
     sp.list_idx = c->d_list_idx;
     sp.list_cnt = c->d_list_cnt;

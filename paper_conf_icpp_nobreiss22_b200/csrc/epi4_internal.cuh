@@ -202,7 +202,8 @@ cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T
                        cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_lop3(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
 cudaError_t launch_quad_tc(const SearchParams& sp, int32_t grid, cudaStream_t s, int64_t* launches);
-cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches);
+cudaError_t launch_tile_table(const SearchParams& sp, int64_t t0, int64_t t1, uint64_t* out, cudaStream_t s,
+                              int64_t* launches);
 int32_t quad_split(int32_t pipe);   // tiles per unit tile (CUDA-core kernel: the two 64-SNP halves)
 int32_t quad_yr(int32_t pipe);      // y-range of a tile
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,

@@ -290,16 +290,18 @@ __device__ __forceinline__ TileInfo decode_tile(const SearchParams& sp, int64_t 
 // The tile table (one uint64 per tile, filled by k_tile_table before the search): a tile change in the hot
 // kernel costs one load instead of decode_tile's binary search over the unit prefix (~log2(units) dependent
 // global loads) and the y-range loop, which stalled the TMA / producer / epilogue warps at every tile change.
-__global__ void __launch_bounds__(256) k_tile_table(SearchParams sp, uint64_t* __restrict__ out) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= sp.ntiles) return;
+// tiles [t0, t1) of the launch's units (one launch per chunk of at most epi4_ctx::tile_chunk tiles)
+__global__ void __launch_bounds__(256) k_tile_table(SearchParams sp, int64_t t0, int64_t t1, uint64_t* __restrict__ out) {
+    const int64_t t = t0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= t1) return;
     const TileInfo ti = decode_tile(sp, t);
-    out[t] = (uint64_t)(uint16_t)ti.wp | ((uint64_t)(uint16_t)ti.x << 16) | ((uint64_t)(uint16_t)ti.y0 << 32) |
-             ((uint64_t)(uint16_t)ti.z << 48);
+    out[t - t0] = (uint64_t)(uint16_t)ti.wp | ((uint64_t)(uint16_t)ti.x << 16) | ((uint64_t)(uint16_t)ti.y0 << 32) |
+                  ((uint64_t)(uint16_t)ti.z << 48);
 }
-cudaError_t launch_tile_table(const SearchParams& sp, uint64_t* out, cudaStream_t s, int64_t* launches) {
-    if (sp.ntiles <= 0) return cudaSuccess;
-    k_tile_table<<<(unsigned)((sp.ntiles + 255) / 256), 256, 0, s>>>(sp, out);
+cudaError_t launch_tile_table(const SearchParams& sp, int64_t t0, int64_t t1, uint64_t* out, cudaStream_t s,
+                              int64_t* launches) {
+    if (t1 <= t0) return cudaSuccess;
+    k_tile_table<<<(unsigned)((t1 - t0 + 255) / 256), 256, 0, s>>>(sp, t0, t1, out);
     if (launches) ++*launches;
     return cudaGetLastError();
 }
