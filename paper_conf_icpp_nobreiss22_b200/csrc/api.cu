@@ -371,8 +371,10 @@ int prepare_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t G, int32_t YR) {
         CU(cudaMalloc(&c->d_prefix, c->units_cap * sizeof(int64_t)));
     }
     if (nu > 0) {   // pageable sources: complete when cudaMemcpy returns
-        CU(cudaMemcpy(c->d_units, pl.units.data(), (size_t)nu * sizeof(Unit), cudaMemcpyHostToDevice));
-        CU(cudaMemcpy(c->d_prefix, pl.prefix.data(), (size_t)nu * sizeof(int64_t), cudaMemcpyHostToDevice));
+        // stream-ordered; pageable sources are staged before cudaMemcpyAsync returns (the vectors may change after)
+        CU(cudaMemcpyAsync(c->d_units, pl.units.data(), (size_t)nu * sizeof(Unit), cudaMemcpyHostToDevice, c->stream));
+        CU(cudaMemcpyAsync(c->d_prefix, pl.prefix.data(), (size_t)nu * sizeof(int64_t), cudaMemcpyHostToDevice,
+                           c->stream));
     }
     if (c->opts.pipe != EPI4_PIPE_LOP3)
         CU(grow(c->d_tiles, c->cap_tiles, (size_t)std::max<int64_t>(1, std::min(maxg, c->tile_chunk)) * sizeof(uint64_t)));
@@ -412,8 +414,10 @@ int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) 
         c->t3_tiles_n = (int64_t)tiles.size();
         if (tiles.empty()) return 0;
         CU(grow(c->d_tiles3, c->cap_tiles3, tiles.size() * sizeof(uint64_t)));
-        // pageable source: the copy is complete when cudaMemcpy returns
-        CU(cudaMemcpy(c->d_tiles3, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice));
+        // stream-ordered (a previous slab build on the stream may still read d_tiles3); the pageable source is
+        // staged before cudaMemcpyAsync returns, so host_tiles may be rebuilt afterwards
+        CU(cudaMemcpyAsync(c->d_tiles3, tiles.data(), tiles.size() * sizeof(uint64_t), cudaMemcpyHostToDevice,
+                           c->stream));
         if (slab_w0 < 0) c->t3_tiles_key = key;
     }
     if (c->t3_tiles_n == 0) return 0;
@@ -483,9 +487,9 @@ int finish_load(epi4_ctx* c) {
         L.resize((size_t)m + 2);
         for (size_t k = have; k < L.size(); ++k) L[k] = std::lgamma((double)k + 1.0);
     }
-    if (c->lgam_m != m) {   // uploaded once per sample count (pageable: complete when cudaMemcpy returns)
+    if (c->lgam_m != m) {   // uploaded once per sample count (stream-ordered; the pageable source is staged)
         CU(grow(c->lgam, c->cap_lgam, ((size_t)m + 2) * sizeof(double)));
-        CU(cudaMemcpy(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice));
+        CU(cudaMemcpyAsync(c->lgam, L.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
         c->lgam_m = m;
     }
     if (c->opts.objective == EPI4_OBJ_MI) {   // X(k) = k ln k, X(0) = 0
@@ -497,7 +501,7 @@ int finish_load(epi4_ctx* c) {
         }
         if (c->xlx_m != m) {
             CU(grow(c->xlx, c->cap_xlx, ((size_t)m + 2) * sizeof(double)));
-            CU(cudaMemcpy(c->xlx, X.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice));
+            CU(cudaMemcpyAsync(c->xlx, X.data(), ((size_t)m + 2) * sizeof(double), cudaMemcpyHostToDevice, c->stream));
             c->xlx_m = m;
         }
     }

@@ -370,7 +370,9 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 // issuers may issue (and complete) the steps of the other parity out of order, so a waiter is only protected
 // from phase aliasing if its previous wait on a ring was on the same issuer's steps: both ring sizes must be
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
-template <int SA, int SB, bool PK16, int FILT>
+// SMP: verification variants (dump / sample hooks compiled in); the production search has neither (their
+// per-quad checks cost ~3 % at C2 in registers and branches)
+template <int SA, int SB, bool PK16, int FILT, bool SMP>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     static_assert(tc::MMA_ISSUERS == 1 ||
                   (SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2),
@@ -789,12 +791,12 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 uint64_t idx = 0;
                 bool offer = false;
                 if (valid) {
-                    uint32_t* dump = sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
+                    uint32_t* dump = SMP && sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
                     offer = true;
-                    if (dump) {
+                    if (SMP && dump) {
                         key = score_quad_rare(d, w, ti.x, y, ti.z, c16, dump);
                         if (d.objective != EPI4_OBJ_K2) key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
-                    } else if (sample_hit(sp, pack_quad(w, ti.x, y, ti.z))) {
+                    } else if (SMP && sample_hit(sp, pack_quad(w, ti.x, y, ti.z))) {
                         key = sample_record_rare(sp, w, ti.x, y, ti.z, c16);
                     } else if (sp.use_filter) {
                         // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
@@ -860,9 +862,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 #endif
 }
 
-template <int SA, int SB, bool PK16, int FILT>
+template <int SA, int SB, bool PK16, int FILT, bool SMP>
 static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
-    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16, FILT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16, FILT, SMP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
@@ -876,7 +878,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16, FILT>, sp);
+    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16, FILT, SMP>, sp);
 }
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
@@ -894,7 +896,7 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     // deepest rings that fit (the A copies carry the long L2 latency; a B stage is only held from its
     // production to its MMA)
     struct Cfg { int sa, sb; };
-    const Cfg cands[] = {{tc::MMA_ISSUERS == 1 ? 5 : 4, tc::MMA_ISSUERS == 1 ? 3 : 4}, {6, 2}, {4, 4}, {4, 2}, {2, 2}};
+    const Cfg cands[] = {{4, 4}, {2, 2}};
     Cfg pick{0, 0};
     for (const Cfg& c : cands)
         if (!pick.sa && fixed + (size_t)c.sa * tc::A_BYTES + (size_t)c.sb * tc::B_BYTES <= (size_t)optin) pick = c;
@@ -910,18 +912,16 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     cudaError_t e = cudaErrorInvalidConfiguration;
     const bool pk16 = sp.d.pk_shift == 16;
     const int filt = sp.use_filter == 2 ? 1 : sp.use_filter == 3 ? 2 : 0;   // FILT 1: chi-square, 2: MI
-#define EPI4_LAUNCH(A_, B_)                                                                        \
-    e = filt == 1 ? (pk16 ? launch_cfg<A_, B_, true, 1>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1>(sp, smem, grid, s)) \
-      : filt == 2 ? (pk16 ? launch_cfg<A_, B_, true, 2>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 2>(sp, smem, grid, s)) \
-                  : (pk16 ? launch_cfg<A_, B_, true, 0>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0>(sp, smem, grid, s))
-    if (pick.sa == 5 && pick.sb == 3) {
-        if constexpr (tc::MMA_ISSUERS == 1) EPI4_LAUNCH(5, 3);
-    } else if (pick.sa == 4 && pick.sb == 6) EPI4_LAUNCH(4, 6);
-    else if (pick.sa == 6 && pick.sb == 2) EPI4_LAUNCH(6, 2);
-    else if (pick.sa == 4 && pick.sb == 4) EPI4_LAUNCH(4, 4);
-    else if (pick.sa == 4 && pick.sb == 2) EPI4_LAUNCH(4, 2);
+    const bool smp = sp.dump != nullptr || sp.samp_cap > 0;
+#define EPI4_LAUNCH_F(A_, B_, SM_)                                                                             \
+    e = filt == 1 ? (pk16 ? launch_cfg<A_, B_, true, 1, SM_>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1, SM_>(sp, smem, grid, s)) \
+      : filt == 2 ? (pk16 ? launch_cfg<A_, B_, true, 2, SM_>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 2, SM_>(sp, smem, grid, s)) \
+                  : (pk16 ? launch_cfg<A_, B_, true, 0, SM_>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0, SM_>(sp, smem, grid, s))
+#define EPI4_LAUNCH(A_, B_) do { if (smp) EPI4_LAUNCH_F(A_, B_, true); else EPI4_LAUNCH_F(A_, B_, false); } while (0)
+    if (pick.sa == 4 && pick.sb == 4) EPI4_LAUNCH(4, 4);
     else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
 #undef EPI4_LAUNCH
+#undef EPI4_LAUNCH_F
     if (launches) ++*launches;
     return e;
 }
