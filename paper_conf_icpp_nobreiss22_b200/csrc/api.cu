@@ -160,6 +160,13 @@ double filter_offset(int64_t m) {
     return -81.0 - 81.0 * C0 - 13.5 - E;
 }
 
+// 32-bit packed words need c0 < 2^bits(n0) and bits(n0) + bits(n1) <= 32 (and counts < 2^22 for the fp32
+// exponent trick); beyond that every table and epilogue word is 64-bit (c0 | c1 << 32)
+int bits_of(int64_t v) { int b = 1; while (b < 62 && ((int64_t)1 << b) <= v) ++b; return b; }
+bool is_wide(int64_t n0, int64_t n1) {
+    return bits_of(n0) + bits_of(n1) > 32 || n0 >= ((int64_t)1 << 22) || n1 >= ((int64_t)1 << 22);
+}
+
 DevData devdata(const epi4_ctx* c) {
     DevData d;
     d.planes[0] = c->planes[0];
@@ -176,11 +183,14 @@ DevData devdata(const epi4_ctx* c) {
     d.pk_shift = 1;
     while (d.pk_shift < 31 && ((int64_t)1 << d.pk_shift) <= c->np[0]) ++d.pk_shift;
     if (c->np[0] < 65536 && c->np[1] < 65536) d.pk_shift = 16;
+    // wide: the two counts do not fit one 32-bit word -> 64-bit packed words (c0 | c1 << 32) everywhere
+    d.wide = is_wide(c->np[0], c->np[1]) ? 1 : 0;
+    if (d.wide) d.pk_shift = 32;
     d.n = c->n;
     d.npad = c->npad;
     d.np[0] = (uint32_t)c->np[0];
     d.np[1] = (uint32_t)c->np[1];
-    d.npk = (uint32_t)c->np[0] | ((uint32_t)c->np[1] << d.pk_shift);
+    d.npk = d.wide ? 0u : (uint32_t)c->np[0] | ((uint32_t)c->np[1] << d.pk_shift);
     d.T1 = c->T1;
     d.T2 = c->T2;
     d.T3 = c->T3;
@@ -447,11 +457,10 @@ int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) 
 int finish_load(epi4_ctx* c) {
     // lower-order tables: packed (control | case << pk_shift) words, epilogue.cuh
     {
-        const DevData dd = devdata(c);
-        if (c->np[0] >= ((int64_t)1 << 22) || c->np[1] >= ((int64_t)1 << 22) ||
-            c->np[1] >= ((int64_t)1 << (32 - dd.pk_shift)))
-            return fail(EPI4_EINVAL, "n0=%lld / n1=%lld: counts are packed (control | case) into one 32-bit word, which "
-                        "needs bits(n0) + bits(n1) <= 32 and each < 2^22", (long long)c->np[0], (long long)c->np[1]);
+        // counts become fp32 values 2^23 + r in the filters and pack passes: each class below 2^23 samples
+        if (c->np[0] >= ((int64_t)1 << 23) || c->np[1] >= ((int64_t)1 << 23))
+            return fail(EPI4_EINVAL, "n0=%lld / n1=%lld: each class must have fewer than 2^23 samples",
+                        (long long)c->np[0], (long long)c->np[1]);
         // chi-square: per-cell numerator r_c0^2 n1 + r_c1^2 n0 <= n0 n1 M must be exact in double (epi4.h)
         if (c->opts.objective == EPI4_OBJ_CHI2 &&
             (double)c->np[0] * (double)c->np[1] * (double)(c->np[0] + c->np[1]) >= 9007199254740992.0)
@@ -459,11 +468,12 @@ int finish_load(epi4_ctx* c) {
                         (long long)c->np[1]);
     }
     const int64_t n = c->n;
-    CU(grow(c->T1, c->cap_T1, (size_t)n * 2 * sizeof(uint32_t)));
-    CU(grow(c->T2, c->cap_T2, (size_t)c2(n) * 4 * sizeof(uint32_t)));
+    const size_t pw = is_wide(c->np[0], c->np[1]) ? 8 : 4;   // bytes per packed word
+    CU(grow(c->T1, c->cap_T1, (size_t)n * 2 * pw));
+    CU(grow(c->T2, c->cap_T2, (size_t)c2(n) * 4 * pw));
     const bool shard = (c->opts.flags & EPI4_FLAG_SHARD_T3) && c->opts.world > 1;
     c->t3_shard = shard ? (c3(n) + c->opts.world - 1) / c->opts.world : c3(n);
-    const size_t t3b = (size_t)c->t3_shard * (shard ? c->opts.world : 1) * 8 * sizeof(uint32_t);
+    const size_t t3b = (size_t)c->t3_shard * (shard ? c->opts.world : 1) * 8 * pw;
     size_t freeb = 0, totb = 0;
     if (t3b > c->cap_T3 || (c->opts.flags & EPI4_FLAG_T3_WINDOWED)) CU(cudaMemGetInfo(&freeb, &totb));   // only when growing
     // windowed T3 (tensor-core pipe): when the resident table does not fit, or on request
@@ -471,7 +481,7 @@ int finish_load(epi4_ctx* c) {
                      ((c->opts.flags & EPI4_FLAG_T3_WINDOWED) ||
                       (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3));
     if (c->t3_windowed) {
-        const size_t slab = t3_slab_bytes(n);
+        const size_t slab = t3_slab_bytes(n) * (pw / 4);
         CU(grow(c->T3, c->cap_T3, slab));
         CU(grow(c->T3x, c->cap_T3x, slab));
     }
@@ -550,7 +560,7 @@ extern "C" int epi4_t3_shard(epi4_ctx* c, void** t3_dev, int64_t* shard_bytes, i
     if (!((c->opts.flags & EPI4_FLAG_SHARD_T3) && c->opts.world > 1))
         return fail(EPI4_ESTATE, "T3 is not sharded (opts.flags & EPI4_FLAG_SHARD_T3 with world > 1)");
     *t3_dev = c->T3;
-    *shard_bytes = c->t3_shard * 8 * (int64_t)sizeof(uint32_t);
+    *shard_bytes = c->t3_shard * 8 * (int64_t)(is_wide(c->np[0], c->np[1]) ? 8 : 4);
     *total_bytes = *shard_bytes * c->opts.world;
     return 0;
 }

@@ -61,6 +61,7 @@ struct DevData {
     int32_t nsteps[2];           // tensor-core pipeline steps per phenotype: pairs of fp4 chunks (512 samples)
     int32_t nrb;                 // 128-row blocks of expl per chunk (= npad / 64)
     int32_t pk_shift;            // (control, case) counts packed as c0 | c1 << pk_shift everywhere (bits(n0))
+    int32_t wide;                // 1: packed words are 64-bit (pk_shift = 32) because bits(n0) + bits(n1) > 32
     int32_t n;                   // SNPs
     int32_t npad;                // SNP rows per chunk: ceil((n + 16) / 64) * 64 (zero rows beyond n)
     uint32_t np[2];              // n0, n1

@@ -24,25 +24,57 @@ namespace epi4 {
 
 // ---- packed counts -----------------------------------------------------------------------------------
 // Every count the epilogue handles is a PACKED pair v = c0 | c1 << pks (controls in the low pks bits, cases
-// above; pks = bits(n0), api.cu checks bits(n0) + bits(n1) <= 32).  The aa recovery of PAPER.md:L126 is a
-// chain of subtractions v_aa = v_* - v_AA - v_Aa in which every operand and every result is the number of
-// samples of one phenotype in a genotype subset, i.e. a non-negative count per field: no borrow ever crosses
-// the field boundary, so one 32-bit subtraction recovers both phenotypes exactly (half the instructions of
-// two separate recoveries, and half the table bytes).
+// above).  The aa recovery of PAPER.md:L126 is a chain of subtractions v_aa = v_* - v_AA - v_Aa in which every
+// operand and every result is the number of samples of one phenotype in a genotype subset, i.e. a non-negative
+// count per field: no borrow ever crosses the field boundary, so one subtraction recovers both phenotypes
+// exactly (half the instructions of two separate recoveries, and half the table bytes).  The packed word P is
+// uint32_t with pks = bits(n0) when bits(n0) + bits(n1) <= 32 (every BASELINE.json config), else ("wide",
+// DevData.wide) uint64_t with pks = 32: the same code on 64-bit words (sample counts up to 2^23 per class).
 //
 // Lower-order tables (api.cu / k_prep.cu, colex ranks):  T3[rank3(i,j,k)][4a+2b+c], T2[rank2(i,j)][2a+b],
-// T1[snp][a], all packed; d.npk = n0 | n1 << pks.
-__device__ __forceinline__ uint4 t3_half(const DevData& d, int64_t r3, int a) {   // cells (a, b, c), 2b + c
-    return __ldg(reinterpret_cast<const uint4*>(d.T3 + r3 * 8 + a * 4));
+// T1[snp][a], all packed P words; npk = n0 | n1 << pks.
+template <typename P>
+struct Q4 { P v[4]; };
+template <typename P>
+struct Q2 { P v[2]; };
+// 4 / 2 consecutive P words at P-index e of a table
+template <typename P>
+__device__ __forceinline__ Q4<P> ldq4(const uint32_t* base, int64_t e) {
+    Q4<P> q;
+    if constexpr (sizeof(P) == 4) {
+        const uint4 t = __ldg(reinterpret_cast<const uint4*>(base + e));
+        q.v[0] = t.x; q.v[1] = t.y; q.v[2] = t.z; q.v[3] = t.w;
+    } else {
+        const ulonglong2 a = __ldg(reinterpret_cast<const ulonglong2*>(base + 2 * e));
+        const ulonglong2 b = __ldg(reinterpret_cast<const ulonglong2*>(base + 2 * e) + 1);
+        q.v[0] = a.x; q.v[1] = a.y; q.v[2] = b.x; q.v[3] = b.y;
+    }
+    return q;
 }
-__device__ __forceinline__ uint4 t2_all(const DevData& d, int64_t r2) {            // cells 2a + b
-    return __ldg(reinterpret_cast<const uint4*>(d.T2 + r2 * 4));
+template <typename P>
+__device__ __forceinline__ Q2<P> ldq2(const uint32_t* base, int64_t e) {
+    Q2<P> q;
+    if constexpr (sizeof(P) == 4) {
+        const uint2 t = __ldg(reinterpret_cast<const uint2*>(base + e));
+        q.v[0] = t.x; q.v[1] = t.y;
+    } else {
+        const ulonglong2 a = __ldg(reinterpret_cast<const ulonglong2*>(base + 2 * e));
+        q.v[0] = a.x; q.v[1] = a.y;
+    }
+    return q;
 }
-__device__ __forceinline__ uint2 t1_all(const DevData& d, int i) {                 // cells a
-    return __ldg(reinterpret_cast<const uint2*>(d.T1 + (int64_t)i * 2));
+template <typename P>
+__device__ __forceinline__ Q4<P> t3_half(const DevData& d, int64_t r3, int a) { return ldq4<P>(d.T3, r3 * 8 + a * 4); }
+template <typename P>
+__device__ __forceinline__ Q4<P> t3x_half(const DevData& d, int64_t r3, int a) { return ldq4<P>(d.T3x, r3 * 8 + a * 4); }
+template <typename P>
+__device__ __forceinline__ Q4<P> t2_all(const DevData& d, int64_t r2) { return ldq4<P>(d.T2, r2 * 4); }
+template <typename P>
+__device__ __forceinline__ Q2<P> t1_all(const DevData& d, int i) { return ldq2<P>(d.T1, (int64_t)i * 2); }
+template <typename P>
+__device__ __forceinline__ P npk_of(const DevData& d) {
+    return sizeof(P) == 4 ? (P)d.npk : (P)d.np[0] | ((P)d.np[1] << 32);
 }
-__device__ __forceinline__ uint32_t u4(const uint4& v, int k) { return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w; }
-__device__ __forceinline__ uint32_t u2(const uint2& v, int k) { return k == 0 ? v.x : v.y; }
 
 // colex ranks of the lower-order tables a quad w < x < y < z reads
 struct QuadRanks {
@@ -81,48 +113,49 @@ __device__ __forceinline__ QuadRanks quad_ranks(const DevData& d, int w, int x, 
 //   one '*'   -> 3-way tables of the other three SNPs
 //   two '*'   -> 2-way tables
 //   three '*' -> 1-way table / n_p
-template <int A>
-__device__ __forceinline__ void fill_slab_w(uint32_t (&S)[27], const uint32_t (&c16)[16], const uint4& twxy,
-                                            const uint4& twxz, const uint4& twyz, const uint4& pwx, const uint4& pwy,
-                                            const uint4& pwz, const uint2& sw) {
+template <int A, typename P>
+__device__ __forceinline__ void fill_slab_w(P (&S)[27], const P (&c16)[16], const Q4<P>& twxy, const Q4<P>& twxz,
+                                            const Q4<P>& twyz, const Q4<P>& pwx, const Q4<P>& pwy, const Q4<P>& pwz,
+                                            const Q2<P>& sw) {
 #pragma unroll
     for (int c = 0; c < 27; ++c) {
         const int b = c / 9, e = (c / 3) % 3, f = c % 3;
         const int ns = (b == 2) + (e == 2) + (f == 2);
-        uint32_t v;
+        P v;
         if (ns == 0) v = c16[A * 8 + b * 4 + e * 2 + f];
         else if (ns == 1) {
-            if (f == 2) v = u4(twxy, b * 2 + e);
-            else if (e == 2) v = u4(twxz, b * 2 + f);
-            else v = u4(twyz, e * 2 + f);
+            if (f == 2) v = twxy.v[b * 2 + e];
+            else if (e == 2) v = twxz.v[b * 2 + f];
+            else v = twyz.v[e * 2 + f];
         } else if (ns == 2) {
-            if (b != 2) v = u4(pwx, A * 2 + b);
-            else if (e != 2) v = u4(pwy, A * 2 + e);
-            else v = u4(pwz, A * 2 + f);
+            if (b != 2) v = pwx.v[A * 2 + b];
+            else if (e != 2) v = pwy.v[A * 2 + e];
+            else v = pwz.v[A * 2 + f];
         } else {
-            v = u2(sw, A);
+            v = sw.v[A];
         }
         S[c] = v;
     }
 }
 // slab w = '*': the (x, y, z) marginal tables
-__device__ __forceinline__ void fill_slab_star(uint32_t (&S)[27], const uint4& txyz0, const uint4& txyz1,
-                                               const uint4& pxy, const uint4& pxz, const uint4& pyz, const uint2& sx,
-                                               const uint2& sy, const uint2& sz, uint32_t npk) {
+template <typename P>
+__device__ __forceinline__ void fill_slab_star(P (&S)[27], const Q4<P>& txyz0, const Q4<P>& txyz1, const Q4<P>& pxy,
+                                               const Q4<P>& pxz, const Q4<P>& pyz, const Q2<P>& sx, const Q2<P>& sy,
+                                               const Q2<P>& sz, P npk) {
 #pragma unroll
     for (int c = 0; c < 27; ++c) {
         const int b = c / 9, e = (c / 3) % 3, f = c % 3;
         const int ns = (b == 2) + (e == 2) + (f == 2);
-        uint32_t v;
-        if (ns == 0) v = b ? u4(txyz1, e * 2 + f) : u4(txyz0, e * 2 + f);
+        P v;
+        if (ns == 0) v = b ? txyz1.v[e * 2 + f] : txyz0.v[e * 2 + f];
         else if (ns == 1) {
-            if (f == 2) v = u4(pxy, b * 2 + e);
-            else if (e == 2) v = u4(pxz, b * 2 + f);
-            else v = u4(pyz, e * 2 + f);
+            if (f == 2) v = pxy.v[b * 2 + e];
+            else if (e == 2) v = pxz.v[b * 2 + f];
+            else v = pyz.v[e * 2 + f];
         } else if (ns == 2) {
-            if (b != 2) v = u2(sx, b);
-            else if (e != 2) v = u2(sy, e);
-            else v = u2(sz, f);
+            if (b != 2) v = sx.v[b];
+            else if (e != 2) v = sy.v[e];
+            else v = sz.v[f];
         } else {
             v = npk;
         }
@@ -131,13 +164,35 @@ __device__ __forceinline__ void fill_slab_star(uint32_t (&S)[27], const uint4& t
 }
 
 // aa recovery on the three axes of a slab (strides 9, 3, 1): 27 three-input subtractions on packed words
-__device__ __forceinline__ void mobius3(uint32_t (&g)[27]) {
+template <typename P>
+__device__ __forceinline__ void mobius3(P (&g)[27]) {
 #pragma unroll
     for (int ax = 0; ax < 3; ++ax) {
         const int s = ax == 0 ? 9 : ax == 1 ? 3 : 1;
 #pragma unroll
         for (int c = 0; c < 27; ++c)
             if (((c / s) % 3) == 2) g[c] = g[c] - g[c - s] - g[c - 2 * s];
+    }
+}
+
+// the two counts of a packed word, as 32-bit integers (r0 controls, r1 cases)
+template <typename P>
+__device__ __forceinline__ uint32_t cnt0(P v, uint32_t pks, uint32_t pkm) {
+    return sizeof(P) == 4 ? (uint32_t)v & pkm : (uint32_t)v;
+}
+template <typename P>
+__device__ __forceinline__ uint32_t cnt1(P v, uint32_t pks) {
+    return sizeof(P) == 4 ? (uint32_t)(v >> pks) : (uint32_t)(v >> 32);
+}
+// 2^23 + r0, 2^23 + r1 as floats (exact for counts < 2^23); with 16-bit fields one byte permute each
+template <bool PK16, typename P>
+__device__ __forceinline__ void cnt_f(P v, uint32_t pks, uint32_t pkm, float& m0, float& m1) {
+    if constexpr (sizeof(P) == 4 && PK16) {
+        m0 = __uint_as_float(__byte_perm((uint32_t)v, 0x4B000000u, 0x7410));
+        m1 = __uint_as_float(__byte_perm((uint32_t)v, 0x4B000000u, 0x7432));
+    } else {
+        m0 = __uint_as_float(cnt0(v, pks, pkm) | 0x4B000000u);
+        m1 = __uint_as_float(cnt1(v, pks) | 0x4B000000u);
     }
 }
 
@@ -151,18 +206,17 @@ __device__ __forceinline__ void mobius3(uint32_t (&g)[27]) {
 // scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
 // is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + 3 FFMA into one of three
 // running sums, 3 MUFU;
-// no table and no conversion instruction (a count r < 2^22 becomes the float 2^23 + r by setting the exponent
+// no table and no conversion instruction (a count r < 2^23 becomes the float 2^23 + r by setting the exponent
 // bits).
 __device__ __forceinline__ float lg2_approx(float x) {
     float y;
     asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
 }
-template <bool PK16>
-__device__ __forceinline__ void cell_T_acc(uint32_t v, uint32_t pks, uint32_t pkm, float& acc) {
-    // 2^23 + r0, 2^23 + r1 (with pks = 16 one byte permute each: [r.lo, r.hi, 0x00, 0x4B])
-    const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
-    const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
+template <bool PK16, typename P>
+__device__ __forceinline__ void cell_T_acc(P v, uint32_t pks, uint32_t pkm, float& acc) {
+    float m0, m1;
+    cnt_f<PK16>(v, pks, pkm, m0, m1);
     const float f0 = m0 - 8388607.0f, f1 = m1 - 8388607.0f;     // r + 1
     const float h0 = m0 - 8388607.5f, h1 = m1 - 8388607.5f;     // r + 1/2
     const float fn = f0 + f1, hn = h0 + f1;                     // n + 2, n + 3/2
@@ -183,10 +237,10 @@ __device__ __forceinline__ float rcp_approx(float x) {
     asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
 }
-template <bool PK16>
-__device__ __forceinline__ void cell_chi_acc(uint32_t v, uint32_t pks, uint32_t pkm, float ca, float cb, float& acc) {
-    const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
-    const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
+template <bool PK16, typename P>
+__device__ __forceinline__ void cell_chi_acc(P v, uint32_t pks, uint32_t pkm, float ca, float cb, float& acc) {
+    float m0, m1;
+    cnt_f<PK16>(v, pks, pkm, m0, m1);
     const float f0 = m0 - 8388608.0f, f1 = m1 - 8388608.0f;     // r0, r1 (exact)
     const float num = fmaf(f0 * ca, f0, (f1 * cb) * f1);
     acc = fmaf(num, rcp_approx(fmaxf(f0 + f1, 1.0f)), acc);
@@ -197,10 +251,10 @@ __device__ __forceinline__ void cell_chi_acc(uint32_t v, uint32_t pks, uint32_t 
 // max(k, 1)).  Each cell value is formed first (two FMAs onto -r_c lg2 r_c; |value| <= r_c bits), then added
 // to a running sum, so |V_computed - V| <= mi_E (api.cu: lg2.approx, the cell roundings, the additions).
 // The kernel scores a quad exactly only if -(ln2 (V + mi_E) + mi_const) <= the current k-th best key.
-template <bool PK16>
-__device__ __forceinline__ void cell_mi_acc(uint32_t v, uint32_t pks, uint32_t pkm, float& acc) {
-    const float m0 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7410)) : __uint_as_float((v & pkm) | 0x4B000000u);
-    const float m1 = PK16 ? __uint_as_float(__byte_perm(v, 0x4B000000u, 0x7432)) : __uint_as_float((v >> pks) | 0x4B000000u);
+template <bool PK16, typename P>
+__device__ __forceinline__ void cell_mi_acc(P v, uint32_t pks, uint32_t pkm, float& acc) {
+    float m0, m1;
+    cnt_f<PK16>(v, pks, pkm, m0, m1);
     const float f0 = m0 - 8388608.0f, f1 = m1 - 8388608.0f, fn = f0 + f1;   // r0, r1, r_c (exact)
     const float cell = fmaf(f0, lg2_approx(fmaxf(f0, 1.0f)), fmaf(f1, lg2_approx(fmaxf(f1, 1.0f)),
                                                                   -fn * lg2_approx(fmaxf(fn, 1.0f))));
@@ -215,22 +269,21 @@ __device__ __forceinline__ void cell_mi_acc(uint32_t v, uint32_t pks, uint32_t p
 // MODE 6: the fp32 MI sum V (above); MODE 1: exact K2 in double, t_c = (L[r_c0 + r_c1 + 1] -
 // L[r_c0]) - L[r_c1], K2 += t_c, c = 0..80 (reading #4); MODE 2: exact K2 and the
 // 2 x 81 cells written to dump (controls first).
-template <int MODE, bool PK16 = false>
+template <int MODE, bool PK16 = false, typename P = uint32_t>
 __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, int w, int x, int y, int z,
-                                          const uint32_t (&c16)[16], float& flt, double& k2, uint32_t* dump) {
-    const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
+                                          const P (&c16)[16], float& flt, double& k2, uint32_t* dump) {
+    const uint32_t pks = (uint32_t)d.pk_shift, pkm = sizeof(P) == 4 ? (1u << pks) - 1u : 0xFFFFFFFFu;
     // all table reads up front (one round of load latency per quad)
-    const uint4 txyz0 = __ldg(reinterpret_cast<const uint4*>(d.T3x + q.xyz * 8)),
-                txyz1 = __ldg(reinterpret_cast<const uint4*>(d.T3x + q.xyz * 8 + 4));
-    const uint4 pxy = t2_all(d, q.xy), pxz = t2_all(d, q.xz), pyz = t2_all(d, q.yz);
-    const uint2 sx = t1_all(d, x), sy = t1_all(d, y), sz = t1_all(d, z);
-    const uint4 twxy0 = t3_half(d, q.wxy, 0), twxz0 = t3_half(d, q.wxz, 0), twyz0 = t3_half(d, q.wyz, 0);
-    const uint4 twxy1 = t3_half(d, q.wxy, 1), twxz1 = t3_half(d, q.wxz, 1), twyz1 = t3_half(d, q.wyz, 1);
-    const uint4 pwx = t2_all(d, q.wx), pwy = t2_all(d, q.wy), pwz = t2_all(d, q.wz);
-    const uint2 sw = t1_all(d, w);
+    const Q4<P> txyz0 = t3x_half<P>(d, q.xyz, 0), txyz1 = t3x_half<P>(d, q.xyz, 1);
+    const Q4<P> pxy = t2_all<P>(d, q.xy), pxz = t2_all<P>(d, q.xz), pyz = t2_all<P>(d, q.yz);
+    const Q2<P> sx = t1_all<P>(d, x), sy = t1_all<P>(d, y), sz = t1_all<P>(d, z);
+    const Q4<P> twxy0 = t3_half<P>(d, q.wxy, 0), twxz0 = t3_half<P>(d, q.wxz, 0), twyz0 = t3_half<P>(d, q.wyz, 0);
+    const Q4<P> twxy1 = t3_half<P>(d, q.wxy, 1), twxz1 = t3_half<P>(d, q.wxz, 1), twyz1 = t3_half<P>(d, q.wyz, 1);
+    const Q4<P> pwx = t2_all<P>(d, q.wx), pwy = t2_all<P>(d, q.wy), pwz = t2_all<P>(d, q.wz);
+    const Q2<P> sw = t1_all<P>(d, w);
     float fa = 0.0f, fb = 0.0f, fc = 0.0f;
     double kk = 0.0;
-    auto consume = [&](const uint32_t (&S)[27], int base) {
+    auto consume = [&](const P (&S)[27], int base) {
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
             if (MODE == 0) {
@@ -242,7 +295,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
             } else if (MODE == 4) {
                 // Pearson chi-square (EPI4_OBJ_CHI2): S += (r0^2 n1 + r1^2 n0) / r_c over cells with r_c > 0,
                 // exact uint64 numerator, one correctly rounded division (oracle_chi2's order)
-                const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks, rc = r0 + r1;
+                const uint32_t r0 = cnt0(S[c], pks, pkm), r1 = cnt1(S[c], pks), rc = r0 + r1;
                 if (rc) {
                     const unsigned long long num = (unsigned long long)r0 * r0 * d.np[1] +
                                                    (unsigned long long)r1 * r1 * d.np[0];
@@ -250,10 +303,10 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
                 }
             } else if (MODE == 3) {
                 // mutual information (EPI4_OBJ_MI): (X(r0) + X(r1)) - X(r0 + r1), X(k) = k ln k
-                const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+                const uint32_t r0 = cnt0(S[c], pks, pkm), r1 = cnt1(S[c], pks);
                 kk = __dadd_rn(kk, __dsub_rn(__dadd_rn(__ldg(d.xlx + r0), __ldg(d.xlx + r1)), __ldg(d.xlx + (r0 + r1))));
             } else {
-                const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+                const uint32_t r0 = cnt0(S[c], pks, pkm), r1 = cnt1(S[c], pks);
                 const double t = __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1));
                 kk = __dadd_rn(kk, t);
                 if (MODE == 2) {
@@ -263,20 +316,20 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
             }
         }
     };
-    uint32_t R2[27];
-    fill_slab_star(R2, txyz0, txyz1, pxy, pxz, pyz, sx, sy, sz, d.npk);
+    P R2[27];
+    fill_slab_star<P>(R2, txyz0, txyz1, pxy, pxz, pyz, sx, sy, sz, npk_of<P>(d));
     mobius3(R2);
     {
-        uint32_t S[27];
-        fill_slab_w<0>(S, c16, twxy0, twxz0, twyz0, pwx, pwy, pwz, sw);
+        P S[27];
+        fill_slab_w<0, P>(S, c16, twxy0, twxz0, twyz0, pwx, pwy, pwz, sw);
         mobius3(S);
         consume(S, 0);
 #pragma unroll
         for (int c = 0; c < 27; ++c) R2[c] -= S[c];
     }
     {
-        uint32_t S[27];
-        fill_slab_w<1>(S, c16, twxy1, twxz1, twyz1, pwx, pwy, pwz, sw);
+        P S[27];
+        fill_slab_w<1, P>(S, c16, twxy1, twxz1, twyz1, pwx, pwy, pwz, sw);
         mobius3(S);
         consume(S, 27);
 #pragma unroll
@@ -295,26 +348,28 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
 // exact K2 of one quad (double, canonical order) from its packed contraction counts; optionally dumps its 162
 // cells.  Not inlined: in the tensor-core epilogue it runs only for filter candidates, so its registers must
 // not add to the hot loop's.
-static __device__ __noinline__ double score_quad(const DevData& d, int w, int x, int y, int z,
-                                                 const uint32_t (&c16)[16], uint32_t* dump_row) {
+template <typename P = uint32_t>
+static __device__ __noinline__ double score_quad(const DevData& d, int w, int x, int y, int z, const P (&c16)[16],
+                                                 uint32_t* dump_row) {
     float flt;
     double k2;
     const QuadRanks q = quad_ranks(d, w, x, y, z);
-    if (dump_row) quad_eval<2>(d, q, w, x, y, z, c16, flt, k2, dump_row);
-    else if (d.objective == EPI4_OBJ_MI) quad_eval<3>(d, q, w, x, y, z, c16, flt, k2, nullptr);
-    else if (d.objective == EPI4_OBJ_CHI2) quad_eval<4>(d, q, w, x, y, z, c16, flt, k2, nullptr);
-    else quad_eval<1>(d, q, w, x, y, z, c16, flt, k2, nullptr);
+    if (dump_row) quad_eval<2, false, P>(d, q, w, x, y, z, c16, flt, k2, dump_row);
+    else if (d.objective == EPI4_OBJ_MI) quad_eval<3, false, P>(d, q, w, x, y, z, c16, flt, k2, nullptr);
+    else if (d.objective == EPI4_OBJ_CHI2) quad_eval<4, false, P>(d, q, w, x, y, z, c16, flt, k2, nullptr);
+    else quad_eval<1, false, P>(d, q, w, x, y, z, c16, flt, k2, nullptr);
     return k2;
 }
 // Call-site wrapper for the hot loops: the counts are copied into an array local to the (rare) branch that
 // calls the noinline scorer, so the loop's own c16 never has its address taken and stays in registers (passing
 // c16 itself made the compiler store all 16 counts to the stack on every quad: 1.5 G STL per C2 slice, ncu).
+template <typename P = uint32_t>
 static __device__ __forceinline__ double score_quad_rare(const DevData& d, int w, int x, int y, int z,
-                                                         const uint32_t (&c16)[16], uint32_t* dump_row) {
-    uint32_t t[16];
+                                                         const P (&c16)[16], uint32_t* dump_row) {
+    P t[16];
 #pragma unroll
     for (int k = 0; k < 16; ++k) t[k] = c16[k];
-    return score_quad(d, w, x, y, z, t, dump_row);
+    return score_quad<P>(d, w, x, y, z, t, dump_row);
 }
 // Verification sample (epi4_set_sample): is quad `idx` sampled?  Then record it: packed index, exact key of the
 // context's objective and its 2 x 81 counts, from the counts the search kernel itself produced.  Returns the
@@ -322,25 +377,27 @@ static __device__ __forceinline__ double score_quad_rare(const DevData& d, int w
 __device__ __forceinline__ bool sample_hit(const SearchParams& sp, uint64_t idx) {
     return sp.samp_cap && (mix64(idx ^ sp.samp_seed) & sp.samp_mask) == 0;
 }
+template <typename P = uint32_t>
 static __device__ __noinline__ double sample_record(const SearchParams& sp, int w, int x, int y, int z,
-                                                    const uint32_t (&c16)[16]) {
+                                                    const P (&c16)[16]) {
     const unsigned long long slot = atomicAdd(sp.samp_n, 1ull);
     uint32_t scratch[162];
     uint32_t* row = slot < (unsigned long long)sp.samp_cap ? sp.samp_counts + slot * 162 : scratch;
-    double key = score_quad(sp.d, w, x, y, z, c16, row);            // K2 + counts
-    if (sp.d.objective != EPI4_OBJ_K2) key = score_quad(sp.d, w, x, y, z, c16, nullptr);
+    double key = score_quad<P>(sp.d, w, x, y, z, c16, row);            // K2 + counts
+    if (sp.d.objective != EPI4_OBJ_K2) key = score_quad<P>(sp.d, w, x, y, z, c16, nullptr);
     if (slot < (unsigned long long)sp.samp_cap) {
         sp.samp_idx[slot] = pack_quad(w, x, y, z);
         sp.samp_key[slot] = key;
     }
     return key;
 }
+template <typename P = uint32_t>
 static __device__ __forceinline__ double sample_record_rare(const SearchParams& sp, int w, int x, int y, int z,
-                                                            const uint32_t (&c16)[16]) {
-    uint32_t t[16];
+                                                            const P (&c16)[16]) {
+    P t[16];
 #pragma unroll
     for (int k = 0; k < 16; ++k) t[k] = c16[k];
-    return sample_record(sp, w, x, y, z, t);
+    return sample_record<P>(sp, w, x, y, z, t);
 }
 
 // Third-order search: exact K2 of triple w < x < y from its 8 packed non-aa counts
@@ -348,27 +405,28 @@ static __device__ __forceinline__ double sample_record_rare(const SearchParams& 
 // cells S[9a + 3b + c] (digit 2 = '*') from c8, T2, T1 and n, aa recovered on the three axes,
 // K2 = sum_c ((L[r_c + 1] - L[r_c0]) - L[r_c1]) in canonical order c = 9a + 3b + c (reading #4); with
 // EPI4_OBJ_MI / EPI4_OBJ_CHI2 the key is -M*I / -X^2 of the 2 x 27 table, as in quad_eval MODE 3 / 4.
-static __device__ __noinline__ double score_triple(const DevData& d, int w, int x, int y, const uint32_t (&c8)[8]) {
-    const uint32_t pks = (uint32_t)d.pk_shift, pkm = (1u << pks) - 1u;
-    const uint4 pwx = t2_all(d, c2(x) + w), pwy = t2_all(d, c2(y) + w), pxy = t2_all(d, c2(y) + x);
-    const uint2 sw = t1_all(d, w), sx = t1_all(d, x), sy = t1_all(d, y);
-    uint32_t S[27];
+template <typename P = uint32_t>
+static __device__ __noinline__ double score_triple(const DevData& d, int w, int x, int y, const P (&c8)[8]) {
+    const uint32_t pks = (uint32_t)d.pk_shift, pkm = sizeof(P) == 4 ? (1u << pks) - 1u : 0xFFFFFFFFu;
+    const Q4<P> pwx = t2_all<P>(d, c2(x) + w), pwy = t2_all<P>(d, c2(y) + w), pxy = t2_all<P>(d, c2(y) + x);
+    const Q2<P> sw = t1_all<P>(d, w), sx = t1_all<P>(d, x), sy = t1_all<P>(d, y);
+    P S[27];
 #pragma unroll
     for (int c = 0; c < 27; ++c) {
         const int a = c / 9, b = (c / 3) % 3, e = c % 3;
         const int ns = (a == 2) + (b == 2) + (e == 2);
-        uint32_t v;
+        P v;
         if (ns == 0) v = c8[4 * a + 2 * b + e];
         else if (ns == 1) {
-            if (a == 2) v = u4(pxy, 2 * b + e);
-            else if (b == 2) v = u4(pwy, 2 * a + e);
-            else v = u4(pwx, 2 * a + b);
+            if (a == 2) v = pxy.v[2 * b + e];
+            else if (b == 2) v = pwy.v[2 * a + e];
+            else v = pwx.v[2 * a + b];
         } else if (ns == 2) {
-            if (a != 2) v = u2(sw, a);
-            else if (b != 2) v = u2(sx, b);
-            else v = u2(sy, e);
+            if (a != 2) v = sw.v[a];
+            else if (b != 2) v = sx.v[b];
+            else v = sy.v[e];
         } else {
-            v = d.npk;
+            v = npk_of<P>(d);
         }
         S[c] = v;
     }
@@ -377,7 +435,7 @@ static __device__ __noinline__ double score_triple(const DevData& d, int w, int 
     if (d.objective == EPI4_OBJ_MI) {   // -M*I over the 27 cells (oracle mi_27's order)
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
-            const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+            const uint32_t r0 = cnt0(S[c], pks, pkm), r1 = cnt1(S[c], pks);
             kk = __dadd_rn(kk, __dsub_rn(__dadd_rn(__ldg(d.xlx + r0), __ldg(d.xlx + r1)), __ldg(d.xlx + (r0 + r1))));
         }
         return -__dadd_rn(kk, d.mi_const);
@@ -386,7 +444,7 @@ static __device__ __noinline__ double score_triple(const DevData& d, int w, int 
         if (d.np[0] == 0 || d.np[1] == 0) return 0.0;
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
-            const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks, rc = r0 + r1;
+            const uint32_t r0 = cnt0(S[c], pks, pkm), r1 = cnt1(S[c], pks), rc = r0 + r1;
             if (rc) {
                 const unsigned long long num = (unsigned long long)r0 * r0 * d.np[1] +
                                                (unsigned long long)r1 * r1 * d.np[0];
@@ -398,17 +456,18 @@ static __device__ __noinline__ double score_triple(const DevData& d, int w, int 
     }
 #pragma unroll
     for (int c = 0; c < 27; ++c) {
-        const uint32_t r0 = S[c] & pkm, r1 = S[c] >> pks;
+        const uint32_t r0 = cnt0(S[c], pks, pkm), r1 = cnt1(S[c], pks);
         kk = __dadd_rn(kk, __dsub_rn(__dsub_rn(__ldg(d.lgam + (r0 + r1 + 1)), __ldg(d.lgam + r0)), __ldg(d.lgam + r1)));
     }
     return kk;
 }
 
 // pack separate control / case counts (CUDA-core kernels)
+template <typename P = uint32_t>
 __device__ __forceinline__ void pack16(const DevData& d, const uint32_t (&c0)[16], const uint32_t (&c1)[16],
-                                       uint32_t (&c16)[16]) {
+                                       P (&c16)[16]) {
 #pragma unroll
-    for (int k = 0; k < 16; ++k) c16[k] = c0[k] | (c1[k] << d.pk_shift);
+    for (int k = 0; k < 16; ++k) c16[k] = (P)c0[k] | ((P)c1[k] << d.pk_shift);
 }
 
 // ---------------------------------------------------------------------------------------------

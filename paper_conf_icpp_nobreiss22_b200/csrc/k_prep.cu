@@ -226,6 +226,11 @@ cudaError_t launch_ones_plane(uint32_t* planes, int32_t n, int32_t npad, int32_t
 }
 
 // ---- lower-order tables ---------------------------------------------------------------------------
+// packed (control, case) word of the tables: c0 | c1 << pk_shift, 32 or (wide) 64 bits
+template <typename P>
+__device__ __forceinline__ P pkw(const DevData& d, uint32_t c0, uint32_t c1) { return (P)c0 | ((P)c1 << d.pk_shift); }
+
+template <typename P>
 __global__ void __launch_bounds__(256) k_pop1(DevData d, uint32_t* __restrict__ T1) {
     const int snp = blockIdx.x * blockDim.x + threadIdx.x;
     if (snp >= d.n) return;
@@ -237,7 +242,9 @@ __global__ void __launch_bounds__(256) k_pop1(DevData d, uint32_t* __restrict__ 
                 const uint4 v = __ldg(reinterpret_cast<const uint4*>(d.planes[p] + plane_off(kc, d.npad, snp, g, 0)));
                 c[p][g] += __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
             }
-    reinterpret_cast<uint2*>(T1)[snp] = make_uint2(c[0][0] | (c[1][0] << d.pk_shift), c[0][1] | (c[1][1] << d.pk_shift));
+    P* o = reinterpret_cast<P*>(T1) + (int64_t)snp * 2;
+    o[0] = pkw<P>(d, c[0][0], c[1][0]);
+    o[1] = pkw<P>(d, c[0][1], c[1][1]);
 }
 
 __device__ __forceinline__ void decode2(int64_t r, int& i, int& j) {
@@ -262,6 +269,7 @@ __device__ __forceinline__ void ld_planes(const DevData& d, int p, int kc, int s
     v[1][0] = b.x; v[1][1] = b.y; v[1][2] = b.z; v[1][3] = b.w;
 }
 
+template <typename P>
 __global__ void __launch_bounds__(256) k_pop2(DevData d, uint32_t* __restrict__ T2, int64_t npairs) {
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= npairs) return;
@@ -284,11 +292,12 @@ __global__ void __launch_bounds__(256) k_pop2(DevData d, uint32_t* __restrict__ 
 #pragma unroll
         for (int q = 0; q < 4; ++q) out[p][q] = c[q];
     }
-    const uint32_t s = (uint32_t)d.pk_shift;
-    reinterpret_cast<uint4*>(T2)[r] = make_uint4(out[0][0] | (out[1][0] << s), out[0][1] | (out[1][1] << s),
-                                                 out[0][2] | (out[1][2] << s), out[0][3] | (out[1][3] << s));
+    P* o = reinterpret_cast<P*>(T2) + r * 4;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) o[q] = pkw<P>(d, out[0][q], out[1][q]);
 }
 
+template <typename P>
 __global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ T3, int64_t lo, int64_t hi) {
     const int64_t r = lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= hi) return;
@@ -321,23 +330,23 @@ __global__ void __launch_bounds__(256) k_pop3(DevData d, uint32_t* __restrict__ 
 #pragma unroll
         for (int q = 0; q < 8; ++q) out[p][q] = c[q];
     }
-    const uint32_t s = (uint32_t)d.pk_shift;
-    uint4* o = reinterpret_cast<uint4*>(T3 + r * 8);
-    o[0] = make_uint4(out[0][0] | (out[1][0] << s), out[0][1] | (out[1][1] << s), out[0][2] | (out[1][2] << s),
-                      out[0][3] | (out[1][3] << s));
-    o[1] = make_uint4(out[0][4] | (out[1][4] << s), out[0][5] | (out[1][5] << s), out[0][6] | (out[1][6] << s),
-                      out[0][7] | (out[1][7] << s));
+    P* o = reinterpret_cast<P*>(T3) + r * 8;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) o[q] = pkw<P>(d, out[0][q], out[1][q]);
 }
 
 cudaError_t launch_pop(const DevData& d, uint32_t* T1, uint32_t* T2, uint32_t* T3, int64_t t3_lo, int64_t t3_hi,
                        cudaStream_t s, int64_t* launches) {
-    k_pop1<<<(d.n + 255) / 256, 256, 0, s>>>(d, T1);
+    if (d.wide) k_pop1<uint64_t><<<(d.n + 255) / 256, 256, 0, s>>>(d, T1);
+    else k_pop1<uint32_t><<<(d.n + 255) / 256, 256, 0, s>>>(d, T1);
     if (launches) ++*launches;
     const int64_t np2 = c2(d.n);
-    k_pop2<<<(unsigned)((np2 + 255) / 256), 256, 0, s>>>(d, T2, np2);
+    if (d.wide) k_pop2<uint64_t><<<(unsigned)((np2 + 255) / 256), 256, 0, s>>>(d, T2, np2);
+    else k_pop2<uint32_t><<<(unsigned)((np2 + 255) / 256), 256, 0, s>>>(d, T2, np2);
     if (launches) ++*launches;
     if (t3_hi > t3_lo) {   // the triples [t3_lo, t3_hi) of the colex order (all of them unless sharded)
-        k_pop3<<<(unsigned)((t3_hi - t3_lo + 255) / 256), 256, 0, s>>>(d, T3, t3_lo, t3_hi);
+        if (d.wide) k_pop3<uint64_t><<<(unsigned)((t3_hi - t3_lo + 255) / 256), 256, 0, s>>>(d, T3, t3_lo, t3_hi);
+        else k_pop3<uint32_t><<<(unsigned)((t3_hi - t3_lo + 255) / 256), 256, 0, s>>>(d, T3, t3_lo, t3_hi);
         if (launches) ++*launches;
     }
     return cudaGetLastError();

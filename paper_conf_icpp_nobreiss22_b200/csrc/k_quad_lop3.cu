@@ -110,14 +110,16 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
                     c1[c] = s_cnt[((1 * LOP3_Q + m) * 16 + c) * LOP3_THREADS + tid];
                 }
                 uint32_t* dump = sp.dump ? sp.dump + rank4(w, x, y, z) * 162 : nullptr;
-                uint32_t c16[16];
-                pack16(d, c0, c1, c16);
-                if (!dump && sample_hit(sp, pack_quad(w, x, y, z))) {
-                    key = sample_record(sp, w, x, y, z, c16);
-                } else {
-                    key = score_quad(d, w, x, y, z, c16, dump);
-                    if (dump && d.objective != EPI4_OBJ_K2) key = score_quad(d, w, x, y, z, c16, nullptr);
-                }
+                auto eval = [&](auto tag) {
+                    using P = decltype(tag);
+                    P c16[16];
+                    pack16<P>(d, c0, c1, c16);
+                    if (!dump && sample_hit(sp, pack_quad(w, x, y, z))) return sample_record<P>(sp, w, x, y, z, c16);
+                    double k = score_quad<P>(d, w, x, y, z, c16, dump);
+                    if (dump && d.objective != EPI4_OBJ_K2) k = score_quad<P>(d, w, x, y, z, c16, nullptr);
+                    return k;
+                };
+                key = d.wide ? eval(uint64_t{}) : eval(uint32_t{});
                 idx = pack_quad(w, x, y, z);
                 ++my_quads;
             }

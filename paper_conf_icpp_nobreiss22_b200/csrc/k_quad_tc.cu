@@ -372,8 +372,13 @@ __device__ long long g_trace[2][TR_EV][TR_STEPS];
 // multiples of MMA_WARPS, PROD_STRIDE and TMA_WARPS.
 // SMP: verification variants (dump / sample hooks compiled in); the production search has neither (their
 // per-quad checks cost ~3 % at C2 in registers and branches)
-template <int SA, int SB, bool PK16, int FILT, bool SMP>
+// WIDE: 64-bit packed counts (bits(n0) + bits(n1) > 32, epilogue.cuh): the (control, case) pair of a count no
+// longer fits one TMEM column, so there is no pack pass and no region rotation: tile t accumulates its controls
+// in region 0 and its cases in region 1, the epilogue reads both, and the next tile starts once it has (the
+// epilogue is a small share of a tile at the sample counts that need this mode).
+template <int SA, int SB, bool PK16, int FILT, bool SMP, bool WIDE>
 __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
+    using P = std::conditional_t<WIDE, uint64_t, uint32_t>;
     static_assert(tc::MMA_ISSUERS == 1 ||
                   (SA % 2 == 0 && SB % 2 == 0 && tc::MMA_WARPS == 2 && tc::PROD_STRIDE == 2 && tc::TMA_WARPS == 2),
                   "ring sizes must be multiples of the alternating warps' stride (phase aliasing)");
@@ -474,18 +479,22 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 const int buf = it & 1;
                 const long long te0 = PCLK();
                 // the p0 region held the packed counts of tile it - 2: both CTAs' epilogues are done with them
-                if (it >= 2) mbar_wait(&ep_bar[buf], (uint32_t)(((it >> 1) & 1) ^ 1));
+                if (WIDE) {          // both regions held tile it - 1
+                    if (it >= 1) mbar_wait(&ep_bar[(it - 1) & 1], (uint32_t)(((it - 1) >> 1) & 1));
+                } else if (it >= 2) {
+                    mbar_wait(&ep_bar[buf], (uint32_t)(((it >> 1) & 1) ^ 1));
+                }
                 t_tempty += PCLK() - te0;
                 tc_fence_after();
                 const int r1 = r0 == 2 ? 0 : r0 + 1;
 #pragma unroll 1
                 for (int p = 0; p < 2; ++p) {
-                    if (p == 1 && it >= 1) {
+                    if (!WIDE && p == 1 && it >= 1) {
                         // the p1 region held the controls of tile it - 1: its pack pass moved them out
                         mbar_wait(&pk_bar, (uint32_t)((it - 1) & 1));
                         tc_fence_after();
                     }
-                    const uint32_t dcol = tmem + (uint32_t)((p ? r1 : r0) * tc::N);
+                    const uint32_t dcol = tmem + (uint32_t)((WIDE ? p : (p ? r1 : r0)) * tc::N);
                     const int nch = p ? nch1_r : nch0_r;
 #pragma unroll 1
                     for (int kc = 0; kc < nch; ++kc, ++gstep) {
@@ -708,11 +717,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             tc_fence_after();
             const int w = (ti.wp * 2 + (int)rank) * EPI4_WR + wl;
             const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
-            const uint32_t R0 = tq + (uint32_t)(r0 * tc::N), R1 = tq + (uint32_t)(r1 * tc::N);
+            const uint32_t R0 = tq + (uint32_t)((WIDE ? 0 : r0) * tc::N), R1 = tq + (uint32_t)((WIDE ? 1 : r1) * tc::N);
             // pass 1: pack each (control, case) count pair into one 32-bit word, in place in the case region,
             // and zero the control region, which the next tile's case accumulation reuses
 #pragma unroll 1
-            for (int g = h; g < tc::NG; g += 2) {
+            for (int g = h; g < (WIDE ? 0 : tc::NG); g += 2) {
                 uint32_t v0[16], v1[16];
                 tmem_ld16(R0 + 16 * g, v0);
                 tmem_ld16(R1 + 16 * g, v1);
@@ -724,19 +733,33 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 tmem_st16(R1 + 16 * g, v1);                                              // the mantissa
                 tmem_zero16(R0 + 16 * g);
             }
-            tmem_wait_st();
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) {
-                if (leader) mbar_arrive_local(&pk_bar);
-                else mbar_arrive_cluster(&pk_bar, 0);   // the leader's barrier
+            if (!WIDE) {
+                tmem_wait_st();
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if (leader) mbar_arrive_local(&pk_bar);
+                    else mbar_arrive_cluster(&pk_bar, 0);   // the leader's barrier
+                }
             }
             // pass 2: score the quads from the packed counts
 #pragma unroll 1
             for (int g = h; g < tc::NG; g += 2) {
-                uint32_t v[16];
-                tmem_ld16(R1 + 16 * g, v);
-                tmem_wait_ld();
+                P v[16];
+                if constexpr (WIDE) {   // unpacked fp32 counts of both regions -> 64-bit packed words
+                    uint32_t v0[16], v1[16];
+                    tmem_ld16(R0 + 16 * g, v0);
+                    tmem_ld16(R1 + 16 * g, v1);
+                    tmem_wait_ld();
+                    tmem_zero16(R0 + 16 * g);
+#pragma unroll
+                    for (int k = 0; k < 16; ++k)
+                        v[k] = (uint64_t)(__float_as_uint(__uint_as_float(v0[k]) + 8388608.0f) & 0x7FFFFFu) |
+                               ((uint64_t)(__float_as_uint(__uint_as_float(v1[k]) + 8388608.0f) & 0x7FFFFFu) << 32);
+                } else {
+                    tmem_ld16(R1 + 16 * g, v);
+                    tmem_wait_ld();
+                }
                 tmem_zero16(R1 + 16 * g);                 // ready for a later tile's accumulation
                 if (g + 2 >= tc::NG) {
                     tmem_wait_st();
@@ -747,13 +770,13 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         else mbar_arrive_cluster(&ep_bar[buf], 0);   // the leader's barrier
                     }
                 }
-                uint32_t c16[16];
+                P c16[16];
 #pragma unroll
                 for (int k = 0; k < 8; ++k) {
                     // send my values for the other lane's quad, keep mine; lane a keeps c16[8a + k] = its own
                     // v[8a + k] and takes c16[8(1-a) + k] from the partner (packed control | case words)
-                    const uint32_t sv = a ? v[k] : v[8 + k];
-                    const uint32_t rv = __shfl_xor_sync(0xffffffffu, sv, 1);
+                    const P sv = a ? v[k] : v[8 + k];
+                    const P rv = __shfl_xor_sync(0xffffffffu, sv, 1);
                     c16[k] = a ? rv : v[k];
                     c16[8 + k] = a ? v[8 + k] : rv;
                 }
@@ -766,9 +789,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         const int64_t e = sp.t3_slab_w0 >= 0
                                               ? (int64_t)(w - sp.t3_slab_w0) * c2(d.n) + c2(y) + ti.x
                                               : rank3(w, ti.x, y);
-                        uint4* o = reinterpret_cast<uint4*>(sp.t3_out + e * 8);
-                        o[0] = make_uint4(c16[0], c16[2], c16[4], c16[6]);
-                        o[1] = make_uint4(c16[8], c16[10], c16[12], c16[14]);
+                        P* o = reinterpret_cast<P*>(sp.t3_out) + e * 8;
+#pragma unroll
+                        for (int k = 0; k < 8; ++k) o[k] = c16[2 * k];
                     }
                     continue;
                 }
@@ -778,8 +801,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     double key3 = 0.0;
                     uint64_t idx3 = 0;
                     if (v3) {
-                        const uint32_t c8[8] = {c16[0], c16[2], c16[4], c16[6], c16[8], c16[10], c16[12], c16[14]};
-                        key3 = score_triple(d, w, ti.x, y, c8);
+                        const P c8[8] = {c16[0], c16[2], c16[4], c16[6], c16[8], c16[10], c16[12], c16[14]};
+                        key3 = score_triple<P>(d, w, ti.x, y, c8);
                         idx3 = pack_quad(w, ti.x, y, 0);
                         ++my_quads;
                     }
@@ -794,18 +817,18 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     uint32_t* dump = SMP && sp.dump ? sp.dump + rank4(w, ti.x, y, ti.z) * 162 : nullptr;
                     offer = true;
                     if (SMP && dump) {
-                        key = score_quad_rare(d, w, ti.x, y, ti.z, c16, dump);
-                        if (d.objective != EPI4_OBJ_K2) key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
+                        key = score_quad_rare<P>(d, w, ti.x, y, ti.z, c16, dump);
+                        if (d.objective != EPI4_OBJ_K2) key = score_quad_rare<P>(d, w, ti.x, y, ti.z, c16, nullptr);
                     } else if (SMP && sample_hit(sp, pack_quad(w, ti.x, y, ti.z))) {
-                        key = sample_record_rare(sp, w, ti.x, y, ti.z, c16);
+                        key = sample_record_rare<P>(sp, w, ti.x, y, ti.z, c16);
                     } else if (sp.use_filter) {
                         // fp32 filter (epilogue.cuh); only possible top-k members get the exact score.
                         // FILT 0: Stirling K2 bound; FILT 1: chi-square upper bound (key = -X^2); FILT 2: MI
                         // upper bound (key = -M*I)
                         float flt;
                         double unused;
-                        quad_eval<FILT == 1 ? 5 : FILT == 2 ? 6 : 0, PK16>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y, ti.z, c16, flt,
-                                                           unused, nullptr);
+                        quad_eval<FILT == 1 ? 5 : FILT == 2 ? 6 : 0, PK16, P>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y,
+                                                                              ti.z, c16, flt, unused, nullptr);
                         const double thr = *reinterpret_cast<volatile double*>(tk.thr);
                         if (FILT == 1)
                             offer = d.chi_M - (double)flt * (1.0 + 1.0 / 4096.0) <= thr;
@@ -815,11 +838,11 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                             offer = (double)flt * 0.69314718055994530942 + d.flt_off <= thr;
                         if (offer) {
                             // rare path: the noinline exact scorer takes the counts through local memory
-                            key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
+                            key = score_quad_rare<P>(d, w, ti.x, y, ti.z, c16, nullptr);
                             ++n_exact;
                         }
                     } else {
-                        key = score_quad_rare(d, w, ti.x, y, ti.z, c16, nullptr);
+                        key = score_quad_rare<P>(d, w, ti.x, y, ti.z, c16, nullptr);
                     }
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;
@@ -862,9 +885,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
 #endif
 }
 
-template <int SA, int SB, bool PK16, int FILT, bool SMP>
+template <int SA, int SB, bool PK16, int FILT, bool SMP, bool WIDE = false>
 static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaStream_t s) {
-    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16, FILT, SMP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_quad_tc<SA, SB, PK16, FILT, SMP, WIDE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
@@ -878,7 +901,7 @@ static cudaError_t launch_cfg(SearchParams sp, size_t smem, int32_t grid, cudaSt
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16, FILT, SMP>, sp);
+    return cudaLaunchKernelEx(&cfg, k_quad_tc<SA, SB, PK16, FILT, SMP, WIDE>, sp);
 }
 
 // tiles per unit tile: the tensor-core kernel pairs the two 64-SNP halves of a 128-SNP w-range in one
@@ -917,11 +940,17 @@ cudaError_t launch_quad_tc(const SearchParams& sp_in, int32_t grid, cudaStream_t
     e = filt == 1 ? (pk16 ? launch_cfg<A_, B_, true, 1, SM_>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 1, SM_>(sp, smem, grid, s)) \
       : filt == 2 ? (pk16 ? launch_cfg<A_, B_, true, 2, SM_>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 2, SM_>(sp, smem, grid, s)) \
                   : (pk16 ? launch_cfg<A_, B_, true, 0, SM_>(sp, smem, grid, s) : launch_cfg<A_, B_, false, 0, SM_>(sp, smem, grid, s))
-#define EPI4_LAUNCH(A_, B_) do { if (smp) EPI4_LAUNCH_F(A_, B_, true); else EPI4_LAUNCH_F(A_, B_, false); } while (0)
+#define EPI4_LAUNCH_W(A_, B_, SM_)                                                                             \
+    e = filt == 1 ? launch_cfg<A_, B_, false, 1, SM_, true>(sp, smem, grid, s)                                 \
+      : filt == 2 ? launch_cfg<A_, B_, false, 2, SM_, true>(sp, smem, grid, s)                                 \
+                  : launch_cfg<A_, B_, false, 0, SM_, true>(sp, smem, grid, s)
+#define EPI4_LAUNCH(A_, B_) do { if (sp.d.wide) { if (smp) EPI4_LAUNCH_W(A_, B_, true); else EPI4_LAUNCH_W(A_, B_, false); } \
+                                 else if (smp) EPI4_LAUNCH_F(A_, B_, true); else EPI4_LAUNCH_F(A_, B_, false); } while (0)
     if (pick.sa == 4 && pick.sb == 4) EPI4_LAUNCH(4, 4);
     else if (pick.sa == 2 && pick.sb == 2) EPI4_LAUNCH(2, 2);
 #undef EPI4_LAUNCH
 #undef EPI4_LAUNCH_F
+#undef EPI4_LAUNCH_W
     if (launches) ++*launches;
     return e;
 }

@@ -115,11 +115,18 @@ __global__ void __launch_bounds__(128) k_tables(DevData d, const uint64_t* __res
     }
     uint32_t g[162];
     {
-        uint32_t c0[16], c1[16], c16[16];
+        uint32_t c0[16], c1[16];
         for (int c = 0; c < 16; ++c) { c0[c] = c4[0][c]; c1[c] = c4[1][c]; }
-        pack16(d, c0, c1, c16);
         uint32_t tmp[162];
-        (void)score_quad(d, s[0], s[1], s[2], s[3], c16, tmp);
+        if (d.wide) {
+            uint64_t c16[16];
+            pack16<uint64_t>(d, c0, c1, c16);
+            (void)score_quad<uint64_t>(d, s[0], s[1], s[2], s[3], c16, tmp);
+        } else {
+            uint32_t c16[16];
+            pack16<uint32_t>(d, c0, c1, c16);
+            (void)score_quad<uint32_t>(d, s[0], s[1], s[2], s[3], c16, tmp);
+        }
         for (int c = 0; c < 162; ++c) g[c] = tmp[c];
     }
     // sorted cell (digits for s[0..3]) -> cell in the given order: digit of given SNP t = digit[pos[t]]

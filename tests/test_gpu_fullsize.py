@@ -174,3 +174,28 @@ def test_uniform_genotypes_full_C2():
         idx, k2 = e.search(32)
     np.testing.assert_array_equal(idx, ref_idx)
     np.testing.assert_array_equal(k2, ref_k2)
+
+
+@pytest.mark.parametrize("pipe", ["tc", "lop3"])
+@pytest.mark.parametrize("n0,n1", [(91750, 39322), (262144, 262144)])
+def test_wide_counts_beyond_32_packed_bits(pipe, n0, n1):
+    """bits(n0) + bits(n1) > 32 (the C5 sweep's M = 131072 at 30/70; the paper's 2048 x 524288 shape):
+    64-bit packed counts through tables, contraction and epilogue.  Every quad's 2 x 81 table and the top-k
+    against the oracle on a 24-SNP window."""
+    from test_gpu_parity import all_quads
+    d = datagen.make_dataset(24, n0, n1, seed=n0 + 7, planted=(2, 9, 15, 21))
+    allq = all_quads(d.n_snps)
+    ref_idx, ref_k2 = oracle.search(d.geno, d.phen, top_k=128)
+    with _epi().Epi4(0, pipe=pipe) as e:
+        e.load_genotypes(d.geno, d.phen)
+        e.set_sample(0, 0, capacity=len(allq))
+        idx, k2 = e.search(128)
+        q, k, c, n = e.get_sample()
+        t = e.tables(pack(allq[:500]))
+    np.testing.assert_array_equal(idx, ref_idx)
+    np.testing.assert_array_equal(k2, ref_k2)
+    assert tuple(unpack(idx[:1])[0]) == (2, 9, 15, 21)
+    assert n == len(allq)
+    order = np.argsort(q)
+    _check_sample(d, q[order], k[order], c[order])
+    np.testing.assert_array_equal(t, oracle.tables(d.geno, d.phen, allq[:500]))
