@@ -1,0 +1,98 @@
+"""Clocked single-search records beside the bench line: every record carries the nvidia-smi clock
+summary of its own timed region (bench.ClockSampler: median SM clock, max clock, throttle reasons), so it can be
+judged like a bench line.
+
+  python tools/full_search.py --what C3,C4,sweep,paper [--slice-frac 0.1] [--out gpurun_out/full_search.jsonl]
+
+  C3, C4, C5, C2 : one full exhaustive search of the BASELINE.json config; reports the argmin against the planted
+                   quad (SURVEY.md §8(c) parity tier 3) and the top-16 keys, and the search's throughput
+                   (useful quads x M / kernel time, slab rebuilds included for the windowed C4)
+  sweep          : the C5 sample-count sweep (N = 1024, 30/70 cases/controls, M in {16384 .. 262144}; SURVEY.md
+                   §8(d)); M >= 131072 uses the 64-bit packed counts
+  paper          : the paper's best single-GPU shape, N = 2048 x M = 524288 balanced, on a
+                   slice of the plan (--slice-frac of its units, around the planted quad) - a full search is ~45 min
+Each point: one untimed warm-up search on C1, then load + search, timed by the library's CUDA events.
+"""
+import argparse
+import json
+import math
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import datagen  # noqa: E402
+import paper_conf_icpp_nobreiss22_b200 as epi  # noqa: E402
+from bench import ClockSampler, peaks  # noqa: E402
+
+
+def run_point(name, d, units=None, top_k=16):
+    """units: None (full search) or (begin, end) of the 1-rank plan"""
+    n, m = d.n_snps, d.n_samples
+    with epi.Epi4(0, pipe="tc") as e:
+        t0 = time.perf_counter()
+        e.load_genotypes(d.geno, d.phen)
+        t_load = time.perf_counter() - t0
+        with ClockSampler(0) as clk:
+            t0 = time.perf_counter()
+            idx, k2 = e.search(top_k) if units is None else e.search_units(units[0], units[1], top_k)
+            wall = time.perf_counter() - t0
+        st = e.stats()
+    pk, src = peaks()
+    q = st["quads"]
+    kern_s = st["ms_quad"] / 1e3
+    ach = 2.0 * 16.0 * q * m / kern_s / 1e12
+    best = epi.unpack_index(idx[0]) if len(idx) else None
+    return {"point": name, "n_snps": n, "m": m, "n_controls": d.n_controls, "n_cases": d.n_cases,
+            "units": "all" if units is None else f"plan units [{units[0]}, {units[1]})", "quads": q,
+            "full_quads": math.comb(n, 4),
+            "tquads_per_s_kernel": q * m / kern_s / 1e12, "tquads_per_s_search": q * m / wall / 1e12,
+            "kernel_ms": st["ms_quad"], "search_wall_s": wall, "load_s": t_load,
+            "roofline_frac": ach / (4.0 * pk["bf16_tflops_sustained"]),
+            "useful_over_executed": q * 16.0 * m / st["executed_macs"] if st["executed_macs"] else None,
+            "best": {"quad": best, "k2": float(k2[0]) if len(k2) else None}, "planted": d.planted,
+            "planted_is_argmin": d.planted is not None and best == tuple(d.planted),
+            "top16": [[epi.unpack_index(i), float(k)] for i, k in zip(idx, k2)],
+            "clocks": clk.summary(), "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime())}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--what", default="C3,sweep")
+    ap.add_argument("--slice-frac", type=float, default=0.1)
+    ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "full_search.jsonl"))
+    a = ap.parse_args()
+    os.makedirs(os.path.dirname(a.out), exist_ok=True)
+    with epi.Epi4(0, pipe="tc") as e:   # warm-up (module load, first-launch costs)
+        c1 = datagen.make_config("C1")
+        e.load_genotypes(c1.geno, c1.phen)
+        e.search(4)
+    todo = []
+    for w in a.what.split(","):
+        if w == "sweep":
+            for m in (16384, 32768, 65536, 100003, 131072, 262144):
+                n1 = int(round(0.3 * m))
+                todo.append((f"C5-sweep M={m}", lambda m=m, n1=n1: datagen.make_dataset(
+                    1024, m - n1, n1, 2000 + m, planted=datagen.planted_quad_for(1024), name=f"sweep{m}"), None))
+        elif w == "paper":
+            # a contiguous slice of the LPT plan around the planted quad's unit (units of similar cost, every w-range)
+            units, _ = epi.binding.epi4_plan_units(2048, 0, 1)
+            pq = datagen.planted_quad_for(2048)
+            u0 = int([i for i, (wr, x) in enumerate(units.tolist()) if wr == pq[0] // 128 and x == pq[1]][0])
+            k = int(len(units) * a.slice_frac)
+            lo = max(0, u0 - k // 2)
+            todo.append((f"paper shape N=2048 M=524288 ({a.slice_frac:.0%} of the plan around the planted quad)",
+                         lambda: datagen.make_dataset(2048, 262144, 262144, 3001, planted=pq, name="paper2048x524288"),
+                         (lo, min(len(units), lo + k))))
+        else:
+            todo.append((w, lambda w=w: datagen.make_config(w), None))
+    with open(a.out, "a") as f:
+        for name, mk, units in todo:
+            r = run_point(name, mk(), units)
+            print(json.dumps(r), flush=True)
+            f.write(json.dumps(r) + "\n")
+
+
+if __name__ == "__main__":
+    main()
