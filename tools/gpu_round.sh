@@ -10,5 +10,5 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -3
 timeout 1500 python bench.py --steps 5 --warmup 3 > gpurun_out/${T}_bench.json 2> gpurun_out/${T}_bench.err; tail -c 1500 gpurun_out/${T}_bench.json; tail -5 gpurun_out/${T}_bench.err
 timeout 900 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${T}_bench_ref.json 2>&1; tail -c 800 gpurun_out/${T}_bench_ref.json
 timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${T}_launches.csv python bench.py --also none --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/${T}_ncu_launches_bench.log 2>&1; tail -2 gpurun_out/${T}_ncu_launches_bench.log
-timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_quad_tc --launch-skip 1 -c 1 -o gpurun_out/${T}_full_C5slice -f python tools/run_search.py --config C5 --units 100 > gpurun_out/${T}_ncu_full_c5.log 2>&1; tail -2 gpurun_out/${T}_ncu_full_c5.log
+timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_quad_tc --launch-skip 1 -c 1 -o gpurun_out/${T}_full_C5slice -f python tools/run_search.py --config C5 --units 12 > gpurun_out/${T}_ncu_full_c5.log 2>&1; tail -2 gpurun_out/${T}_ncu_full_c5.log
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_quad_tc --launch-skip 1 -c 1 -o gpurun_out/${T}_full_C2slice -f python tools/run_search.py --config C2 --units 300 > gpurun_out/${T}_ncu_full_c2.log 2>&1; tail -2 gpurun_out/${T}_ncu_full_c2.log
