@@ -151,7 +151,8 @@ def measure(cfg, args, world, rank, local, torch, dist, epi):
     # N > 1: every rank builds the 3-way table on its tensor cores (~3 ms at C2, tiny next to the search);
     # --shard-t3 instead builds 1/world of it per rank (POPC kernel) and all-gathers the shares over NCCL
     shard = world > 1 and args.shard_t3
-    eng = epi.Epi4(local, pipe=args.pipe, rank=rank, world=world, shard_t3=shard, objective=args.objective)
+    eng = epi.Epi4(local, pipe=args.pipe, rank=rank, world=world, shard_t3=shard, objective=args.objective,
+                   tile=None if args.tile == "auto" else int(args.tile))
     eng.set_stream(stream.cuda_stream)
     geno_d = torch.from_numpy(d.geno).to(f"cuda:{local}")
     phen_d = torch.from_numpy(d.phen).to(f"cuda:{local}")
@@ -250,6 +251,7 @@ def measure(cfg, args, world, rank, local, torch, dist, epi):
         "config": {"workload": f"{cfg}: N={n} SNPs, M={m} samples ({d.n_controls} controls / "
                                f"{d.n_cases} cases), exhaustive C(N,4)={comb4(n)} quads, top_k={top_k}",
                    "pipe": args.pipe, "objective": args.objective,
+                   "tile_n": int(st.get("tile_n", 0)),
                    "parallelism": f"static LPT over (w-block, x) units x {world} ranks (NCCL world {world})" +
                                   (", T3 sharded + NCCL all_gather" if shard else ""),
                    "l2": "flushed (512 MiB write) before every timed step"},
@@ -373,6 +375,8 @@ def main():
                     "(none to skip)")
     ap.add_argument("--pipe", default="tc", choices=["tc", "lop3"])
     ap.add_argument("--top-k", type=int, default=16)
+    ap.add_argument("--tile", default="auto", choices=["auto", "128", "224"],
+                    help="tensor-core tile geometry (default: chosen by the load from the sample counts)")
     ap.add_argument("--objective", default="k2", choices=["k2", "mi", "chi2"],
                     help="ranking objective (K2 is the paper's and the headline; MI / chi-square: SURVEY §8(f) NEXT-4)")
     ap.add_argument("--no-cpu-baseline", action="store_true")

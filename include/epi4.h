@@ -66,6 +66,12 @@ typedef struct {
  * chosen automatically when the resident table does not fit in HBM (e.g. N = 4096), forced by this flag.
  * epi4_tables is unavailable (EPI4_ESTATE) with a windowed table. */
 #define EPI4_FLAG_T3_WINDOWED 2
+/* opts.flags: tensor-core tile geometry.  By default a load picks N = 224 columns per tile
+ * (28 y SNPs; the A operand amortised over more columns, two TMEM accumulator regions) when the dataset has
+ * >= 24576 controls or needs 64-bit packed counts, else N = 128 (16 y, three regions, the scoring overlaps
+ * both phenotype phases); these flags force one (results are identical, only the speed differs). */
+#define EPI4_FLAG_TILE_N128 4
+#define EPI4_FLAG_TILE_N224 8
 
 /* opts.objective (the table construction does not depend on the score):
  *   EPI4_OBJ_K2: K2 (the paper's), smallest first.
@@ -204,6 +210,7 @@ typedef struct {
                               [2] MMA waiting for the A operand, [3] producer busy, [4] producer waiting for a
                               free B stage, [5] MMA waiting for the B operand, [6] TMA waiting for a free A
                               stage, [7] MMA waiting for a free TMEM region */
+    int64_t tile_n;        /* last search: columns per tensor-core tile (128 or 224, EPI4_FLAG_TILE_*); 0 = lop3 */
 } epi4_stats;
 
 int epi4_get_stats(epi4_ctx* ctx, epi4_stats* out);

@@ -29,12 +29,16 @@ class Epi4:
     """One search context on one GPU (one per rank)."""
 
     def __init__(self, device: int = 0, pipe: str = "tc", rank: int = 0, world: int = 1, grid: int = 0,
-                 debug: int = 0, shard_t3: bool = False, t3_windowed: bool = False, objective: str = "k2"):
+                 debug: int = 0, shard_t3: bool = False, t3_windowed: bool = False, objective: str = "k2",
+                 tile: int | None = None):
         o = binding.epi4_default_opts()
         o.pipe = binding.PIPES[pipe]
         o.rank, o.world, o.grid = int(rank), int(world), int(grid)
         o.debug = int(debug)           # diagnostics only: disables warp roles, results invalid
         o.flags = (binding.EPI4_FLAG_SHARD_T3 if shard_t3 else 0) | (binding.EPI4_FLAG_T3_WINDOWED if t3_windowed else 0)
+        if tile not in (None, 128, 224):
+            raise ValueError("tile must be None (chosen by the load), 128 or 224")
+        o.flags |= {None: 0, 128: binding.EPI4_FLAG_TILE_N128, 224: binding.EPI4_FLAG_TILE_N224}[tile]
         o.objective = {"k2": binding.EPI4_OBJ_K2, "mi": binding.EPI4_OBJ_MI,
                        "chi2": binding.EPI4_OBJ_CHI2}[objective]
         self.shard_t3 = bool(shard_t3) and int(world) > 1

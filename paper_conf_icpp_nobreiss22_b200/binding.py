@@ -22,6 +22,8 @@ EPI4_PIPE_TC, EPI4_PIPE_LOP3 = 0, 1
 EPI4_PTR_HOST, EPI4_PTR_DEVICE = 0, 1
 EPI4_FLAG_SHARD_T3 = 1
 EPI4_FLAG_T3_WINDOWED = 2
+EPI4_FLAG_TILE_N128 = 4
+EPI4_FLAG_TILE_N224 = 8
 EPI4_OBJ_K2, EPI4_OBJ_MI, EPI4_OBJ_CHI2 = 0, 1, 2
 EPI4_MAX_TOPK = 1024
 PIPES = {"tc": EPI4_PIPE_TC, "lop3": EPI4_PIPE_LOP3}
@@ -43,7 +45,7 @@ class epi4_stats(ctypes.Structure):
     _fields_ = [("ms_pack", ctypes.c_double), ("ms_pop", ctypes.c_double), ("ms_quad", ctypes.c_double),
                 ("ms_merge", ctypes.c_double), ("quads", ctypes.c_int64), ("tiles", ctypes.c_int64),
                 ("launches", ctypes.c_int64), ("launches_load", ctypes.c_int64),
-                ("executed_macs", ctypes.c_double), ("prof", ctypes.c_double * 8)]
+                ("executed_macs", ctypes.c_double), ("prof", ctypes.c_double * 8), ("tile_n", ctypes.c_int64)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_}

@@ -69,6 +69,7 @@ struct SearchPlan {
     int32_t n = 0, rank = 0, world = 0, pipe = -1;
     int64_t ub = 0, ue = 0;
     bool windowed = false;
+    int32_t yr = 0;                     // y-range of the tiles the prefix counts
     std::vector<Unit> units;
     std::vector<int64_t> prefix;        // group-relative inclusive prefix of tiles per unit
     std::vector<Group> groups;
@@ -87,6 +88,7 @@ struct epi4_ctx {
     int32_t n = 0, npad = 0;
     int64_t np[2] = {0, 0};
     int32_t nchunks[2] = {0, 0};
+    int32_t tc_yr = EPI4_YR_N128;  // tensor-core tile geometry of this dataset (y per tile: N = 8 tc_yr; tc_tile_yr)
     uint32_t* planes[2] = {nullptr, nullptr};
     uint32_t *T1 = nullptr, *T2 = nullptr, *T3 = nullptr;
     uint32_t* T3x = nullptr;       // windowed T3: the slab FIRST(X) (T3 then holds FIRST(R))
@@ -175,8 +177,6 @@ DevData devdata(const epi4_ctx* c) {
     d.nchunks[1] = c->nchunks[1];
     d.nchunks4[0] = (c->nchunks[0] + 1) / 2;
     d.nchunks4[1] = (c->nchunks[1] + 1) / 2;
-    d.nsteps[0] = (d.nchunks4[0] + 1) / 2;
-    d.nsteps[1] = (d.nchunks4[1] + 1) / 2;
     d.nrb = c->npad / 64;
     // c0 <= n0 < 2^pk_shift; 16 whenever both counts fit 16 bits (the epilogue then unpacks each half into a
     // float with one byte permute, epilogue.cuh cell_T_acc<true>)
@@ -334,7 +334,7 @@ int ensure_lists(epi4_ctx* c, int32_t slots, int32_t cap) {
 int prepare_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t G, int32_t YR) {
     SearchPlan& pl = c->plan;
     if (pl.valid && pl.n == c->n && pl.rank == c->opts.rank && pl.world == c->opts.world && pl.pipe == c->opts.pipe &&
-        pl.windowed == c->t3_windowed && pl.ub == ub && pl.ue == ue)
+        pl.windowed == c->t3_windowed && pl.ub == ub && pl.ue == ue && pl.yr == YR)
         return 0;
     pl.valid = false;
     pl.table_cached = false;
@@ -395,6 +395,7 @@ int prepare_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t G, int32_t YR) {
     pl.windowed = c->t3_windowed;
     pl.ub = ub;
     pl.ue = ue;
+    pl.yr = YR;
     pl.valid = true;
     return 0;
 }
@@ -409,14 +410,14 @@ size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * s
 int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) {
     const int32_t n = c->n;
     // the tile list depends only on (N, slab): the resident list is kept on the device across loads of the same N
-    const int64_t key = (int64_t)n * 2 + (slab_w0 >= 0 ? 1 : 0);
+    const int64_t key = ((int64_t)n * 2 + (slab_w0 >= 0 ? 1 : 0)) * 64 + c->tc_yr;
     if (slab_w0 >= 0 || c->t3_tiles_key != key) {
         std::vector<uint64_t>& tiles = c->host_tiles;
         tiles.clear();
         for (int32_t x = 1; x <= n - 2; ++x)
             for (int32_t wp = 0; wp * EPI4_WP < x; ++wp) {
                 if (slab_w0 >= 0 && wp * EPI4_WP != slab_w0) continue;
-                for (int32_t y0 = x + 1; y0 <= n - 1; y0 += EPI4_YR_TC)
+                for (int32_t y0 = x + 1; y0 <= n - 1; y0 += c->tc_yr)
                     tiles.push_back((uint64_t)(uint16_t)wp | ((uint64_t)(uint16_t)x << 16) |
                                     ((uint64_t)(uint16_t)y0 << 32) | ((uint64_t)(uint16_t)n << 48));
             }
@@ -435,6 +436,7 @@ int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) 
     if (int r = ensure_lists(c, grid, 1)) return r;
     SearchParams sp{};
     sp.d = devdata(c);
+    sp.yr = c->tc_yr;
     sp.tile_info = c->d_tiles3;
     sp.ntiles = c->t3_tiles_n;
     sp.t3_out = out;
@@ -574,12 +576,25 @@ extern "C" int epi4_t3_ready(epi4_ctx* c) {
 
 namespace {
 
+// Tensor-core tile geometry (k_quad_tc.cuh): N = 224 columns amortise the A operand over 1.75x the
+// columns but leave room for only two TMEM regions, so the scoring of a tile overlaps only the first (control)
+// phase of the next; N = 128 keeps three regions.  Measured on one B200 (profiles/r02f_variants.log,
+// r02g_geom_ab.log): N = 224 is 7 % faster on the full C5 search (70002 controls), within noise with 16384
+// controls (C3 sub-window) and 17 % slower with 8192 (C2).  The wide (64-bit packed) mode has two regions in
+// both geometries.  opts.flags can force either.
+int32_t tc_tile_yr(int32_t flags, int64_t n0, int64_t n1) {
+    if (flags & EPI4_FLAG_TILE_N224) return EPI4_YR_N224;
+    if (flags & EPI4_FLAG_TILE_N128) return EPI4_YR_N128;
+    return (n0 >= 24576 || is_wide(n0, n1)) ? EPI4_YR_N224 : EPI4_YR_N128;
+}
+
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
     c->loaded = false;
     c->n = n;
-    c->npad = (n + EPI4_YR + EPI4_WP - 1) / EPI4_WP * EPI4_WP;   // rows past n read as zero planes
+    c->npad = (n + EPI4_YR_MAX + EPI4_WP - 1) / EPI4_WP * EPI4_WP;   // rows past n read as zero planes
     c->np[0] = n0;
     c->np[1] = n1;
+    c->tc_yr = tc_tile_yr(c->opts.flags, n0, n1);
     for (int p = 0; p < 2; ++p) {
         c->nchunks[p] = (int32_t)((c->np[p] + EPI4_CHUNK_SAMPLES - 1) / EPI4_CHUNK_SAMPLES);
         const size_t words = (size_t)c->nchunks[p] * c->npad * 2 * EPI4_CHUNK_WORDS;
@@ -898,7 +913,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     if (c->opts.pipe != EPI4_PIPE_LOP3 && std::max(c->np[0], c->np[1]) > ((int64_t)1 << 24))
         return fail(EPI4_EINVAL, "tensor-core pipe: fp32 accumulators are exact up to 2^24 samples per phenotype "
                                  "(%lld, %lld); use EPI4_PIPE_LOP3", (long long)c->np[0], (long long)c->np[1]);
-    const int32_t G = quad_split(c->opts.pipe), YR = quad_yr(c->opts.pipe);
+    const int32_t G = quad_split(c->opts.pipe), YR = c->opts.pipe == EPI4_PIPE_LOP3 ? EPI4_YR : c->tc_yr;
     if (int r = prepare_units(c, ub, ue, G, YR)) return r;
     const SearchPlan& pl = c->plan;
     int32_t grid = c->opts.grid > 0 ? c->opts.grid : c->sm_count;
@@ -910,6 +925,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
 
     SearchParams sp{};
     sp.d = devdata(c);
+    sp.yr = c->tc_yr;
     sp.t3_slab_w0 = -1;
     sp.tile_counter = c->d_counters;
     sp.topk = top_k;
@@ -1001,12 +1017,14 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
     for (int i = 0; i < 8; ++i) c->stats.prof[i] = (double)ctr[16 + i];
     c->stats.tiles = acc / G;
     // MACs the contraction executes: 256 (w, a) rows (a 128-SNP w-range) x 8 YR columns per unit tile and
-    // sample; the tensor-core operands run over whole 512-sample steps (two fp4 chunks, zero-padded), the
-    // CUDA-core kernel over 128-sample chunks
+    // sample; the tensor-core operands run over whole steps (tc_chunks(yr) fp4 chunks of 256 samples,
+    // zero-padded), the CUDA-core kernel over 128-sample chunks
     const double ksamples = c->opts.pipe == EPI4_PIPE_LOP3
                                 ? (double)(c->nchunks[0] + c->nchunks[1]) * EPI4_CHUNK_SAMPLES
-                                : (double)(sp.d.nsteps[0] + sp.d.nsteps[1]) * 512.0;
+                                : (double)(tc_steps(sp.d.nchunks4[0], c->tc_yr) + tc_steps(sp.d.nchunks4[1], c->tc_yr)) * 256.0 *
+                                      tc_chunks(c->tc_yr);
     c->stats.executed_macs = (double)(acc / G) * 256.0 * 8.0 * YR * ksamples;
+    c->stats.tile_n = c->opts.pipe == EPI4_PIPE_LOP3 ? 0 : 8 * YR;
     *n_out = nout;
     return 0;
 }
@@ -1025,7 +1043,7 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     std::vector<uint64_t>& tiles = c->host_tiles;
     tiles.clear();
     auto add = [&](int32_t wr, int32_t x) {
-        for (int32_t y0 = x + 1; y0 <= c->n - 1; y0 += EPI4_YR_TC)
+        for (int32_t y0 = x + 1; y0 <= c->n - 1; y0 += c->tc_yr)
             tiles.push_back((uint64_t)(uint16_t)wr | ((uint64_t)(uint16_t)x << 16) | ((uint64_t)(uint16_t)y0 << 32) |
                             ((uint64_t)(uint16_t)c->n << 48));
     };
@@ -1040,6 +1058,7 @@ int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_o
     CU(cudaMemsetAsync(c->d_counters, 0, 32 * sizeof(unsigned long long), c->stream));
     SearchParams sp{};
     sp.d = devdata(c);
+    sp.yr = c->tc_yr;
     sp.t3_slab_w0 = -1;
     sp.search3 = 1;
     sp.topk = top_k;

@@ -25,9 +25,21 @@
 #define EPI4_WR 64            // w-range of one CTA / rows of its A operand: 64 SNPs x {AA, Aa}
 #define EPI4_WP 128           // w-range of a work unit (a CTA pair: two 64-SNP halves)
 #define EPI4_YR 16            // y-range of a CUDA-core (LOP3) tile: 16 consecutive SNPs after x
-#ifndef EPI4_YR_TC
-#define EPI4_YR_TC 16         // y-range of a tensor-core tile (N = 128 = 16 x 8 columns; measured best, k_quad_tc.cu)
+// tensor-core tile geometries (k_quad_tc.cuh Geom128 / Geom224): y-range of a tile (8 columns per y) and fp4
+// chunks per pipeline step (overridable for diagnostics builds only)
+#ifndef EPI4_YR_N128
+#define EPI4_YR_N128 16
 #endif
+#ifndef EPI4_CH_N128
+#define EPI4_CH_N128 2
+#endif
+#ifndef EPI4_YR_N224
+#define EPI4_YR_N224 28
+#endif
+#ifndef EPI4_CH_N224
+#define EPI4_CH_N224 1
+#endif
+#define EPI4_YR_MAX 32        // SNP rows a tile may read past its y0 (planes are zero-padded that far)
 #define EPI4_CHUNK_WORDS 4    // 128 samples per chunk
 #define EPI4_CHUNK_SAMPLES 128
 
@@ -39,6 +51,12 @@
 #define EPI4_ST_TOPK_OVF  16u
 
 namespace epi4 {
+
+// fp4 chunks (256 samples) per tensor-core pipeline step of a geometry, and the steps of a phenotype
+__host__ __device__ __forceinline__ int32_t tc_chunks(int32_t yr) { return yr == EPI4_YR_N224 ? EPI4_CH_N224 : EPI4_CH_N128; }
+__host__ __device__ __forceinline__ int32_t tc_steps(int32_t nchunks4, int32_t yr) {
+    return (nchunks4 + tc_chunks(yr) - 1) / tc_chunks(yr);
+}
 
 __host__ __device__ __forceinline__ int64_t c2(int64_t n) { return n * (n - 1) / 2; }
 __host__ __device__ __forceinline__ int64_t c3(int64_t n) { return n * (n - 1) * (n - 2) / 6; }
@@ -58,7 +76,6 @@ struct DevData {
     const uint32_t* planes[2];   // chunked planes per phenotype
     int32_t nchunks[2];          // 128-sample chunks per phenotype
     int32_t nchunks4[2];         // 256-sample fp4 chunks per phenotype (rows of expl)
-    int32_t nsteps[2];           // tensor-core pipeline steps per phenotype: pairs of fp4 chunks (512 samples)
     int32_t nrb;                 // 128-row blocks of expl per chunk (= npad / 64)
     int32_t pk_shift;            // (control, case) counts packed as c0 | c1 << pk_shift everywhere (bits(n0))
     int32_t wide;                // 1: packed words are 64-bit (pk_shift = 32) because bits(n0) + bits(n1) > 32
@@ -100,7 +117,7 @@ __host__ __device__ __forceinline__ int64_t plane_off(int64_t kc, int32_t npad, 
 
 // A work unit (wp, x): the quads (w, x, y, z) with w in the 128-SNP range [128 wp, 128 wp + 128), w < x,
 // second SNP x, and any x < y < z < n.  Its tiles are (y0, z): y in [y0, y0 + yr) with y0 = x + 1 + yr k,
-// and z in (y0, n); a tile holds 128 x yr (w, y) combinations (yr = EPI4_YR_TC tensor core, EPI4_YR CUDA core), split into
+// and z in (y0, n); a tile holds 128 x yr (w, y) combinations (yr = EPI4_YR_N128 / EPI4_YR_N224 tensor core, EPI4_YR CUDA core), split into
 // the two 64-SNP halves of the w-range (the two CTAs of a tensor-core cluster, or two tiles of the CUDA-core
 // kernel).
 struct Unit {
@@ -140,6 +157,7 @@ __device__ __forceinline__ int64_t find_unit(const int64_t* prefix, int64_t nuni
 // Per-search launch parameters common to the contraction kernels.
 struct SearchParams {
     DevData d;
+    int32_t yr;                // tensor-core pipe: y-range of a tile = the geometry (EPI4_YR_N128 / EPI4_YR_N224)
     const Unit* units;
     const int64_t* prefix;     // inclusive prefix of tiles per unit
     const uint64_t* tile_info; // (tensor-core pipe) decoded tiles: wp | x << 16 | y0 << 32 | z << 48 (k_tile_table)
@@ -206,7 +224,6 @@ cudaError_t launch_quad_tc(const SearchParams& sp, int32_t grid, cudaStream_t s,
 cudaError_t launch_tile_table(const SearchParams& sp, int64_t t0, int64_t t1, uint64_t* out, cudaStream_t s,
                               int64_t* launches);
 int32_t quad_split(int32_t pipe);   // tiles per unit tile (CUDA-core kernel: the two 64-SNP halves)
-int32_t quad_yr(int32_t pipe);      // y-range of a tile
 cudaError_t launch_merge(const SearchParams& sp, int32_t nlists, double* out_k2, uint64_t* out_idx,
                          int32_t* out_n, cudaStream_t s, int64_t* launches);
 cudaError_t launch_tables(const DevData& d, const uint64_t* quads, int64_t n, uint32_t* out, unsigned int* status,

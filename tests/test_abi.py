@@ -96,6 +96,7 @@ def test_binding_constants_match_the_header():
     hdr = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include", "epi4.h")).read()
     defs = {m.group(1): int(m.group(2), 0) for m in re.finditer(r"#define\s+(EPI4_\w+)\s+\(?(-?(?:0x)?[0-9A-Fa-f]+)\)?", hdr)}
     for name in ("EPI4_OBJ_K2", "EPI4_OBJ_MI", "EPI4_OBJ_CHI2", "EPI4_FLAG_SHARD_T3", "EPI4_FLAG_T3_WINDOWED",
+                 "EPI4_FLAG_TILE_N128", "EPI4_FLAG_TILE_N224",
                  "EPI4_EINVAL", "EPI4_ENODEV", "EPI4_PIPE_TC", "EPI4_PIPE_LOP3"):
         assert name in defs, name
         assert getattr(binding, name) == defs[name], name

@@ -131,13 +131,14 @@ def _worst_case(n=40, n0=70002, n1=30001, seed=9):
     return datagen.Dataset(geno=g, phen=d.phen, n_controls=n0, n_cases=n1, planted=None, seed=seed, name="worst")
 
 
-@pytest.mark.parametrize("pipe", ["tc", "lop3"])
+@pytest.mark.parametrize("pipe", ["tc", "tc128", "lop3"])   # tc: N = 224 is picked for 70002 controls
 def test_worst_case_all_samples_in_one_cell(pipe):
     from test_gpu_parity import all_quads
     d = _worst_case()
     allq = all_quads(d.n_snps)
     ref_idx, ref_k2 = oracle.search(d.geno, d.phen, top_k=256)
-    with _epi().Epi4(0, pipe=pipe) as e:
+    from test_gpu_parity import _engine
+    with _engine(pipe) as e:
         e.load_genotypes(d.geno, d.phen)
         e.set_sample(0, 0, capacity=len(allq))          # every quad
         idx, k2 = e.search(256)
@@ -176,7 +177,7 @@ def test_uniform_genotypes_full_C2():
     np.testing.assert_array_equal(k2, ref_k2)
 
 
-@pytest.mark.parametrize("pipe", ["tc", "lop3"])
+@pytest.mark.parametrize("pipe", ["tc", "tc128", "lop3"])   # tc: N = 224 is picked for wide counts
 @pytest.mark.parametrize("n0,n1", [(91750, 39322), (262144, 262144)])
 def test_wide_counts_beyond_32_packed_bits(pipe, n0, n1):
     """bits(n0) + bits(n1) > 32 (the C5 sweep's M = 131072 at 30/70; the paper's 2048 x 524288 shape):
@@ -186,7 +187,8 @@ def test_wide_counts_beyond_32_packed_bits(pipe, n0, n1):
     d = datagen.make_dataset(24, n0, n1, seed=n0 + 7, planted=(2, 9, 15, 21))
     allq = all_quads(d.n_snps)
     ref_idx, ref_k2 = oracle.search(d.geno, d.phen, top_k=128)
-    with _epi().Epi4(0, pipe=pipe) as e:
+    from test_gpu_parity import _engine
+    with _engine(pipe) as e:
         e.load_genotypes(d.geno, d.phen)
         e.set_sample(0, 0, capacity=len(allq))
         idx, k2 = e.search(128)

@@ -15,7 +15,8 @@ import oracle
 
 pytestmark = pytest.mark.gpu
 
-PIPES = ["lop3", "tc"]
+PIPES = ["lop3", "tc", "tc224"]   # tc: the tile geometry the load picks (N = 128 for these sample counts)
+PIPES_GEOM = ["lop3", "tc128", "tc224"]   # both tensor-core geometries forced
 
 
 def _epi():
@@ -24,6 +25,10 @@ def _epi():
 
 
 def _engine(pipe="tc", **kw):
+    """pipe: lop3, tc (geometry chosen by the load), tc128 / tc224 (geometry forced, opts.flags)"""
+    if pipe in ("tc128", "tc224"):
+        kw["tile"] = int(pipe[2:])
+        pipe = "tc"
     return _epi().Epi4(0, pipe=pipe, **kw)
 
 
@@ -210,7 +215,7 @@ def _subwindow_ref(cfg):
     return d, idx, k2
 
 
-@pytest.mark.parametrize("pipe", PIPES)
+@pytest.mark.parametrize("pipe", PIPES_GEOM)
 @pytest.mark.parametrize("cfg", ["C2", "C3", "C4", "C5"])
 def test_subwindow_full_samples(cfg, pipe):
     """First W SNPs of the config's dataset with all M samples (ragged 100003 in C5)."""

@@ -50,7 +50,7 @@ def run_point(name, d, units=None, top_k=16):
             "tquads_per_s_kernel": q * m / kern_s / 1e12, "tquads_per_s_search": q * m / wall / 1e12,
             "kernel_ms": st["ms_quad"], "search_wall_s": wall, "load_s": t_load,
             "roofline_frac": ach / (4.0 * pk["bf16_tflops_sustained"]),
-            "useful_over_executed": q * 16.0 * m / st["executed_macs"] if st["executed_macs"] else None,
+            "tile_n": st["tile_n"], "useful_over_executed": q * 16.0 * m / st["executed_macs"] if st["executed_macs"] else None,
             "best": {"quad": best, "k2": float(k2[0]) if len(k2) else None}, "planted": d.planted,
             "planted_is_argmin": d.planted is not None and best == tuple(d.planted),
             "top16": [[epi.unpack_index(i), float(k)] for i, k in zip(idx, k2)],

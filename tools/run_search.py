@@ -17,10 +17,11 @@ ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--debug", type=int, default=0)
 ap.add_argument("--grid", type=int, default=0)
 ap.add_argument("--objective", default="k2", choices=["k2", "mi", "chi2"])
+ap.add_argument("--tile", type=int, default=None, help="force the tensor-core tile geometry (128 / 224)")
 ap.add_argument("--n-snps", type=int, default=None, help="first N SNPs of the config's dataset (all M samples)")
 a = ap.parse_args()
 d = datagen.make_config(a.config, n_snps=a.n_snps)
-with epi.Epi4(0, pipe=a.pipe, debug=a.debug, grid=a.grid, objective=a.objective) as e:
+with epi.Epi4(0, pipe=a.pipe, debug=a.debug, grid=a.grid, objective=a.objective, tile=a.tile) as e:
     e.load_genotypes(d.geno, d.phen)
     for _ in range(a.repeat):
         t0 = time.time()
@@ -28,4 +29,4 @@ with epi.Epi4(0, pipe=a.pipe, debug=a.debug, grid=a.grid, objective=a.objective)
         st = e.stats()
         best = (epi.unpack_index(idx[0]), float(k2[0])) if len(idx) else None
         print(f"{a.config} {a.pipe} {a.objective} dbg={a.debug}: best {best} quad {st['ms_quad']:.2f} ms "
-              f"tiles {st['tiles']} quads {st['quads']} wall {time.time() - t0:.2f}s prof {[f'{v:.3g}' for v in st['prof']]}", flush=True)
+              f"N {st['tile_n']} tiles {st['tiles']} quads {st['quads']} wall {time.time() - t0:.2f}s prof {[f'{v:.3g}' for v in st['prof']]}", flush=True)
