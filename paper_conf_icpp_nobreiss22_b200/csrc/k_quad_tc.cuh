@@ -137,15 +137,22 @@ struct Geom {
     static_assert(ACC_COLS <= tc::SF_COL, "TMEM: accumulators overlap the scale factors");
     static_assert(YH % 2 == 0 && N % 16 == 0 && N <= 256, "two y per producer lane pair; cta_group::2 N");
 };
-// ring depths SA, SB, SA_F, SB_F (measured, profiles/r02f_variants.log; overridable for diagnostics builds)
-#ifndef EPI4_RINGS_N128
-#define EPI4_RINGS_N128 4, 4, 2, 2
+// ring depths SA x SB, fallback SA_F x SB_F (measured, profiles/r02f_variants.log; overridable for diagnostics
+// builds: nvcc splits -D values at commas, so one macro each)
+#ifndef EPI4_SA_N128
+#define EPI4_SA_N128 4
+#define EPI4_SB_N128 4
+#define EPI4_SAF_N128 2
+#define EPI4_SBF_N128 2
 #endif
-#ifndef EPI4_RINGS_N224
-#define EPI4_RINGS_N224 4, 8, 4, 4
+#ifndef EPI4_SA_N224
+#define EPI4_SA_N224 4
+#define EPI4_SB_N224 8
+#define EPI4_SAF_N224 4
+#define EPI4_SBF_N224 4
 #endif
-using Geom128 = Geom<EPI4_YR_N128, EPI4_CH_N128, 3, EPI4_RINGS_N128>;
-using Geom224 = Geom<EPI4_YR_N224, EPI4_CH_N224, 2, EPI4_RINGS_N224>;
+using Geom128 = Geom<EPI4_YR_N128, EPI4_CH_N128, 3, EPI4_SA_N128, EPI4_SB_N128, EPI4_SAF_N128, EPI4_SBF_N128>;
+using Geom224 = Geom<EPI4_YR_N224, EPI4_CH_N224, 2, EPI4_SA_N224, EPI4_SB_N224, EPI4_SAF_N224, EPI4_SBF_N224>;
 
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
