@@ -15,6 +15,18 @@
 #include <vector>
 
 #include "epi4_internal.cuh"
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX v3: host-side phase ranges (ncu --nvtx / Nsight timelines)
+
+namespace {
+// one NVTX range per phase of a call: load (pack / retile, tables), search (plan, slab rebuilds, contraction,
+// merge), third-order search
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
+}  // namespace
 
 using namespace epi4;
 
@@ -147,9 +159,11 @@ namespace {
 // remainder) and E(M) bounds ln2 |A - A_exact| from fp32 arithmetic (A in log2 units).  Over a quad's 243
 // terms, sum (k + 1/2) <= 2M + 203 and every argument is <= M + 2:
 //   lg2.approx: absolute error <= 2^-21 max(1, log2(M + 2)), times the coefficient (k + 1/2);
-//   accumulation: every cell adds its three terms to one of three running sums by FFMA (243 roundings); a
+//   accumulation: every cell adds its three terms to one of two running sums by FFMA (the lanes of an FFMA2
+//   pair, epilogue.cuh cell_T_acc2; 243 roundings); a
 //   running sum is at most P = M + 81 (log2(M + 2) + 2) between cells and at most P + (n + 3/2) log2(M + 2)
-//   inside a cell, so the roundings total <= u (243 P + 3 (M + 122) log2(M + 2)); + 2 final adds of <= P.
+//   inside a cell, so the roundings total <= u (243 P + 3 (M + 122) log2(M + 2)); + 1 final add of <= P (the
+//   bound below keeps 2).
 // E is doubled for safety; at M = 16384 E ~ 0.6, at M = 100003 ~ 4.
 double filter_offset(int64_t m) {
     const double M = (double)m, u = std::ldexp(1.0, -24), l2M = std::log2(M + 2.0), ln2 = std::log(2.0);
@@ -408,6 +422,7 @@ size_t t3_slab_bytes(int64_t n) { return (size_t)EPI4_WP * (size_t)c2(n) * 8 * s
 // once.  slab_w0 < 0: all w-ranges, resident colex layout; else only the w-range starting at slab_w0, written
 // as the slab FIRST([slab_w0, slab_w0 + 128)) (DevData t3_win).
 int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) {
+    NvtxRange nvtx_range("epi4: T3 on the tensor cores");
     const int32_t n = c->n;
     // the tile list depends only on (N, slab): the resident list is kept on the device across loads of the same N
     const int64_t key = ((int64_t)n * 2 + (slab_w0 >= 0 ? 1 : 0)) * 64 + c->tc_yr;
@@ -457,6 +472,7 @@ int build_t3_tc(epi4_ctx* c, uint32_t* out, int32_t slab_w0, int64_t* launches) 
 // pack / retile kernels set (invalid genotype codes, pad bits, AA & Aa), so a bad dataset is still rejected by
 // the load call itself.
 int finish_load(epi4_ctx* c) {
+    NvtxRange nvtx_range("epi4: load tables T1/T2/T3");
     // lower-order tables: packed (control | case << pk_shift) words, epilogue.cuh
     {
         // counts become fp32 values 2^23 + r in the filters and pack passes: each class below 2^23 samples
@@ -481,16 +497,22 @@ int finish_load(epi4_ctx* c) {
     // windowed T3 (tensor-core pipe): when the resident table does not fit, or on request
     c->t3_windowed = c->opts.pipe == EPI4_PIPE_TC && !shard && n >= 3 &&
                      ((c->opts.flags & EPI4_FLAG_T3_WINDOWED) ||
-                      (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3));
+                      (t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3 + c->cap_T3x));
     if (c->t3_windowed) {
         const size_t slab = t3_slab_bytes(n) * (pw / 4);
         CU(grow(c->T3, c->cap_T3, slab));
         CU(grow(c->T3x, c->cap_T3x, slab));
     }
-    if (!c->t3_windowed && t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3)
+    if (!c->t3_windowed && t3b > c->cap_T3 && t3b + ((size_t)1 << 30) > freeb + c->cap_T3 + c->cap_T3x)
         return fail(EPI4_ENOMEM, "3-way tables need %.1f GB but only %.1f GB of HBM are free (N=%d); "
                     "the windowed T3 needs the tensor-core pipe without sharding", t3b / 1e9, freeb / 1e9, c->n);
-    if (!c->t3_windowed) CU(grow(c->T3, c->cap_T3, t3b));
+    if (!c->t3_windowed) {
+        if (c->T3x) {                  // a previous windowed load's FIRST(X) slab: not needed with a resident table
+            dfree(c->T3x);
+            c->cap_T3x = 0;
+        }
+        CU(grow(c->T3, c->cap_T3, t3b));
+    }
     // lgamma table L[k] = lgamma(k + 1) for k in [0, M + 1]
     const int64_t m = c->np[0] + c->np[1];
     std::vector<double>& L = c->host_L;
@@ -716,6 +738,7 @@ int epi4_set_stream(epi4_ctx* c, void* s) {
 
 int epi4_load_bits(epi4_ctx* c, const uint32_t* pc, const uint32_t* pk, int32_t n_snps, int64_t n0, int64_t n1,
                    int32_t ptr_kind) {
+    NvtxRange nvtx_range("epi4_load_bits");
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     c->loaded = false;                    // a rejected load never leaves the previous dataset searchable
     c->t3_pending = false;
@@ -751,6 +774,7 @@ int epi4_load_bits(epi4_ctx* c, const uint32_t* pc, const uint32_t* pk, int32_t 
 
 int epi4_pack_genotypes(epi4_ctx* c, const uint8_t* geno, const uint8_t* phen, int32_t n_snps, int64_t m,
                         int32_t ptr_kind) {
+    NvtxRange nvtx_range("epi4_pack_genotypes");
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     c->loaded = false;                    // a rejected load never leaves the previous dataset searchable
     c->t3_pending = false;
@@ -904,6 +928,7 @@ int epi4_plan_units(int32_t n_snps, int32_t rank, int32_t world, int32_t* out, d
 
 int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64_t* quads_out, double* k2_out,
                       int32_t* n_out) {
+    NvtxRange nvtx_range("epi4_search");
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
     if (c->t3_pending) return fail(EPI4_ESTATE, "sharded T3 incomplete: all-gather the shares, then epi4_t3_ready");
@@ -1030,6 +1055,7 @@ int epi4_search_units(epi4_ctx* c, int64_t ub, int64_t ue, int32_t top_k, uint64
 }
 
 int epi4_search3(epi4_ctx* c, int32_t top_k, uint64_t* triples_out, double* k2_out, int32_t* n_out) {
+    NvtxRange nvtx_range("epi4_search3");
     if (!c) return fail(EPI4_EINVAL, "ctx is NULL");
     if (!c->loaded) return fail(EPI4_ESTATE, "search before any load");
     if (c->opts.pipe != EPI4_PIPE_TC) return fail(EPI4_EINVAL, "the third-order search runs on the tensor-core pipe");

@@ -204,8 +204,8 @@ __device__ __forceinline__ void cnt_f(P v, uint32_t pks, uint32_t pkm, float& m0
 // K2 - (ln2 sum T_c - 81 - 81 C0) lies in (-13.5, 3.375).  With the fp32 rounding bound E(M) computed on the
 // host (api.cu: filter_offset), K2 > ln2 A - 81 - 81 C0 - 13.5 - E for the computed A = sum T_c, so a quad is
 // scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
-// is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + 3 FFMA into one of three
-// running sums, 3 MUFU;
+// is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + 3 FFMA into a running sum, 3 MUFU
+// (the search uses the paired form cell_T_acc2 below: two running sums in the lanes of an fp32 pair);
 // no table and no conversion instruction (a count r < 2^23 becomes the float 2^23 + r by setting the exponent
 // bits).
 __device__ __forceinline__ float lg2_approx(float x) {
@@ -223,6 +223,55 @@ __device__ __forceinline__ void cell_T_acc(P v, uint32_t pks, uint32_t pkm, floa
     acc = fmaf(hn, lg2_approx(fn), acc);   // the cell's three terms go straight into the running sum
     acc = fmaf(-h0, lg2_approx(f0), acc);  // (rounding bound: api.cu filter_offset)
     acc = fmaf(-h1, lg2_approx(f1), acc);
+}
+
+// The same cell terms for two cells at once with sm_100's packed fp32 pairs (FADD2 / FFMA2: two IEEE
+// round-to-nearest operations per instruction, lane-wise identical to the scalar ones): cell a goes to lane 0 and
+// cell b to lane 1 of the running pair acc2, each lane adding its cell's three terms in the scalar order above,
+// so the rounding bound (api.cu filter_offset: every rounding <= u times a partial sum of cell terms) is unchanged.
+// Per two cells: 4 PRMT, 6 FADD2, 6 MUFU, 3 FFMA2 (19 instructions instead of 28).
+__device__ __forceinline__ uint64_t f2_pack(float lo, float hi) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+    return r;
+}
+__device__ __forceinline__ void f2_unpack(uint64_t v, float& lo, float& hi) {
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
+}
+__device__ __forceinline__ uint64_t f2_add(uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ uint64_t f2_sub(uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ uint64_t f2_fma(uint64_t a, uint64_t b, uint64_t c) {
+    uint64_t r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
+__device__ __forceinline__ uint64_t f2_lg2(uint64_t v) {
+    float lo, hi;
+    f2_unpack(v, lo, hi);
+    return f2_pack(lg2_approx(lo), lg2_approx(hi));
+}
+template <bool PK16, typename P>
+__device__ __forceinline__ void cell_T_acc2(P va, P vb, uint32_t pks, uint32_t pkm, uint64_t& acc2) {
+    float a0, a1, b0, b1;
+    cnt_f<PK16>(va, pks, pkm, a0, a1);
+    cnt_f<PK16>(vb, pks, pkm, b0, b1);
+    const uint64_t m0 = f2_pack(a0, b0), m1 = f2_pack(a1, b1);            // 2^23 + r0, 2^23 + r1 of both cells
+    const uint64_t c1 = f2_pack(8388607.0f, 8388607.0f), ch = f2_pack(8388607.5f, 8388607.5f);
+    const uint64_t f0 = f2_sub(m0, c1), f1 = f2_sub(m1, c1);             // r + 1
+    const uint64_t nh0 = f2_sub(ch, m0), nh1 = f2_sub(ch, m1);           // -(r + 1/2), exact
+    const uint64_t fn = f2_add(f0, f1);                                   // n + 2
+    const uint64_t hn = f2_sub(f1, nh0);                                  // n + 3/2 = (r0 + 1/2) + (r1 + 1)
+    acc2 = f2_fma(hn, f2_lg2(fn), acc2);
+    acc2 = f2_fma(nh0, f2_lg2(f0), acc2);
+    acc2 = f2_fma(nh1, f2_lg2(f1), acc2);
 }
 
 // ---- the fp32 chi-square filter (EPI4_OBJ_CHI2) ---------------------------------------------------------
@@ -282,13 +331,20 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
     const Q4<P> pwx = t2_all<P>(d, q.wx), pwy = t2_all<P>(d, q.wy), pwz = t2_all<P>(d, q.wz);
     const Q2<P> sw = t1_all<P>(d, w);
     float fa = 0.0f, fb = 0.0f, fc = 0.0f;
+    uint64_t acc2 = 0;   // MODE 0: two running sums (+0.0f, +0.0f) in the lanes of an fp32 pair
     double kk = 0.0;
     auto consume = [&](const P (&S)[27], int base) {
+        if constexpr (MODE == 0) {   // cells 2j, 2j+1 of the slab as a pair, cell 26 into lane 0 (scalar)
+#pragma unroll
+            for (int c = 0; c + 1 < 27; c += 2) cell_T_acc2<PK16>(S[c], S[c + 1], pks, pkm, acc2);
+            float lo, hi;
+            f2_unpack(acc2, lo, hi);
+            cell_T_acc<PK16>(S[26], pks, pkm, lo);
+            acc2 = f2_pack(lo, hi);
+        } else {
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
-            if (MODE == 0) {
-                cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
-            } else if (MODE == 6) {
+            if (MODE == 6) {
                 cell_mi_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
             } else if (MODE == 5) {
                 cell_chi_acc<PK16>(S[c], pks, pkm, d.chi_a, d.chi_b, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
@@ -315,6 +371,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
                 }
             }
         }
+        }
     };
     P R2[27];
     fill_slab_star<P>(R2, txyz0, txyz1, pxy, pxz, pyz, sx, sy, sz, npk_of<P>(d));
@@ -336,7 +393,13 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) R2[c] -= S[c];
     }
     consume(R2, 54);
-    flt = fa + fb + fc;
+    if (MODE == 0) {
+        float lo, hi;
+        f2_unpack(acc2, lo, hi);
+        flt = lo + hi;
+    } else {
+        flt = fa + fb + fc;
+    }
     if (MODE == 4) {   // chi-square: X^2 = M S / (n0 n1) - M (0 with an empty phenotype); key = -X^2
         const double n0 = __uint2double_rn(d.np[0]), n1 = __uint2double_rn(d.np[1]), M = __dadd_rn(n0, n1);
         k2 = (d.np[0] == 0 || d.np[1] == 0) ? 0.0 : -__dsub_rn(__ddiv_rn(__dmul_rn(M, kk), __dmul_rn(n0, n1)), M);
@@ -478,6 +541,8 @@ struct TopKSmem {
     int* cnt;
     int* lock;
     double* thr;         // k2 of the last entry when full, +inf otherwise (monotone non-increasing)
+    double* stage_k;     // [8][WL_MAX] staging of the per-warp register lists (wl_merge_store)
+    uint64_t* stage_i;
     int cap;
 };
 
@@ -539,6 +604,77 @@ __device__ __forceinline__ void warp_offer(TopKSmem& tk, bool has, double key, u
     if (lane == 0) atomicExch(tk.lock, 0);
 }
 
+// (4b) race-free alternative for top_k <= 32 (the tensor-core kernel's default): every warp keeps its own sorted
+// list in registers, lane j holding the j-th smallest (K2, index) key of the warp (empty = +inf / ~0); no state
+// is shared between warps, so no lock.  At the end of the kernel the warps stage their lists in shared memory,
+// meet at a named barrier, and one warp merges them into the CTA's list (wl_merge_store).
+constexpr int WL_MAX = 32;
+struct WarpList {
+    double k;
+    uint64_t i;
+};
+__device__ __forceinline__ void wl_init(WarpList& L) {
+    L.k = __longlong_as_double(0x7ff0000000000000LL);
+    L.i = ~0ull;
+}
+// the key of entry cap - 1 (+inf while the list has fewer than cap entries); uniform across the warp
+__device__ __forceinline__ double wl_thr(const WarpList& L, int cap) { return __shfl_sync(0xffffffffu, L.k, cap - 1); }
+// insert one key (all 32 lanes, uniform kk / ii); entries past cap are kept sorted but never read
+__device__ __forceinline__ void wl_insert(WarpList& L, int cap, double kk, uint64_t ii) {
+    const int lane = threadIdx.x & 31;
+    const int pos = __popc(__ballot_sync(0xffffffffu, key_less(L.k, L.i, kk, ii)));
+    if (pos >= cap) return;
+    const double uk = __shfl_up_sync(0xffffffffu, L.k, 1);
+    const uint64_t ui = __shfl_up_sync(0xffffffffu, L.i, 1);
+    if (lane > pos) { L.k = uk; L.i = ui; }
+    else if (lane == pos) { L.k = kk; L.i = ii; }
+}
+// offer one key per lane (has = false lanes offer nothing); thr is updated to the list's new threshold
+__device__ __forceinline__ void wl_offer(WarpList& L, int cap, double& thr, bool has, double key, uint64_t idx) {
+    unsigned m = __ballot_sync(0xffffffffu, has && key <= thr);
+    if (!m) return;
+    while (m) {
+        const int src = __ffs(m) - 1;
+        m &= m - 1;
+        wl_insert(L, cap, __shfl_sync(0xffffffffu, key, src), __shfl_sync(0xffffffffu, idx, src));
+    }
+    thr = wl_thr(L, cap);
+}
+// the CTA's list of a previous launch (global slot `slot`) into warp list L (call with one warp)
+__device__ __forceinline__ void wl_load(WarpList& L, const SearchParams& sp, int slot) {
+    const int lane = threadIdx.x & 31, cnt = sp.list_cnt[slot];
+    wl_init(L);
+    if (lane < cnt) {
+        L.k = sp.list_k2[(int64_t)slot * sp.topk + lane];
+        L.i = sp.list_idx[(int64_t)slot * sp.topk + lane];
+    }
+}
+// nw warps (ids ew = 0..nw-1, named barrier `bar` over their 32 nw threads) fold their lists into the CTA's global
+// slot: staging area stage[nw][32] in shared memory, then warp 0 merges (every staged key through wl_insert)
+__device__ __forceinline__ void wl_merge_store(const WarpList& L, int cap, int ew, int nw, int bar, double* stage_k,
+                                               uint64_t* stage_i, const SearchParams& sp, int slot) {
+    const int lane = threadIdx.x & 31;
+    stage_k[ew * WL_MAX + lane] = L.k;
+    stage_i[ew * WL_MAX + lane] = L.i;
+    asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(32 * nw) : "memory");
+    if (ew != 0) return;
+    WarpList R;
+    wl_init(R);
+    for (int w = 0; w < nw; ++w)
+        for (int j = 0; j < cap; ++j) {
+            const double kk = stage_k[w * WL_MAX + j];
+            if (!(kk < __longlong_as_double(0x7ff0000000000000LL))) break;   // the rest of this list is empty
+            wl_insert(R, cap, kk, stage_i[w * WL_MAX + j]);
+        }
+    const bool full = lane < cap && R.k < __longlong_as_double(0x7ff0000000000000LL);
+    if (full) {
+        sp.list_k2[(int64_t)slot * sp.topk + lane] = R.k;
+        sp.list_idx[(int64_t)slot * sp.topk + lane] = R.i;
+    }
+    const int cnt = __popc(__ballot_sync(0xffffffffu, full));
+    if (lane == 0) sp.list_cnt[slot] = cnt;
+}
+
 // carve the top-k state from dynamic shared memory (8-byte aligned base)
 __device__ __forceinline__ TopKSmem topk_carve(unsigned char* base, int cap) {
     TopKSmem tk;
@@ -547,10 +683,12 @@ __device__ __forceinline__ TopKSmem topk_carve(unsigned char* base, int cap) {
     tk.thr = reinterpret_cast<double*>(base + 16 * cap);
     tk.cnt = reinterpret_cast<int*>(base + 16 * cap + 8);
     tk.lock = reinterpret_cast<int*>(base + 16 * cap + 12);
+    tk.stage_k = reinterpret_cast<double*>(base + 16 * cap + 16);
+    tk.stage_i = reinterpret_cast<uint64_t*>(base + 16 * cap + 16 + 8 * 32 * sizeof(double));
     tk.cap = cap;
     return tk;
 }
-__host__ __device__ constexpr size_t topk_smem_bytes(int cap) { return 16 * (size_t)cap + 16; }
+__host__ __device__ constexpr size_t topk_smem_bytes(int cap) { return 16 * (size_t)cap + 16 + 8 * 32 * 16; }
 
 // load this CTA's list from its global slot (call with all threads, followed by a barrier)
 __device__ __forceinline__ void topk_load(TopKSmem& tk, const SearchParams& sp, int slot, int tid, int nthr) {

@@ -28,6 +28,12 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
     __syncthreads();
     const DevData& d = sp.d;
     unsigned long long my_quads = 0;
+    // top_k <= 32: race-free per-warp register lists (epilogue.cuh WarpList), else the CTA's locked list
+    const bool wlist = sp.topk <= WL_MAX;
+    WarpList wlst;
+    wl_init(wlst);
+    if (wlist && tid < 32) wl_load(wlst, sp, blockIdx.x);
+    double wthr = wlist ? wl_thr(wlst, sp.topk) : 0.0;
 
     for (;;) {
         if (tid == 0) s_tile = (long long)atomicAdd(sp.tile_counter, 1ull);
@@ -123,11 +129,13 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
                 idx = pack_quad(w, x, y, z);
                 ++my_quads;
             }
-            warp_offer(tk, valid, key, idx);
+            if (wlist) wl_offer(wlst, sp.topk, wthr, valid, key, idx);
+            else warp_offer(tk, valid, key, idx);
         }
     }
     __syncthreads();
-    topk_store(tk, sp, blockIdx.x, tid, LOP3_THREADS);
+    if (wlist) wl_merge_store(wlst, sp.topk, tid >> 5, LOP3_THREADS / 32, 1, tk.stage_k, tk.stage_i, sp, blockIdx.x);
+    else topk_store(tk, sp, blockIdx.x, tid, LOP3_THREADS);
     // useful-quad counter
     unsigned long long v = my_quads;
 #pragma unroll

@@ -732,6 +732,12 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         int it = 0;
         const uint32_t pks = (uint32_t)d.pk_shift;
         int r0 = 0;                                     // the MMA issuers' region rotation
+        // top_k <= 32: a race-free list per warp in registers (epilogue.cuh WarpList); else the CTA's locked list
+        const bool wlist = sp.topk <= WL_MAX && !sp.t3_out;
+        WarpList wlst;
+        wl_init(wlst);
+        if (wlist && ew == 0) wl_load(wlst, sp, blockIdx.x);   // the CTA's keys from the previous launches
+        double wthr = wlist ? wl_thr(wlst, sp.topk) : 0.0;
         for (int64_t tile = first_tile; tile < sp.ntiles; tile += tile_stride, ++it) {
             const TileInfo ti = load_tile(sp, tile);
             const int buf = it & 1;
@@ -833,7 +839,8 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         idx3 = pack_quad(w, ti.x, y, 0);
                         ++my_quads;
                     }
-                    warp_offer(tk, v3, key3, idx3);
+                    if (wlist) wl_offer(wlst, sp.topk, wthr, v3, key3, idx3);
+                    else warp_offer(tk, v3, key3, idx3);
                     continue;
                 }
                 const bool valid = (w < ti.x) && (y < ti.z) && score;
@@ -856,7 +863,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                         double unused;
                         quad_eval<FILT == 1 ? 5 : FILT == 2 ? 6 : 0, PK16, P>(d, quad_ranks(d, w, ti.x, y, ti.z), w, ti.x, y,
                                                                               ti.z, c16, flt, unused, nullptr);
-                        const double thr = *reinterpret_cast<volatile double*>(tk.thr);
+                        const double thr = wlist ? wthr : *reinterpret_cast<volatile double*>(tk.thr);
                         if (FILT == 1)
                             offer = d.chi_M - (double)flt * (1.0 + 1.0 / 4096.0) <= thr;
                         else if (FILT == 2)
@@ -874,11 +881,14 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                     idx = pack_quad(w, ti.x, y, ti.z);
                     ++my_quads;
                 }
-                warp_offer(tk, offer, key, idx);
+                if (wlist) wl_offer(wlst, sp.topk, wthr, offer, key, idx);
+                else warp_offer(tk, offer, key, idx);
             }
             t_busy += PCLK() - t1;
             if (G::REGIONS == 3) r0 = r0 == 0 ? 2 : r0 - 1;
         }
+        // fold the 8 warp lists into the CTA's global slot (named barrier 1 over the epilogue warps)
+        if (wlist) wl_merge_store(wlst, sp.topk, ew, tc::EPI_WARPS, 1, tk.stage_k, tk.stage_i, sp, blockIdx.x);
         unsigned long long v = my_quads, ne = n_exact;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
@@ -899,7 +909,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     tc_fence_after();
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tc::TMEM_COLS));
-    if (!sp.t3_out) topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
+    if (!sp.t3_out && sp.topk > WL_MAX) topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
 #if EPI4_PROF
     if (tracing && tid == 0) {
         for (int k = 0; k < TR_STEPS; ++k)

@@ -91,3 +91,20 @@ def test_multirank_path_on_one_gpu():
                        capture_output=True, text=True, timeout=600, cwd=root)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
     assert "OK" in r.stdout
+
+
+def test_multirank_nccl_on_two_gpus():
+    """The same flow over NCCL with one rank per GPU (device-tensor all_gather of the T3 shares and of the top-k
+    lists): needs >= 2 visible GPUs, skipped on a one-GPU box."""
+    import os
+    import subprocess
+    import sys
+    import torch
+    if torch.cuda.device_count() < 2:
+        pytest.skip("needs 2 GPUs (one rank per GPU over NCCL)")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--standalone", "--nproc-per-node", "2",
+                        os.path.join(root, "tools", "multirank_one_gpu.py"), "--backend", "nccl", "--n-snps", "160"],
+                       capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    assert "OK" in r.stdout
