@@ -225,6 +225,9 @@ __device__ __forceinline__ void cell_T_acc(P v, uint32_t pks, uint32_t pkm, floa
     acc = fmaf(-h1, lg2_approx(f1), acc);
 }
 
+#ifndef EPI4_FILTER_F2
+#define EPI4_FILTER_F2 0    // 1: the paired FFMA2 filter below (fewer instructions, measured 1.5 % slower at C2, profiles/r02l_topk.log)
+#endif
 // The same cell terms for two cells at once with sm_100's packed fp32 pairs (FADD2 / FFMA2: two IEEE
 // round-to-nearest operations per instruction, lane-wise identical to the scalar ones): cell a goes to lane 0 and
 // cell b to lane 1 of the running pair acc2, each lane adding its cell's three terms in the scalar order above,
@@ -334,7 +337,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
     uint64_t acc2 = 0;   // MODE 0: two running sums (+0.0f, +0.0f) in the lanes of an fp32 pair
     double kk = 0.0;
     auto consume = [&](const P (&S)[27], int base) {
-        if constexpr (MODE == 0) {   // cells 2j, 2j+1 of the slab as a pair, cell 26 into lane 0 (scalar)
+        if constexpr (MODE == 0 && EPI4_FILTER_F2) {   // cells 2j, 2j+1 of the slab as a pair, cell 26 into lane 0
 #pragma unroll
             for (int c = 0; c + 1 < 27; c += 2) cell_T_acc2<PK16>(S[c], S[c + 1], pks, pkm, acc2);
             float lo, hi;
@@ -344,7 +347,9 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         } else {
 #pragma unroll
         for (int c = 0; c < 27; ++c) {
-            if (MODE == 6) {
+            if (MODE == 0) {
+                cell_T_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
+            } else if (MODE == 6) {
                 cell_mi_acc<PK16>(S[c], pks, pkm, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
             } else if (MODE == 5) {
                 cell_chi_acc<PK16>(S[c], pks, pkm, d.chi_a, d.chi_b, c % 3 == 0 ? fa : c % 3 == 1 ? fb : fc);
@@ -393,7 +398,7 @@ __device__ __forceinline__ void quad_eval(const DevData& d, const QuadRanks& q, 
         for (int c = 0; c < 27; ++c) R2[c] -= S[c];
     }
     consume(R2, 54);
-    if (MODE == 0) {
+    if (MODE == 0 && EPI4_FILTER_F2) {
         float lo, hi;
         f2_unpack(acc2, lo, hi);
         flt = lo + hi;
@@ -609,6 +614,10 @@ __device__ __forceinline__ void warp_offer(TopKSmem& tk, bool has, double key, u
 // is shared between warps, so no lock.  At the end of the kernel the warps stage their lists in shared memory,
 // meet at a named barrier, and one warp merges them into the CTA's list (wl_merge_store).
 constexpr int WL_MAX = 32;
+#ifndef EPI4_WARP_LISTS
+#define EPI4_WARP_LISTS 0   // 1: per-warp register lists for top_k <= 32 (race-free; measured 1-2 % slower, profiles/r02l_topk.log)
+#endif
+__host__ __device__ constexpr bool use_warp_lists(int topk) { return EPI4_WARP_LISTS && topk <= WL_MAX; }
 struct WarpList {
     double k;
     uint64_t i;

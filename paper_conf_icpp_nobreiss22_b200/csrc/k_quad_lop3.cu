@@ -29,7 +29,7 @@ __global__ void __launch_bounds__(LOP3_THREADS, 1) k_quad_lop3(SearchParams sp) 
     const DevData& d = sp.d;
     unsigned long long my_quads = 0;
     // top_k <= 32: race-free per-warp register lists (epilogue.cuh WarpList), else the CTA's locked list
-    const bool wlist = sp.topk <= WL_MAX;
+    const bool wlist = use_warp_lists(sp.topk);
     WarpList wlst;
     wl_init(wlst);
     if (wlist && tid < 32) wl_load(wlst, sp, blockIdx.x);

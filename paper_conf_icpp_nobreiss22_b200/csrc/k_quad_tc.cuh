@@ -733,7 +733,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
         const uint32_t pks = (uint32_t)d.pk_shift;
         int r0 = 0;                                     // the MMA issuers' region rotation
         // top_k <= 32: a race-free list per warp in registers (epilogue.cuh WarpList); else the CTA's locked list
-        const bool wlist = sp.topk <= WL_MAX && !sp.t3_out;
+        const bool wlist = use_warp_lists(sp.topk) && !sp.t3_out;
         WarpList wlst;
         wl_init(wlst);
         if (wlist && ew == 0) wl_load(wlst, sp, blockIdx.x);   // the CTA's keys from the previous launches
@@ -909,7 +909,7 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     tc_fence_after();
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tc::TMEM_COLS));
-    if (!sp.t3_out && sp.topk > WL_MAX) topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
+    if (!sp.t3_out && !use_warp_lists(sp.topk)) topk_store(tk, sp, blockIdx.x, tid, tc::THREADS);
 #if EPI4_PROF
     if (tracing && tid == 0) {
         for (int k = 0; k < TR_STEPS; ++k)
