@@ -159,11 +159,10 @@ namespace {
 // remainder) and E(M) bounds ln2 |A - A_exact| from fp32 arithmetic (A in log2 units).  Over a quad's 243
 // terms, sum (k + 1/2) <= 2M + 203 and every argument is <= M + 2:
 //   lg2.approx: absolute error <= 2^-21 max(1, log2(M + 2)), times the coefficient (k + 1/2);
-//   accumulation: every cell adds its three terms to one of two running sums by FFMA (the lanes of an FFMA2
-//   pair, epilogue.cuh cell_T_acc2; 243 roundings); a
+//   accumulation: every cell adds its three terms to one of three running sums by FFMA (or, with
+//   EPI4_FILTER_F2, one of the two lanes of an FFMA2 pair, epilogue.cuh cell_T_acc2; 243 roundings either way); a
 //   running sum is at most P = M + 81 (log2(M + 2) + 2) between cells and at most P + (n + 3/2) log2(M + 2)
-//   inside a cell, so the roundings total <= u (243 P + 3 (M + 122) log2(M + 2)); + 1 final add of <= P (the
-//   bound below keeps 2).
+//   inside a cell, so the roundings total <= u (243 P + 3 (M + 122) log2(M + 2)); + 2 final adds of <= P.
 // E is doubled for safety; at M = 16384 E ~ 0.6, at M = 100003 ~ 4.
 double filter_offset(int64_t m) {
     const double M = (double)m, u = std::ldexp(1.0, -24), l2M = std::log2(M + 2.0), ln2 = std::log(2.0);

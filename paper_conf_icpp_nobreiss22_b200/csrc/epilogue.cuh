@@ -205,7 +205,7 @@ __device__ __forceinline__ void cnt_f(P v, uint32_t pks, uint32_t pkm, float& m0
 // host (api.cu: filter_offset), K2 > ln2 A - 81 - 81 C0 - 13.5 - E for the computed A = sum T_c, so a quad is
 // scored exactly (double, lgamma table) only if ln2 A + flt_off <= the CTA's current k-th best K2: the top-k
 // is exactly the oracle's.  Per cell: 3 ALU (unpack; 2 with pks = 16), 6 FADD + 3 FFMA into a running sum, 3 MUFU
-// (the search uses the paired form cell_T_acc2 below: two running sums in the lanes of an fp32 pair);
+// (with EPI4_FILTER_F2 the paired form cell_T_acc2 below: two running sums in the lanes of an fp32 pair);
 // no table and no conversion instruction (a count r < 2^23 becomes the float 2^23 + r by setting the exponent
 // bits).
 __device__ __forceinline__ float lg2_approx(float x) {

@@ -113,7 +113,8 @@ constexpr int CLUSTER = 2;
 //     third region, so the controls of tile t+1 start once the pack pass has emptied region 0 and its cases
 //     once the scoring of tile t has read region 1 — hidden when the first (larger) phenotype phase is longer
 //     than the scoring, i.e. at large sample counts (selected by the load, api.cu tc_tile_yr).
-template <int YR_, int CHUNKS_, int REGIONS_, int SA_, int SB_, int SAF_, int SBF_>
+template <int YR_, int CHUNKS_, int REGIONS_, int SA_, int SB_, int SAF_, int SBF_, bool LATE_ = false,
+          int RCTL_ = tc::REGS_CTL, int RPROD_ = tc::REGS_PROD>
 struct Geom {
     static constexpr int YR = YR_, N = 8 * YR_;                // UMMA N
     static constexpr int CHUNKS = CHUNKS_;                     // fp4 chunks per pipeline stage
@@ -128,6 +129,11 @@ struct Geom {
     static constexpr int ACC_COLS = REGIONS * N;
     static constexpr int NG = N / 16;                          // 16-column groups of an accumulator
     static constexpr int SA = SA_, SB = SB_, SA_F = SAF_, SB_F = SBF_;
+    // LATE: a producer issues the loads of its next step's singles after building (and publishing) this one, so
+    // the two register sets do not overlap (with 28 y per tile the overlapping sets spill at 120 registers)
+    static constexpr bool LATE = LATE_;
+    static constexpr int REGS_CTL = RCTL_, REGS_PROD = RPROD_;                  // setmaxnreg per warpgroup
+    static constexpr int REGS_EPI = ((65536 / 128 - REGS_CTL - REGS_PROD) / 2) / 8 * 8;
     // block-scaled instruction descriptor: A/B E2M1 (format 1 at bits 7 and 10), K-major, N>>3 at bit 17,
     // scale format E8M0 (bit 23), M>>4 at bit 24, scale-factor ids 0, K = 64 (bit 31 = 0)
     static constexpr uint32_t IDESC =
@@ -151,8 +157,20 @@ struct Geom {
 #define EPI4_SAF_N224 4
 #define EPI4_SBF_N224 4
 #endif
-using Geom128 = Geom<EPI4_YR_N128, EPI4_CH_N128, 3, EPI4_SA_N128, EPI4_SB_N128, EPI4_SAF_N128, EPI4_SBF_N128>;
-using Geom224 = Geom<EPI4_YR_N224, EPI4_CH_N224, 2, EPI4_SA_N224, EPI4_SB_N224, EPI4_SAF_N224, EPI4_SBF_N224>;
+#ifndef EPI4_LATE_N224
+#define EPI4_LATE_N224 0
+#endif
+#ifndef EPI4_RCTL_N224
+#define EPI4_RCTL_N224 40
+#define EPI4_RPROD_N224 120
+#endif
+#ifndef EPI4_LATE_N128
+#define EPI4_LATE_N128 0
+#endif
+using Geom128 = Geom<EPI4_YR_N128, EPI4_CH_N128, 3, EPI4_SA_N128, EPI4_SB_N128, EPI4_SAF_N128, EPI4_SBF_N128,
+                     EPI4_LATE_N128>;
+using Geom224 = Geom<EPI4_YR_N224, EPI4_CH_N224, 2, EPI4_SA_N224, EPI4_SB_N224, EPI4_SAF_N224, EPI4_SBF_N224,
+                     EPI4_LATE_N224, EPI4_RCTL_N224, EPI4_RPROD_N224>;
 
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -479,9 +497,9 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
     // need few registers; the epilogue warpgroups take the rest (EPI4_REGS_EPI) so the per-quad evaluation
     // runs without spills and with more loads in flight.
     if (tc::REGSPLIT) {
-        if (rw < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_CTL));
-        else if (rw < 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(tc::REGS_PROD));
-        else asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(tc::REGS_EPI));
+        if (rw < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(G::REGS_CTL));
+        else if (rw < 8) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(G::REGS_PROD));
+        else asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(G::REGS_EPI));
     }
     if (rw < tc::MMA_WARPS) {
         // ===================== MMA issuers (leader CTA) =====================
@@ -669,8 +687,10 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
             for (int k = 0; k < 4; ++k) cx[k] = nx[k];
 #pragma unroll
             for (int k = 0; k < YK; ++k) cy[k] = ny[k];
-            load(pre);                                            // next own step's singles (in flight)
-            pre.advance(sp, G::PROD_STRIDE);
+            if (!G::LATE) {
+                load(pre);                                        // next own step's singles (in flight)
+                pre.advance(sp, G::PROD_STRIDE);
+            }
             const long long t0 = PCLK();
             mbar_wait(&bempty_bar[sb], (uint32_t)((step / SB) & 1) ^ 1u);   // B slot free (MMA of step - SB done)
             const long long t1 = PCLK();
@@ -704,6 +724,10 @@ __global__ void __launch_bounds__(tc::THREADS, 1) k_quad_tc(SearchParams sp) {
                 TRACE(9, step);
             }
             __syncwarp();
+            if (G::LATE) {
+                load(pre);                                        // next own step's singles, after this one is out
+                pre.advance(sp, G::PROD_STRIDE);
+            }
             if (EPI4_PROF) {
                 const long long t3 = PCLK();
                 t_busy += t3 - t1;
