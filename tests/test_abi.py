@@ -100,3 +100,12 @@ def test_binding_constants_match_the_header():
                  "EPI4_EINVAL", "EPI4_ENODEV", "EPI4_PIPE_TC", "EPI4_PIPE_LOP3"):
         assert name in defs, name
         assert getattr(binding, name) == defs[name], name
+
+
+def test_tile_option_is_validated_before_any_device_call():
+    """Epi4(tile=...) accepts only None / 128 / 224 (EPI4_FLAG_TILE_*); anything else fails in the binding,
+    before a context is created."""
+    import pytest
+    import paper_conf_icpp_nobreiss22_b200 as epi
+    with pytest.raises(ValueError):
+        epi.Epi4(0, tile=160)
