@@ -1,5 +1,9 @@
-# final round measurements: the standard round script + the driver's torchrun launch form at N=1
-bash tools/gpu_round.sh
-timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29511 \
-  bench.py --gpus 1 --steps 3 --warmup 3 --no-cpu-baseline > gpurun_out/bench_torchrun.json 2> gpurun_out/bench_torchrun.err
-tail -c 600 gpurun_out/bench_torchrun.json
+# End-of-round check of HEAD (run under gpurun): the GPU parity suite, smoke, and the bench line (ours + reference arm).
+# usage: bash tools/gpu_final.sh <tag>
+T=${1:-r02}
+mkdir -p gpurun_out
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit --format=csv
+timeout 1500 python -m pytest tests -m gpu -q -x --durations=10 2>&1 | tail -16 > gpurun_out/${T}_pytest_gpu.log; tail -3 gpurun_out/${T}_pytest_gpu.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -3 | tee gpurun_out/${T}_smoke.log
+timeout 1500 python bench.py --steps 5 --warmup 3 > gpurun_out/${T}_bench.json 2> gpurun_out/${T}_bench.err; tail -c 600 gpurun_out/${T}_bench.json
+timeout 900 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${T}_bench_ref.json 2>&1; tail -c 300 gpurun_out/${T}_bench_ref.json
