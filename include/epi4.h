@@ -68,7 +68,7 @@ typedef struct {
 #define EPI4_FLAG_T3_WINDOWED 2
 /* opts.flags: tensor-core tile geometry.  By default a load picks N = 224 columns per tile
  * (28 y SNPs; the A operand amortised over more columns, two TMEM accumulator regions) when the dataset has
- * >= 24576 controls or needs 64-bit packed counts, else N = 128 (16 y, three regions, the scoring overlaps
+ * >= 16384 controls or needs 64-bit packed counts, else N = 128 (16 y, three regions, the scoring overlaps
  * both phenotype phases); these flags force one (results are identical, only the speed differs). */
 #define EPI4_FLAG_TILE_N128 4
 #define EPI4_FLAG_TILE_N224 8

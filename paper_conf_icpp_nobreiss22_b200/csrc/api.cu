@@ -600,13 +600,13 @@ namespace {
 // Tensor-core tile geometry (k_quad_tc.cuh): N = 224 columns amortise the A operand over 1.75x the
 // columns but leave room for only two TMEM regions, so the scoring of a tile overlaps only the first (control)
 // phase of the next; N = 128 keeps three regions.  Measured on one B200 (profiles/r02f_variants.log,
-// r02g_geom_ab.log): N = 224 is 7 % faster on the full C5 search (70002 controls), within noise with 16384
-// controls (C3 sub-window) and 17 % slower with 8192 (C2).  The wide (64-bit packed) mode has two regions in
+// r02g_geom_ab.log, r02s_c3_geom.log): N = 224 is 7 % faster on the full C5 search (70002 controls), 4 % on the
+// full C3 search (16384 controls: 150.0 vs 156.2 s) and 17 % slower with 8192 (C2).  The wide (64-bit packed) mode has two regions in
 // both geometries.  opts.flags can force either.
 int32_t tc_tile_yr(int32_t flags, int64_t n0, int64_t n1) {
     if (flags & EPI4_FLAG_TILE_N224) return EPI4_YR_N224;
     if (flags & EPI4_FLAG_TILE_N128) return EPI4_YR_N128;
-    return (n0 >= 24576 || is_wide(n0, n1)) ? EPI4_YR_N224 : EPI4_YR_N128;
+    return (n0 >= 16384 || is_wide(n0, n1)) ? EPI4_YR_N224 : EPI4_YR_N128;
 }
 
 int alloc_planes(epi4_ctx* c, int32_t n, int64_t n0, int64_t n1) {
